@@ -1,0 +1,388 @@
+#!/usr/bin/env python
+"""bench.py — MEGA GAT layer fwd+bwd on B200 (BASELINE.json metric).
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl mega|reference]
+                  [--config products|reddit|arxiv|pubmed|cora] [--dtype bf16|fp32]
+
+One "step" = one pass of the whole hot path over the
+workload: every GAT layer of the config forward (projection on tensor cores,
+fused attention) then backward (attention backward, projection backward).
+`value` = layers * E / step time: GAT layer fwd+bwd edges per second, whole
+job.  Inputs are resident in HBM when the timed region starts; `e2e` repeats
+the measurement with the step's inputs copied from pinned host memory and the
+parameter gradients read back every step.  `--impl reference` times the CPU
+oracle (oracle/, the only other place bench.py runs it) on a bounded sample.
+Multi-GPU (torchrun, N > 1): destination partitions of the MEGA order, one per
+rank; see paper_conf_icdcs_dengr24_b200/dist.py.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "GAT layer fwd+bwd edges/sec and HBM GB/s fraction at 1/2/4/8 B200"
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="mega", choices=["mega", "reference"])
+    ap.add_argument("--config", default="products")
+    ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
+    ap.add_argument("--order", default="traversal")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    return ap.parse_args()
+
+
+# ------------------------------------------------------------------ helpers
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
+                                          "-i", str(self.index), "-lms", "100"], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        time.sleep(0.25)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def __exit__(self, *exc):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 4 + i and "Active" in r[4 + i]
+                          and "Not" not in r[4 + i]})
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return {"hbm_gbs": d["hbm_gbs"], "bf16_tflops": d.get("bf16_tflops_sustained", d["bf16_tflops"]),
+                "source": "measured (MEASURED_PEAKS.json)"}
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "source": "fallback (B200_PROFILING.md)"}
+
+
+def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
+    """Compulsory HBM bytes per launch of each library call:
+    every gathered row counted once (perfect on-chip reuse), per-edge streams once."""
+    rows = n if rows is None else rows
+    items = 16 * rows
+    if call == "gat_fwd":     # KB2 (+KB7): idx, items, Wh, er, el, out, lse
+        return 4 * m + items + n * D * sb + n * H * 4 + rows * H * 4 + rows * D * sb + rows * H * 4
+    if call == "gat_bwd_src":  # KB3 + KB4 (+merge): g,out -> Dlt; cdst, items, Wh, er, g_i, el/lse/Dlt, dz, dWh
+        return (2 * rows * D * sb + rows * H * 4) + (4 * m + 16 * n + n * D * sb + n * H * 4 + rows * D * sb
+                                                    + 3 * rows * H * 4 + 4 * m * H + n * D * 4)
+    if call == "gat_bwd_dst":  # KB5: indptr, csr2csc, dz, dWh RMW, Wh, bf16 copy
+        return 4 * (rows + 1) + 4 * m + 4 * m * H + 2 * rows * D * 4 + rows * D * sb + (rows * D * sb if sb == 2 else 0)
+    raise KeyError(call)
+
+
+# ------------------------------------------------------------------ workload
+def build_workload(cfg_name, dtype, order, rank=0, world=1):
+    import synth
+    cfg = synth.CONFIGS[cfg_name]
+    t0 = time.time()
+    indptr, indices, gstats = synth.make_graph(cfg)
+    t_gen = time.time() - t0
+    from paper_conf_icdcs_dengr24_b200 import mega as M
+    t0 = time.time()
+    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world)
+    t_pre = time.time() - t0
+    perm = layout.view(0)["perm"].astype(np.int64)
+    layers = []
+    in_dim = cfg.f_in
+    for li in range(cfg.layers):
+        inp = synth.make_layer_inputs(cfg, layer=li, in_dim=in_dim)
+        if dtype == "bf16":
+            inp["w"] = synth.bf16_round(inp["w"])
+        layers.append(inp)
+        in_dim = cfg.dim
+    x0 = layers[0]["x"][perm]
+    g_last = layers[-1]["grad_out"][perm]
+    if dtype == "bf16":
+        x0, g_last = synth.bf16_round(x0), synth.bf16_round(g_last)
+    return {"cfg": cfg, "indptr": indptr, "indices": indices, "layout": layout, "perm": perm, "layers": layers,
+            "x0": np.ascontiguousarray(x0), "g_last": np.ascontiguousarray(g_last), "gen_s": t_gen, "pre_s": t_pre,
+            "graph_stats": gstats}
+
+
+class Model:
+    """The config's GAT stack on one GPU, every step through libmega.so."""
+
+    def __init__(self, wl, dtype, dev):
+        import torch
+        from paper_conf_icdcs_dengr24_b200.layer import GATLayer
+        self.torch = torch
+        cfg = wl["cfg"]
+        tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
+        self.x0 = torch.tensor(wl["x0"], device=dev).to(tdt).contiguous()
+        self.g = torch.tensor(wl["g_last"], device=dev).to(tdt).contiguous()
+        wl["layout"].bind(0)
+        self.layers = []
+        x = self.x0
+        for li, inp in enumerate(wl["layers"]):
+            w = torch.tensor(inp["w"], device=dev).to(tdt).contiguous()
+            L = GATLayer(wl["layout"], x, w, torch.tensor(inp["a_l"], device=dev),
+                         torch.tensor(inp["a_r"], device=dev), cfg.heads, cfg.head_dim, in_dim=inp["in_dim"],
+                         want_grad_x=li > 0)
+            self.layers.append(L)
+            x = L.out
+        self.launches = sum(L.launches_per_step() for L in self.layers)
+
+    def step(self, ev=None):
+        """ev: optional dict name -> list of (start, end) event pairs to record into."""
+        torch = self.torch
+
+        def timed(name, fn):
+            if ev is None:
+                fn()
+                return
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record()
+            fn()
+            e.record()
+            ev.setdefault(name, []).append((s, e))
+
+        from paper_conf_icdcs_dengr24_b200 import mega as M
+        for L in self.layers:
+            timed("project_fwd", L.project)
+            timed("gat_fwd", lambda: L.attend(True))
+        g = self.g
+        for L in reversed(self.layers):
+            timed("gat_bwd_src", lambda: L.attend_backward(g, M.MEGA_BWD_PHASE_SRC))
+            timed("gat_bwd_dst", lambda: L.attend_backward(g, M.MEGA_BWD_PHASE_DST))
+            timed("project_bwd", L.project_backward)
+            g = L.grad_x
+
+
+# ------------------------------------------------------------------ CPU oracle
+def cpu_sample(wl, seconds_target, H, F):
+    """Bounded sample for the CPU oracle: the first R destination rows of the MEGA
+    order with all their in-edges (sources stay global), one GAT layer fwd+bwd."""
+    from oracle import coracle
+    ip = wl["layout"].view(0)
+    indptr_new = ip["indptr"].astype(np.int64)
+    src_new = ip["src"]
+    n = len(indptr_new) - 1
+    rng = np.random.default_rng(0)
+    import synth
+    Wh = synth.bf16_round(rng.standard_normal((n, H, F)).astype(np.float32))
+    g = synth.bf16_round(rng.standard_normal((n, H, F)).astype(np.float32))
+    a_l = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
+    a_r = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
+
+    def run(R):
+        sub_ptr = np.minimum(indptr_new, indptr_new[R])
+        sub_idx = src_new[:indptr_new[R]]
+        t0 = time.perf_counter()
+        f = coracle.gat_forward(sub_ptr, sub_idx, Wh, a_l, a_r)
+        coracle.gat_backward(sub_ptr, sub_idx, Wh, a_l, a_r, g, fwd=f)
+        return time.perf_counter() - t0, int(indptr_new[R])
+
+    R = max(1, min(n, int(np.searchsorted(indptr_new, 200000))))
+    t, e = run(R)
+    if t < seconds_target / 3 and R < n:
+        scale = seconds_target / max(t, 1e-3)
+        R = max(R + 1, min(n, int(np.searchsorted(indptr_new, min(wl["cfg"].m, int(e * scale))))))
+    return run, R
+
+
+def cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except AttributeError:
+        return os.cpu_count()
+
+
+# ------------------------------------------------------------------ main paths
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    wl = build_workload(args.config, args.dtype, args.order)
+    cfg = wl["cfg"]
+    per_step = max(2.0, min(10.0, 150.0 / max(1, args.steps + args.warmup)))
+    run, R = cpu_sample(wl, per_step, cfg.heads, cfg.head_dim)
+    for _ in range(args.warmup):
+        run(R)
+    times, edges = [], 0
+    for _ in range(args.steps):
+        t, e = run(R)
+        times.append(t)
+        edges = e
+    tot = float(np.sum(times))
+    value = edges * args.steps / tot
+    sample = (f"oracle/c fp64 GAT fwd+bwd (one layer, H={cfg.heads}, F={cfg.head_dim}) over the first {R} "
+              f"destination rows of the MEGA order ({edges} edges, sources global, n={cfg.n})")
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic (mega-synth v1)", "config": {"workload": f"{cfg.name}-shaped sample", "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "edges/s", "cores": cores(), "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def run_mega(args):
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    if world > 1 or args.gpus > 1:
+        from paper_conf_icdcs_dengr24_b200 import dist as D
+        return D.bench_distributed(args, build_workload, METRIC, ClockSampler, peaks, algorithmic_bytes,
+                                   cpu_sample, cores)
+    if not torch.cuda.is_available():
+        raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
+    dev = torch.device("cuda:0")
+    torch.cuda.set_device(dev)
+    t0 = time.time()
+    wl = build_workload(args.config, args.dtype, args.order)
+    cfg = wl["cfg"]
+    log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s")
+    model = Model(wl, args.dtype, dev)
+    for _ in range(max(3, args.warmup)):
+        model.step()
+    torch.cuda.synchronize()
+    # ---- device-timed region (inputs resident; inputs >> L2 so no flush) ----
+    ev = {}
+    start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(0) as clk:
+        torch.cuda.synchronize()
+        start.record()
+        for _ in range(args.steps):
+            model.step(ev)
+        end.record()
+        torch.cuda.synchronize()
+    ms = start.elapsed_time(end) / args.steps
+    calls = {k: float(np.mean([s.elapsed_time(e) for s, e in v])) for k, v in ev.items()}
+    per_step_calls = {k: float(np.sum([s.elapsed_time(e) for s, e in v])) / args.steps for k, v in ev.items()}
+    L = cfg.layers
+    value = L * cfg.m / (ms * 1e-3)
+    # roofline of the dominant attention call
+    pk = peaks()
+    sb = 2 if args.dtype == "bf16" else 4
+    att = {k: per_step_calls[k] for k in ("gat_fwd", "gat_bwd_src", "gat_bwd_dst")}
+    dom = max(att, key=att.get)
+    bytes_per_launch = algorithmic_bytes(dom, cfg.n, cfg.m, cfg.heads, cfg.dim, sb)
+    achieved = bytes_per_launch / (calls[dom] * 1e-3) / 1e9
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", f"traffic_{cfg.name}_{args.dtype}.json")
+    if os.path.exists(tp):
+        traffic = json.load(open(tp)).get(dom)
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
+                "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "algorithmic_bytes": bytes_per_launch,
+                "launch_ms": calls[dom], "peak_source": pk["source"]}
+    # ---- e2e: pinned host inputs -> device each step, grads back ----
+    e2e = None
+    if not args.no_e2e:
+        hx = model.x0.cpu().pin_memory()
+        hg = model.g.cpu().pin_memory()
+        outs = [L_.grad_w for L_ in model.layers] + [L_.grad_attn_l for L_ in model.layers] + \
+               [L_.grad_attn_r for L_ in model.layers]
+        hout = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
+        h2d = hx.numel() * hx.element_size() + hg.numel() * hg.element_size()
+        d2h = sum(o.numel() * o.element_size() for o in outs)
+        for _ in range(2):
+            model.x0.copy_(hx, non_blocking=True); model.g.copy_(hg, non_blocking=True)
+            model.step()
+            for h, o in zip(hout, outs):
+                h.copy_(o, non_blocking=True)
+            torch.cuda.synchronize()
+        s2, e2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s2.record()
+        for _ in range(args.steps):
+            model.x0.copy_(hx, non_blocking=True)
+            model.g.copy_(hg, non_blocking=True)
+            model.step()
+            for h, o in zip(hout, outs):
+                h.copy_(o, non_blocking=True)
+        e2.record()
+        torch.cuda.synchronize()
+        ms_e2e = s2.elapsed_time(e2) / args.steps
+        e2e = {"value": L * cfg.m / (ms_e2e * 1e-3), "unit": "edges/s", "h2d_bytes_per_step": int(h2d),
+               "d2h_bytes_per_step": int(d2h), "ms_per_step": ms_e2e}
+    # ---- CPU oracle baseline (bounded sample) ----
+    cpu = None
+    if not args.no_cpu_baseline:
+        run, R = cpu_sample(wl, args.cpu_seconds, cfg.heads, cfg.head_dim)
+        t, e = run(R)
+        cpu = {"value": e / t, "unit": "edges/s", "cores": cores(), "kind": "oracle",
+               "sample": f"oracle/c fp64 one-layer GAT fwd+bwd over the first {R} destination rows of the MEGA "
+                         f"order ({e} edges, all sources, n={cfg.n}); {t:.1f} s"}
+    st = wl["layout"].stats()
+    line = {
+        "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": 1, "steps": args.steps,
+        "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": args.dtype,
+        "data": "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)",
+        "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
+                   "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
+                   "order": args.order, "parallelism": "single GPU",
+                   "value_definition": "layers * E / step time (each layer's edges fwd+bwd)",
+                   "l2": "no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)},
+        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
+        "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
+        "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",
+                                      "tile_unique_sources", "max_in_degree", "preprocess_seconds")},
+        "setup_s": time.time() - t0,
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_mega(args)
+
+
+if __name__ == "__main__":
+    main()

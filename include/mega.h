@@ -1,0 +1,246 @@
+/*
+ * mega.h — C ABI of libmega.so, the B200-native hot path of MEGA
+ * (Deng & Rao, "MEGA: More Efficient Graph Attention for GNNs", ICDCS'24).
+ * ABI version 1.  C linkage; plain pointers and sizes; no C++ or torch types.
+ *
+ * Citations "PAPER.md:L" are lines of the paper text;
+ * DESIGN.md "Rn" are the documented readings of ambiguous passages.
+ *
+ * What the library computes (BASELINE.json north_star; GAT [14] cited at
+ * PAPER.md:49; layer skeleton PAPER.md:51-55):
+ *   a1  mega_preprocess   one traversal of the graph (Algorithm 1,
+ *                         PAPER.md:239-306, reading R) -> node order -> an
+ *                         exact relabelled layout (CSR, CSC, work items,
+ *                         partitions) that preserves the edge multiset.
+ *   a2  mega_project_fwd  Wh = X W (tensor cores), el = Wh.a_l, er = Wh.a_r.
+ *   a3-a5 mega_gat_fwd    e_ij = LeakyReLU(a_l.Wh_i + a_r.Wh_j) for every edge
+ *                         j->i, per-destination softmax, out_i = sum alpha Wh_j.
+ *   a6-a8 mega_gat_bwd    gradients w.r.t. Wh, a_l, a_r.
+ *   a9  mega_project_bwd  dW = X^T dWh, dX = dWh W^T.
+ *
+ * Conventions
+ *   - Node ids: "new" ids are positions in the traversal order (perm[new] =
+ *     old).  Every feature/ctx array passed to the compute calls is indexed
+ *     by NEW ids; use mega_layout_view().perm to permute.
+ *   - i = destination (CSR row, the aggregating node), j = source.  attn_l
+ *     multiplies the DESTINATION row and attn_r the SOURCE row, exactly as
+ *     north_star writes e_ij (DGL's GATConv names them the other way round).
+ *   - Features are row-major [rows][ld] with D = heads*head_dim used columns,
+ *     heads concatenated (column h*head_dim + f).  attn_l/attn_r are fp32
+ *     [heads*head_dim] in the same column order.
+ *   - ctx is an fp32 block of four planes [4][ctx_n][heads]: el, er, lse,
+ *     Dlt, indexed by GLOBAL new node id (ctx_n = num_nodes).  lse = -inf for
+ *     rows with no in-edges (whose out row is 0) (R6).
+ *   - Multi-part layouts (num_parts = k > 1, destination-partitioned across k
+ *     GPUs): part p owns rows [bounds[p], bounds[p+1]).  For
+ *     part p, `out`, `grad_out` are LOCAL row arrays [rows_p][ld]; `feat`,
+ *     `grad_feat` and ctx are GLOBAL [num_nodes].
+ *   - Memory: the library never allocates device memory.  The caller owns
+ *     every device buffer (the layout image, features, ctx, workspaces,
+ *     outputs).  Host arrays passed in are read only during the call.
+ *   - Streams: every device call is asynchronous and stream-ordered on the
+ *     caller's stream (NULL = legacy default stream); the library never
+ *     synchronises with the host unless MEGA_DEBUG_SYNC=1 is set in the
+ *     environment (then every call synchronises and checks for faults).
+ *   - Errors: every function returns mega_status; mega_last_error() gives a
+ *     thread-local message for the last failure.  Arguments are validated on
+ *     the host before any launch; outputs are unspecified after an error.
+ *     Asynchronous device faults surface at the caller's next synchronisation.
+ *   - Determinism: no atomics on any value path; results are bitwise
+ *     reproducible run to run on the same GPU and layout.
+ */
+#ifndef MEGA_H
+#define MEGA_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define MEGA_ABI_VERSION 1
+
+typedef struct CUstream_st *mega_stream_t; /* == cudaStream_t */
+
+typedef enum {
+  MEGA_OK = 0,
+  MEGA_ERR_INVALID_ARGUMENT = 1, /* null pointer, bad size, misaligned pointer/ld, bad dtype */
+  MEGA_ERR_INVALID_GRAPH = 2,    /* indptr not monotone, indptr[n] != m, index out of range */
+  MEGA_ERR_UNSUPPORTED = 3,      /* shape outside the kernels' supported set; device not sm_100 */
+  MEGA_ERR_OUT_OF_MEMORY = 4,    /* host allocation failed, or a caller buffer is too small */
+  MEGA_ERR_CUDA = 5,             /* a CUDA runtime / cuBLAS call failed (message has details) */
+  MEGA_ERR_STATE = 6,            /* layout part not bound, or bound to another device */
+  MEGA_ERR_IO = 7                /* mega_layout_save / _load file errors or bad format */
+} mega_status;
+
+typedef enum { MEGA_F32 = 0, MEGA_BF16 = 1 } mega_dtype;
+
+typedef enum {
+  MEGA_ORDER_TRAVERSAL = 0, /* MEGA: traversal R of Algorithm 1 (the method) */
+  MEGA_ORDER_IDENTITY = 1,  /* ablation: input order */
+  MEGA_ORDER_DEGREE = 2,    /* ablation: stable sort by (-in-degree, id) */
+  MEGA_ORDER_RANDOM = 3     /* ablation: Fisher-Yates on splitmix64(seed) */
+} mega_order;
+
+/* Input graph: CSR by destination.  Row i lists the sources j of the edges
+ * j -> i (the paper's (v_src, v_dst) pairs).  Duplicate edges
+ * and self-loops are allowed and kept (multiset semantics, R4/R5).
+ * Requires 0 <= num_edges < 2^31 and 0 < num_nodes < 2^31. */
+typedef struct {
+  int64_t num_nodes;
+  int64_t num_edges;
+  const int64_t *indptr;  /* host [num_nodes + 1], indptr[0] = 0, monotone, indptr[n] = m */
+  const int32_t *indices; /* host [num_edges], 0 <= j < num_nodes */
+} mega_csr;
+
+/* Schedule options.  Initialise with
+ * mega_schedule_opts_init(); struct_size guards ABI evolution. */
+typedef struct {
+  uint32_t struct_size;
+  int32_t window;        /* omega; 0 = auto clamp(round(m/n), 1, 64) */
+  int32_t candidate_cap; /* K tier-1 candidates examined per step; 0 = 32 */
+  int32_t order;         /* mega_order; non-TRAVERSAL orders exist for A/B ablations */
+  int32_t seg_edges;     /* S: rows/sources with more edges are split into segments; 0 = auto */
+  int32_t num_parts;     /* k >= 1 destination partitions (one per GPU) */
+  uint64_t seed;         /* MEGA_ORDER_RANDOM only */
+} mega_schedule_opts;
+
+typedef struct mega_layout mega_layout;
+
+typedef struct {
+  uint32_t struct_size;
+  int64_t num_nodes, num_edges, num_parts;
+  int64_t window, candidate_cap, seg_edges, order;
+  int64_t path_length; /* |P|: appearances incl. revisits */
+  int64_t revisits;    /* |P| - n */
+  int64_t jumps;       /* tier-3 picks after the start (virtual edges) */
+  int64_t tile_unique_sources; /* sum over 64-row tiles of distinct sources (reuse = m / this) */
+  int64_t max_in_degree, max_out_degree;
+  double preprocess_seconds;
+} mega_layout_stats;
+
+/* Read-only host view of one part (for parity tests and for moving data into
+ * the new order).  Pointers stay valid until mega_layout_destroy. */
+typedef struct {
+  uint32_t struct_size;
+  int64_t num_nodes, num_edges; /* whole graph */
+  int64_t row_begin, row_end;   /* rows of this part (new ids) */
+  int64_t part_edges;
+  int64_t num_fwd_items, num_fwd_splits, num_bwd_items, num_bwd_splits;
+  int64_t num_parts;
+  const int32_t *perm;       /* [num_nodes]   old id of new id */
+  const int32_t *new_of_old; /* [num_nodes] */
+  const int32_t *bounds;     /* [num_parts+1] row bounds of all parts */
+  const int32_t *indptr;     /* [rows+1]  part-local CSR positions, rows sorted by (src, eid) */
+  const int32_t *src;        /* [part_edges] new source id */
+  const int32_t *eid;        /* [part_edges] position of the edge in the input CSR */
+  const int32_t *cindptr;    /* [num_nodes+1] CSC over this part's edges, by new source id */
+  const int32_t *cdst;       /* [part_edges] local destination row */
+  const int32_t *cpos;       /* [part_edges] CSR position of CSC entry */
+  const int32_t *csr2csc;    /* [part_edges] inverse of cpos */
+  const int32_t *fwd_items;  /* [num_fwd_items][4] (row, e_begin, e_end, slot|-1) over CSR */
+  const int32_t *fwd_splits; /* [num_fwd_splits][3] (row, first_slot, nseg) */
+  const int32_t *bwd_items;  /* [num_bwd_items][4] over CSC rows (sources) */
+  const int32_t *bwd_splits; /* [num_bwd_splits][3] */
+} mega_layout_view;
+
+/* Flags */
+#define MEGA_FLAG_ELER_IN_CTX 1u /* mega_gat_fwd: el/er planes of ctx are already valid (from
+                                    mega_project_fwd); otherwise they are computed from feat */
+#define MEGA_BWD_PHASE_SRC 2u    /* mega_gat_bwd: Dlt + source-major pass -> partial grad_feat for
+                                    ALL sources (k > 1: reduce over ranks before PHASE_DST), grad_attn_r */
+#define MEGA_BWD_PHASE_DST 4u    /* mega_gat_bwd: destination pass -> adds del_i a_l to this part's rows
+                                    of grad_feat, grad_attn_l.  Neither phase flag = both. */
+
+int mega_abi_version(void);
+const char *mega_status_string(mega_status s);
+const char *mega_last_error(void); /* thread-local; "" if none */
+void mega_schedule_opts_init(mega_schedule_opts *opts);
+
+/* a1. Reorganise (host, once per graph).  Traverses the graph once with
+ * reading R of Algorithm 1 to get the node order,
+ * then rewrites the CSR into the layout.  The edge
+ * multiset is preserved exactly.  *out receives a new layout owned by the
+ * caller (free with mega_layout_destroy).  Errors: INVALID_ARGUMENT (null,
+ * opts), INVALID_GRAPH (CSR checks), OUT_OF_MEMORY. */
+mega_status mega_preprocess(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout **out);
+void mega_layout_destroy(mega_layout *layout);
+mega_status mega_layout_stats_get(const mega_layout *layout, mega_layout_stats *out);
+mega_status mega_layout_view_get(const mega_layout *layout, int32_t part, mega_layout_view *out);
+
+/* Persist / restore a layout (host part only; bind again after load).
+ * Versioned little-endian binary with a checksum.  Errors: IO. */
+mega_status mega_layout_save(const mega_layout *layout, const char *path);
+mega_status mega_layout_load(const char *path, mega_layout **out);
+
+/* Device image of one part: size, then an async H2D copy into a caller-owned
+ * device buffer (>= bytes, 256-byte aligned) on `stream`, on the current
+ * device.  The buffer must outlive every compute call on this part.  A part
+ * may be re-bound (to another buffer or device).  Errors: INVALID_ARGUMENT,
+ * OUT_OF_MEMORY (buffer too small), CUDA. */
+mega_status mega_layout_device_bytes(const mega_layout *layout, int32_t part, size_t *bytes);
+mega_status mega_layout_bind_device(mega_layout *layout, int32_t part, void *dev_buf, size_t bytes,
+                                    mega_stream_t stream);
+
+/* Workspace sizes (bytes, device) for mega_gat_fwd and mega_gat_bwd on a
+ * part at this head shape and dtype. */
+mega_status mega_gat_workspace_bytes(const mega_layout *layout, int32_t part, int heads, int head_dim,
+                                     mega_dtype dtype, size_t *fwd_ws, size_t *bwd_ws);
+
+/* a2. Projection (neural operator): feat = x * w on tensor
+ * cores (bf16 inputs, fp32 accumulation; MEGA_F32 = true fp32, no TF32),
+ * then el/er of every projected row into ctx rows [ctx_row0, ctx_row0+rows).
+ *   x    device [rows][ldx] dtype, w device [in_dim][heads*head_dim] dtype,
+ *   feat device [rows][ldf] dtype, ctx device fp32 [4][ctx_n][heads].
+ * Errors: INVALID_ARGUMENT, UNSUPPORTED, CUDA. */
+mega_status mega_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
+                             int head_dim, const float *attn_l, const float *attn_r, mega_dtype dtype, void *feat,
+                             int64_t ldf, float *ctx, int64_t ctx_n, int64_t ctx_row0, mega_stream_t stream);
+
+/* a3-a5. Fused forward over `part`: per-edge score, per-destination online
+ * softmax and attention-weighted aggregation, one pass over the edges
+ * (PAPER.md:7, 84 — the irregular graph op the paper targets).
+ *   feat  device [num_nodes][ldf] dtype (all sources, new order)
+ *   out   device [rows_p][ldo] dtype  (written; 0 for rows without in-edges)
+ *   ctx   device fp32 [4][num_nodes][heads]: writes lse (and el/er unless
+ *         MEGA_FLAG_ELER_IN_CTX)
+ *   ws    device, >= fwd_ws bytes from mega_gat_workspace_bytes.
+ * Supported shapes: heads <= 8; head_dim a multiple of 8 (bf16) / 4 (fp32);
+ * D/8 (bf16) or D/4 (fp32) a power of two <= 32 or a multiple of 32 up to 256;
+ * ld*sizeof(dtype) a multiple of 16 and 16-byte aligned pointers.
+ * Errors: INVALID_ARGUMENT, UNSUPPORTED, STATE (part not bound here), CUDA. */
+mega_status mega_gat_fwd(const mega_layout *layout, int32_t part, const void *feat, int64_t ldf,
+                         const float *attn_l, const float *attn_r, int heads, int head_dim, mega_dtype dtype,
+                         float negative_slope, uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws,
+                         size_t ws_bytes, mega_stream_t stream);
+
+/* a6-a8. Backward of mega_gat_fwd:
+ *   Dlt_i = g_i.out_i; source-major pass over the CSC recomputing alpha and
+ *   accumulating dWh_j = sum alpha g_i + der_j a_r, storing dz per edge;
+ *   destination pass del_i = sum dz, dWh_i += del_i a_l.
+ *   grad_out     device [rows_p][ldg] dtype
+ *   grad_feat    device fp32 [num_nodes][ldgf] (written)
+ *   grad_feat_lp optional device dtype [num_nodes][ldlp] copy of the final
+ *                grad_feat rows of this part (operand of mega_project_bwd), or NULL
+ *   grad_attn_l/r device fp32 [heads*head_dim] (written)
+ * flags: MEGA_BWD_PHASE_* (see above).  Errors as mega_gat_fwd. */
+mega_status mega_gat_bwd(const mega_layout *layout, int32_t part, const void *feat, int64_t ldf,
+                         const float *attn_l, const float *attn_r, int heads, int head_dim, mega_dtype dtype,
+                         float negative_slope, uint32_t flags, const void *out, int64_t ldo, const void *grad_out,
+                         int64_t ldg, float *ctx, float *grad_feat, int64_t ldgf, void *grad_feat_lp,
+                         int64_t ldlp, float *grad_attn_l, float *grad_attn_r, void *ws, size_t ws_bytes,
+                         mega_stream_t stream);
+
+/* a9. Projection backward on tensor cores: grad_w = x^T grad_feat (fp32
+ * [in_dim][D], written) and, if grad_x != NULL, grad_x = grad_feat w^T
+ * (dtype [rows][ldgx]).  grad_feat is fp32 for MEGA_F32 and the bf16 copy
+ * (grad_feat_lp of mega_gat_bwd) for MEGA_BF16.  Errors as mega_project_fwd. */
+mega_status mega_project_bwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
+                             int head_dim, mega_dtype dtype, const void *grad_feat, int64_t ldgf, void *grad_x,
+                             int64_t ldgx, float *grad_w, mega_stream_t stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MEGA_H */

@@ -1,0 +1,308 @@
+// C ABI: errors, options, layout lifetime, views, persistence and device binding.
+#include <cuda_runtime.h>
+
+#include <cstdio>
+#include <cstring>
+#include <new>
+
+#include "mega_internal.h"
+
+namespace mega {
+static thread_local std::string g_last_error;
+
+mega_status fail(mega_status s, const std::string &msg) {
+  g_last_error = msg;
+  return s;
+}
+void clear_error() { g_last_error.clear(); }
+
+static const size_t kAlign = 256;
+static size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
+
+// Device image of one part: 9 int32 arrays at 256-byte aligned offsets.
+size_t part_image_bytes(const mega_layout *L, int part, size_t offs[9]) {
+  const Part &P = L->parts[part];
+  const size_t sizes[9] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(), P.csr2csc.size(),
+                           P.fwd_items.size(), P.fwd_splits.size(), P.bwd_items.size(), P.bwd_splits.size()};
+  size_t off = 0;
+  for (int i = 0; i < 9; ++i) {
+    offs[i] = off;
+    off = align_up(off + sizes[i] * sizeof(int32_t));
+  }
+  return off;
+}
+}  // namespace mega
+
+using namespace mega;
+
+extern "C" {
+
+int mega_abi_version(void) { return MEGA_ABI_VERSION; }
+
+const char *mega_status_string(mega_status s) {
+  switch (s) {
+    case MEGA_OK: return "MEGA_OK";
+    case MEGA_ERR_INVALID_ARGUMENT: return "MEGA_ERR_INVALID_ARGUMENT";
+    case MEGA_ERR_INVALID_GRAPH: return "MEGA_ERR_INVALID_GRAPH";
+    case MEGA_ERR_UNSUPPORTED: return "MEGA_ERR_UNSUPPORTED";
+    case MEGA_ERR_OUT_OF_MEMORY: return "MEGA_ERR_OUT_OF_MEMORY";
+    case MEGA_ERR_CUDA: return "MEGA_ERR_CUDA";
+    case MEGA_ERR_STATE: return "MEGA_ERR_STATE";
+    case MEGA_ERR_IO: return "MEGA_ERR_IO";
+  }
+  return "MEGA_ERR_UNKNOWN";
+}
+
+const char *mega_last_error(void) { return g_last_error.c_str(); }
+
+void mega_schedule_opts_init(mega_schedule_opts *o) {
+  if (!o) return;
+  std::memset(o, 0, sizeof *o);
+  o->struct_size = sizeof *o;
+  o->order = MEGA_ORDER_TRAVERSAL;
+  o->num_parts = 1;
+}
+
+mega_status mega_preprocess(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout **out) {
+  clear_error();
+  if (!csr || !opts || !out) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  *out = nullptr;
+  if (opts->struct_size != sizeof(mega_schedule_opts))
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "mega_schedule_opts.struct_size mismatch (call mega_schedule_opts_init)");
+  const int64_t n = csr->num_nodes, m = csr->num_edges;
+  if (n <= 0 || n >= (1LL << 31)) return fail(MEGA_ERR_INVALID_GRAPH, "num_nodes must be in [1, 2^31)");
+  if (m < 0 || m >= (1LL << 31)) return fail(MEGA_ERR_INVALID_GRAPH, "num_edges must be in [0, 2^31)");
+  if (!csr->indptr || (m > 0 && !csr->indices)) return fail(MEGA_ERR_INVALID_ARGUMENT, "null CSR array");
+  if (opts->num_parts < 1 || opts->num_parts > 1024) return fail(MEGA_ERR_INVALID_ARGUMENT, "num_parts must be in [1, 1024]");
+  if (opts->candidate_cap < 0 || opts->candidate_cap > 64)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "candidate_cap must be in [0, 64]");
+  if (opts->window < 0 || opts->seg_edges < 0) return fail(MEGA_ERR_INVALID_ARGUMENT, "negative window/seg_edges");
+  if (opts->order < 0 || opts->order > MEGA_ORDER_RANDOM) return fail(MEGA_ERR_INVALID_ARGUMENT, "unknown order");
+  if (csr->indptr[0] != 0 || csr->indptr[n] != m) return fail(MEGA_ERR_INVALID_GRAPH, "indptr[0] != 0 or indptr[n] != m");
+  for (int64_t i = 0; i < n; ++i)
+    if (csr->indptr[i + 1] < csr->indptr[i]) return fail(MEGA_ERR_INVALID_GRAPH, "indptr not monotone");
+  for (int64_t e = 0; e < m; ++e)
+    if (csr->indices[e] < 0 || csr->indices[e] >= n)
+      return fail(MEGA_ERR_INVALID_GRAPH, "source index out of range at edge " + std::to_string(e));
+  mega_layout *L = new (std::nothrow) mega_layout();
+  if (!L) return fail(MEGA_ERR_OUT_OF_MEMORY, "layout allocation");
+  try {
+    mega_status s = build_layout(csr, opts, L);
+    if (s != MEGA_OK) { delete L; return s; }
+  } catch (const std::bad_alloc &) {
+    delete L;
+    return fail(MEGA_ERR_OUT_OF_MEMORY, "host allocation failed while building the layout");
+  }
+  *out = L;
+  return MEGA_OK;
+}
+
+void mega_layout_destroy(mega_layout *L) { delete L; }
+
+mega_status mega_layout_stats_get(const mega_layout *L, mega_layout_stats *out) {
+  clear_error();
+  if (!L || !out) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  *out = L->stats;
+  return MEGA_OK;
+}
+
+mega_status mega_layout_view_get(const mega_layout *L, int32_t part, mega_layout_view *v) {
+  clear_error();
+  if (!L || !v) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  const Part &P = L->parts[part];
+  std::memset(v, 0, sizeof *v);
+  v->struct_size = sizeof *v;
+  v->num_nodes = L->n;
+  v->num_edges = L->m;
+  v->row_begin = P.row_begin;
+  v->row_end = P.row_end;
+  v->part_edges = (int64_t)P.src.size();
+  v->num_fwd_items = (int64_t)P.fwd_items.size() / 4;
+  v->num_fwd_splits = (int64_t)P.fwd_splits.size() / 3;
+  v->num_bwd_items = (int64_t)P.bwd_items.size() / 4;
+  v->num_bwd_splits = (int64_t)P.bwd_splits.size() / 3;
+  v->num_parts = (int64_t)L->parts.size();
+  v->perm = L->perm.data();
+  v->new_of_old = L->new_of_old.data();
+  v->bounds = L->bounds.data();
+  v->indptr = P.indptr.data();
+  v->src = P.src.data();
+  v->eid = P.eid.data();
+  v->cindptr = P.cindptr.data();
+  v->cdst = P.cdst.data();
+  v->cpos = P.cpos.data();
+  v->csr2csc = P.csr2csc.data();
+  v->fwd_items = P.fwd_items.data();
+  v->fwd_splits = P.fwd_splits.data();
+  v->bwd_items = P.bwd_items.data();
+  v->bwd_splits = P.bwd_splits.data();
+  return MEGA_OK;
+}
+
+mega_status mega_layout_device_bytes(const mega_layout *L, int32_t part, size_t *bytes) {
+  clear_error();
+  if (!L || !bytes) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  size_t offs[9];
+  *bytes = part_image_bytes(L, part, offs);
+  return MEGA_OK;
+}
+
+mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf, size_t bytes,
+                                    mega_stream_t stream) {
+  clear_error();
+  if (!L || !dev_buf) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  if (reinterpret_cast<uintptr_t>(dev_buf) % 256) return fail(MEGA_ERR_INVALID_ARGUMENT, "dev_buf must be 256-byte aligned");
+  size_t offs[9];
+  const size_t need = part_image_bytes(L, part, offs);
+  if (bytes < need) return fail(MEGA_ERR_OUT_OF_MEMORY, "device buffer smaller than mega_layout_device_bytes");
+  Part &P = L->parts[part];
+  int dev = 0;
+  cudaError_t ce = cudaGetDevice(&dev);
+  if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(ce));
+  const std::vector<int32_t> *arrs[9] = {&P.indptr, &P.src, &P.cindptr, &P.cdst, &P.csr2csc,
+                                         &P.fwd_items, &P.fwd_splits, &P.bwd_items, &P.bwd_splits};
+  char *base = static_cast<char *>(dev_buf);
+  for (int i = 0; i < 9; ++i) {
+    if (arrs[i]->empty()) continue;
+    ce = cudaMemcpyAsync(base + offs[i], arrs[i]->data(), arrs[i]->size() * sizeof(int32_t), cudaMemcpyHostToDevice,
+                         (cudaStream_t)stream);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("layout H2D copy: ") + cudaGetErrorString(ce));
+  }
+  P.device = dev;
+  P.dev_base = dev_buf;
+  DevPart &D = P.dev;
+  D.indptr = reinterpret_cast<const int32_t *>(base + offs[0]);
+  D.src = reinterpret_cast<const int32_t *>(base + offs[1]);
+  D.cindptr = reinterpret_cast<const int32_t *>(base + offs[2]);
+  D.cdst = reinterpret_cast<const int32_t *>(base + offs[3]);
+  D.csr2csc = reinterpret_cast<const int32_t *>(base + offs[4]);
+  D.fwd_items = reinterpret_cast<const int4 *>(base + offs[5]);
+  D.fwd_splits = reinterpret_cast<const int32_t *>(base + offs[6]);
+  D.bwd_items = reinterpret_cast<const int4 *>(base + offs[7]);
+  D.bwd_splits = reinterpret_cast<const int32_t *>(base + offs[8]);
+  D.n = L->n;
+  D.rows = P.row_end - P.row_begin;
+  D.row_begin = P.row_begin;
+  D.edges = (int64_t)P.src.size();
+  D.n_fwd_items = (int32_t)(P.fwd_items.size() / 4);
+  D.n_fwd_splits = (int32_t)(P.fwd_splits.size() / 3);
+  D.n_fwd_slots = P.n_fwd_slots;
+  D.n_bwd_items = (int32_t)(P.bwd_items.size() / 4);
+  D.n_bwd_splits = (int32_t)(P.bwd_splits.size() / 3);
+  D.n_bwd_slots = P.n_bwd_slots;
+  return MEGA_OK;
+}
+
+}  // extern "C"
+
+// ---- persistence: "MEGALYT1" | version | sizes | arrays | fnv1a-64 checksum ----
+namespace {
+struct Writer {
+  FILE *f;
+  uint64_t h = 1469598103934665603ULL;
+  bool ok = true;
+  void raw(const void *p, size_t n) {
+    const unsigned char *c = static_cast<const unsigned char *>(p);
+    for (size_t i = 0; i < n; ++i) { h ^= c[i]; h *= 1099511628211ULL; }
+    if (fwrite(p, 1, n, f) != n) ok = false;
+  }
+  template <typename T> void pod(const T &x) { raw(&x, sizeof x); }
+  void vec(const std::vector<int32_t> &v) {
+    uint64_t n = v.size();
+    pod(n);
+    if (n) raw(v.data(), n * sizeof(int32_t));
+  }
+};
+struct Reader {
+  FILE *f;
+  uint64_t h = 1469598103934665603ULL;
+  bool ok = true;
+  void raw(void *p, size_t n) {
+    if (fread(p, 1, n, f) != n) { ok = false; return; }
+    const unsigned char *c = static_cast<const unsigned char *>(p);
+    for (size_t i = 0; i < n; ++i) { h ^= c[i]; h *= 1099511628211ULL; }
+  }
+  template <typename T> void pod(T &x) { raw(&x, sizeof x); }
+  void vec(std::vector<int32_t> &v) {
+    uint64_t n = 0;
+    pod(n);
+    if (!ok || n > (1ULL << 34)) { ok = false; return; }
+    v.resize(n);
+    if (n) raw(v.data(), n * sizeof(int32_t));
+  }
+};
+const char kMagic[8] = {'M', 'E', 'G', 'A', 'L', 'Y', 'T', '1'};
+}  // namespace
+
+extern "C" {
+
+mega_status mega_layout_save(const mega_layout *L, const char *path) {
+  clear_error();
+  if (!L || !path) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  FILE *f = fopen(path, "wb");
+  if (!f) return fail(MEGA_ERR_IO, std::string("cannot open ") + path);
+  Writer w{f};
+  w.raw(kMagic, 8);
+  int32_t ver = MEGA_ABI_VERSION;
+  w.pod(ver);
+  w.pod(L->n); w.pod(L->m); w.pod(L->opts); w.pod(L->stats);
+  w.vec(L->perm); w.vec(L->new_of_old); w.vec(L->bounds);
+  uint64_t k = L->parts.size();
+  w.pod(k);
+  for (const Part &P : L->parts) {
+    w.pod(P.row_begin); w.pod(P.row_end); w.pod(P.n_fwd_slots); w.pod(P.n_bwd_slots);
+    w.vec(P.indptr); w.vec(P.src); w.vec(P.eid); w.vec(P.cindptr); w.vec(P.cdst); w.vec(P.cpos);
+    w.vec(P.csr2csc); w.vec(P.fwd_items); w.vec(P.fwd_splits); w.vec(P.bwd_items); w.vec(P.bwd_splits);
+  }
+  uint64_t sum = w.h;
+  bool ok = w.ok && fwrite(&sum, sizeof sum, 1, f) == 1;
+  ok = (fclose(f) == 0) && ok;
+  return ok ? MEGA_OK : fail(MEGA_ERR_IO, "write failed");
+}
+
+mega_status mega_layout_load(const char *path, mega_layout **out) {
+  clear_error();
+  if (!path || !out) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  *out = nullptr;
+  FILE *f = fopen(path, "rb");
+  if (!f) return fail(MEGA_ERR_IO, std::string("cannot open ") + path);
+  mega_layout *L = new (std::nothrow) mega_layout();
+  if (!L) { fclose(f); return fail(MEGA_ERR_OUT_OF_MEMORY, "layout allocation"); }
+  Reader r{f};
+  char magic[8];
+  r.raw(magic, 8);
+  int32_t ver = 0;
+  r.pod(ver);
+  if (!r.ok || std::memcmp(magic, kMagic, 8) != 0 || ver != MEGA_ABI_VERSION) {
+    fclose(f); delete L;
+    return fail(MEGA_ERR_IO, "not a MEGA layout file (magic/version)");
+  }
+  try {
+    r.pod(L->n); r.pod(L->m); r.pod(L->opts); r.pod(L->stats);
+    r.vec(L->perm); r.vec(L->new_of_old); r.vec(L->bounds);
+    uint64_t k = 0;
+    r.pod(k);
+    if (!r.ok || k < 1 || k > 1024) throw 0;
+    L->parts.resize(k);
+    for (Part &P : L->parts) {
+      r.pod(P.row_begin); r.pod(P.row_end); r.pod(P.n_fwd_slots); r.pod(P.n_bwd_slots);
+      r.vec(P.indptr); r.vec(P.src); r.vec(P.eid); r.vec(P.cindptr); r.vec(P.cdst); r.vec(P.cpos);
+      r.vec(P.csr2csc); r.vec(P.fwd_items); r.vec(P.fwd_splits); r.vec(P.bwd_items); r.vec(P.bwd_splits);
+      if (!r.ok) throw 0;
+    }
+  } catch (...) {
+    fclose(f); delete L;
+    return fail(MEGA_ERR_IO, "truncated or corrupt layout file");
+  }
+  uint64_t expect = r.h, sum = 0;
+  bool ok = r.ok && fread(&sum, sizeof sum, 1, f) == 1 && sum == expect;
+  fclose(f);
+  if (!ok) { delete L; return fail(MEGA_ERR_IO, "layout file checksum mismatch"); }
+  *out = L;
+  return MEGA_OK;
+}
+
+}  // extern "C"

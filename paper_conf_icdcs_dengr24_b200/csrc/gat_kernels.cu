@@ -1,0 +1,1034 @@
+// a3-a8: the GAT attention kernels for sm_100a and their C-ABI entry points.
+//
+// Memory-bound graph operators: no tensor cores here
+// (north_star).  Design:
+//   * a "group" of G lanes owns one work item (a destination row or a
+//     segment of one); each lane holds V 16-byte vectors of a feature row, so
+//     one source row is fetched with G*V coalesced 128-bit loads;
+//   * scores are computed once per (edge, head): in the score phase lane l
+//     handles edge base+l for all heads, then the group's online softmax
+//     state (running max, per-lane partial sums) is updated with shuffles;
+//   * probabilities and source ids are staged in shared memory and the
+//     aggregation loop keeps U rows in flight per lane;
+//   * rows/sources longer than S edges were split by mega_preprocess into
+//     segments whose partial softmax states are merged deterministically
+//     (no atomics anywhere on the value path);
+//   * items are assigned grid-stride in path order, so concurrently running
+//     groups work on neighbouring rows of the MEGA order and share sources
+//     in L1/L2 (the locality the traversal creates).
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdlib>
+#include <mutex>
+#include <type_traits>
+#include <unordered_map>
+
+#include "mega_internal.h"
+
+namespace mega {
+namespace kern {
+
+constexpr int MAXH = 8;
+constexpr int WPB = 8;
+constexpr int TPB = WPB * 32;
+constexpr int MAX_GRID = 4096;  // upper bound for per-block partial buffers
+constexpr int SP = MAXH + 1;    // smem row pitch (bank-conflict free)
+
+template <typename T> struct Tr;
+template <> struct Tr<float> { static constexpr int EPV = 4; };
+template <> struct Tr<__nv_bfloat16> { static constexpr int EPV = 8; };
+
+__device__ __forceinline__ uint4 ldg16(const void *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
+__device__ __forceinline__ int ld_stream(const int32_t *p) {
+  int v;
+  asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ void st16(void *p, uint4 v) { *reinterpret_cast<uint4 *>(p) = v; }
+
+__device__ __forceinline__ void unpack(const uint4 &r, float (&x)[4], float) {
+  x[0] = __uint_as_float(r.x); x[1] = __uint_as_float(r.y);
+  x[2] = __uint_as_float(r.z); x[3] = __uint_as_float(r.w);
+}
+__device__ __forceinline__ void unpack(const uint4 &r, float (&x)[8], __nv_bfloat16) {
+  x[0] = __uint_as_float(r.x << 16); x[1] = __uint_as_float(r.x & 0xffff0000u);
+  x[2] = __uint_as_float(r.y << 16); x[3] = __uint_as_float(r.y & 0xffff0000u);
+  x[4] = __uint_as_float(r.z << 16); x[5] = __uint_as_float(r.z & 0xffff0000u);
+  x[6] = __uint_as_float(r.w << 16); x[7] = __uint_as_float(r.w & 0xffff0000u);
+}
+__device__ __forceinline__ uint32_t pk2(float a, float b) {
+  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t *>(&t);
+}
+__device__ __forceinline__ uint4 pack(const float (&x)[4], float) {
+  return make_uint4(__float_as_uint(x[0]), __float_as_uint(x[1]), __float_as_uint(x[2]), __float_as_uint(x[3]));
+}
+__device__ __forceinline__ uint4 pack(const float (&x)[8], __nv_bfloat16) {
+  return make_uint4(pk2(x[0], x[1]), pk2(x[2], x[3]), pk2(x[4], x[5]), pk2(x[6], x[7]));
+}
+
+template <int G> __device__ __forceinline__ float gmax(float v, unsigned mask) {
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(mask, v, o, G));
+  return v;
+}
+template <int G> __device__ __forceinline__ float gsum(float v, unsigned mask) {
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, G);
+  return v;
+}
+__device__ __forceinline__ float sel(const float (&a)[MAXH], int i) {
+  float r = a[0];
+#pragma unroll
+  for (int h = 1; h < MAXH; ++h)
+    if (i == h) r = a[h];
+  return r;
+}
+// H consecutive fp32 values (16-byte vectors when H % 4 == 0)
+__device__ __forceinline__ void load_h(const float *p, int H, float (&v)[MAXH]) {
+  if ((H & 3) == 0) {
+#pragma unroll
+    for (int q = 0; q < MAXH / 4; ++q)
+      if (4 * q < H) {
+        float4 t = __ldg(reinterpret_cast<const float4 *>(p) + q);
+        v[4 * q] = t.x; v[4 * q + 1] = t.y; v[4 * q + 2] = t.z; v[4 * q + 3] = t.w;
+      }
+  } else {
+#pragma unroll
+    for (int h = 0; h < MAXH; ++h)
+      if (h < H) v[h] = __ldg(p + h);
+  }
+}
+__device__ __forceinline__ float leaky(float z, float slope) { return z > 0.f ? z : slope * z; }
+
+// Sum per-vector partial dot products over the lanes (and vectors) of a head.
+// LPH = lanes per head within one vector (F / EPV).
+template <int G, int U, int V>
+__device__ __forceinline__ void head_reduce(float (&p)[U][V], int LPH, unsigned mask) {
+  if (LPH <= G) {
+    for (int o = LPH >> 1; o > 0; o >>= 1) {
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) p[u][v] += __shfl_xor_sync(mask, p[u][v], o, G);
+    }
+  } else {
+    const int VPH = LPH / G;
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      float q[V];
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        float t = 0.f;
+#pragma unroll
+        for (int v2 = 0; v2 < V; ++v2)
+          if (v2 / VPH == v / VPH) t += p[u][v2];
+        q[v] = t;
+      }
+#pragma unroll
+      for (int v = 0; v < V; ++v) p[u][v] = gsum<G>(q[v], mask);
+    }
+  }
+}
+// Does this lane write the (reduced) value of vector v's head?
+template <int G>
+__device__ __forceinline__ bool head_lead(int gl, int v, int LPH) {
+  return LPH <= G ? (gl % LPH) == 0 : (gl == 0 && (v % (LPH / G)) == 0);
+}
+
+// Reduce per-lane [V][EPV] accumulators over all groups of the block and
+// store the block's [D] partial (fixed order -> deterministic).
+template <int G, int V, int EPV>
+__device__ void block_partial(float (&acc)[V][EPV], float *s_red, float *dst, int D) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G;
+#pragma unroll
+  for (int o = G; o < 32; o <<= 1)
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) acc[v][k] += __shfl_xor_sync(0xffffffffu, acc[v][k], o);
+  __syncthreads();
+  for (int ww = 0; ww < WPB; ++ww) {
+    if (w == ww && lane < G) {
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) {
+          const int col = (v * G + gl) * EPV + k;
+          s_red[col] = (ww == 0 ? 0.f : s_red[col]) + acc[v][k];
+        }
+    }
+    __syncthreads();
+  }
+  for (int d = threadIdx.x; d < D; d += TPB) dst[d] = s_red[d];
+}
+
+struct FwdArgs {
+  DevPart L;
+  const void *feat;
+  int64_t ldf;
+  const float *el, *er;
+  float *lse;
+  int H, F, D;
+  float slope;
+  void *out;
+  int64_t ldo;
+  float *ws_m, *ws_l, *ws_acc;
+};
+
+// ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
+  __shared__ float s_p[WPB][32][SP];
+  __shared__ int s_j[WPB][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int H = a.H;
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
+  const T *feat = static_cast<const T *>(a.feat);
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
+    const int4 item = a.L.fwd_items[it];
+    const int64_t grow = a.L.row_begin + item.x;
+    float elr[MAXH], mrun[MAXH], lrun[MAXH];
+    load_h(a.el + grow * H, H, elr);
+#pragma unroll
+    for (int h = 0; h < MAXH; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
+    float acc[V][EPV];
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+    for (int base = item.y; base < item.z; base += G) {
+      const int e = base + gl;
+      const bool valid = e < item.z;
+      const int j = valid ? ld_stream(a.L.src + e) : 0;
+      float erj[MAXH], sc[MAXH];
+      load_h(a.er + (int64_t)j * H, H, erj);
+#pragma unroll
+      for (int h = 0; h < MAXH; ++h) {
+        sc[h] = 1.f;
+        if (h < H) {
+          const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
+          const float mn = fmaxf(mrun[h], gmax<G>(s, gmask));
+          sc[h] = expf(mrun[h] - mn);
+          const float p = valid ? expf(s - mn) : 0.f;
+          lrun[h] = fmaf(lrun[h], sc[h], p);
+          mrun[h] = mn;
+          s_p[w][lane][h] = p;
+        }
+      }
+      s_j[w][lane] = j;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const float f = sel(sc, hv[v]);
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
+      }
+      __syncwarp(gmask);
+      const int cnt = min(G, item.z - base), rb = grp * G;
+      for (int k0 = 0; k0 < cnt; k0 += U) {
+        uint4 raw[U][V];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (k0 + u < cnt) {
+            const T *rp = feat + (int64_t)s_j[w][rb + k0 + u] * a.ldf + gl * EPV;
+#pragma unroll
+            for (int v = 0; v < V; ++v) raw[u][v] = ldg16(rp + v * G * EPV);
+          }
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (k0 + u < cnt) {
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const float pw = s_p[w][rb + k0 + u][hv[v]];
+              float x[EPV];
+              unpack(raw[u][v], x, T());
+#pragma unroll
+              for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
+            }
+          }
+      }
+      __syncwarp(gmask);
+    }
+    float lt[MAXH];
+#pragma unroll
+    for (int h = 0; h < MAXH; ++h) lt[h] = h < H ? gsum<G>(lrun[h], gmask) : 0.f;
+    if (item.w < 0) {
+      T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const float Lh = sel(lt, hv[v]);
+        const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
+        float y[EPV];
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) y[k] = acc[v][k] * inv;
+        st16(orow + v * G * EPV, pack(y, T()));
+      }
+      for (int h = gl; h < H; h += G) {
+        const float Lh = sel(lt, h);
+        a.lse[grow * H + h] = Lh > 0.f ? sel(mrun, h) + logf(Lh) : -INFINITY;
+      }
+    } else {
+      const int64_t slot = item.w;
+      for (int h = gl; h < H; h += G) {
+        a.ws_m[slot * H + h] = sel(mrun, h);
+        a.ws_l[slot * H + h] = sel(lt, h);
+      }
+      float *pr = a.ws_acc + slot * a.D + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+              make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+    }
+  }
+}
+
+// Merge the partial softmax states of split rows: M = max m_k,
+// L = sum l_k e^{m_k - M}, out = sum acc_k e^{m_k - M} / L, lse = M + log L.
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) gat_fwd_merge_kernel(const FwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const int H = a.H;
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_splits; it += stride) {
+    const int r = a.L.fwd_splits[3 * it], s0 = a.L.fwd_splits[3 * it + 1], ns = a.L.fwd_splits[3 * it + 2];
+    const int64_t grow = a.L.row_begin + r;
+    for (int h = gl; h < H; h += G) {
+      float M = -INFINITY;
+      for (int k = 0; k < ns; ++k) M = fmaxf(M, a.ws_m[(int64_t)(s0 + k) * H + h]);
+      float Ls = 0.f;
+      for (int k = 0; k < ns; ++k) Ls += a.ws_l[(int64_t)(s0 + k) * H + h] * expf(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
+      a.lse[grow * H + h] = M + logf(Ls);
+    }
+    T *orow = static_cast<T *>(a.out) + (int64_t)r * a.ldo;
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const int col = (v * G + gl) * EPV, h = col / a.F;
+      float M = -INFINITY;
+      for (int k = 0; k < ns; ++k) M = fmaxf(M, a.ws_m[(int64_t)(s0 + k) * H + h]);
+      float Ls = 0.f, y[EPV];
+#pragma unroll
+      for (int q = 0; q < EPV; ++q) y[q] = 0.f;
+      for (int k = 0; k < ns; ++k) {
+        const float f = expf(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
+        Ls += a.ws_l[(int64_t)(s0 + k) * H + h] * f;
+        const float *pa = a.ws_acc + (int64_t)(s0 + k) * a.D + col;
+#pragma unroll
+        for (int q = 0; q < EPV; ++q) y[q] = fmaf(f, pa[q], y[q]);
+      }
+      const float inv = 1.f / Ls;
+#pragma unroll
+      for (int q = 0; q < EPV; ++q) y[q] *= inv;
+      st16(orow + col, pack(y, T()));
+    }
+  }
+}
+
+// ---- a2 epilogue (when features did not come from mega_project_fwd): el, er ----
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) eler_kernel(const T *feat, int64_t ldf, int64_t rows, int64_t row0,
+                                                   const float *al, const float *ar, int H, int F, float *el,
+                                                   float *er) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int LPH = F / EPV;
+  float cl[V][EPV], cr[V][EPV];
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int col = (v * G + gl) * EPV;
+    hv[v] = col / F;
+#pragma unroll
+    for (int k = 0; k < EPV; ++k) { cl[v][k] = al[col + k]; cr[v][k] = ar[col + k]; }
+  }
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < rows; r += stride) {
+    float pl[1][V], pr[1][V];
+    const T *rp = feat + r * ldf + gl * EPV;
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      float x[EPV];
+      unpack(ldg16(rp + v * G * EPV), x, T());
+      float sl = 0.f, sr = 0.f;
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) { sl = fmaf(cl[v][k], x[k], sl); sr = fmaf(cr[v][k], x[k], sr); }
+      pl[0][v] = sl; pr[0][v] = sr;
+    }
+    head_reduce<G, 1, V>(pl, LPH, gmask);
+    head_reduce<G, 1, V>(pr, LPH, gmask);
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+      if (head_lead<G>(gl, v, LPH)) {
+        el[(row0 + r) * H + hv[v]] = pl[0][v];
+        er[(row0 + r) * H + hv[v]] = pr[0][v];
+      }
+  }
+}
+
+struct BwdArgs {
+  DevPart L;
+  const void *feat;
+  int64_t ldf;
+  const float *al, *ar;
+  int H, F, D;
+  float slope;
+  const void *out;
+  int64_t ldo;
+  const void *gout;
+  int64_t ldg;
+  const float *el, *er, *lse;
+  float *dlt;
+  float *gfeat;
+  int64_t ldgf;
+  void *gfeat_lp;
+  int64_t ldlp;
+  float *dz, *ws_bacc, *ws_bder, *ws_dar, *ws_dar2, *ws_dal;
+  float *gal, *gar;
+  int nb_src, nb_merge, nb_dst;
+};
+
+// ---- a6: Dlt_i = g_i . out_i ----
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int LPH = a.F / EPV, H = a.H;
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
+    const T *gr = static_cast<const T *>(a.gout) + r * a.ldg + gl * EPV;
+    const T *orr = static_cast<const T *>(a.out) + r * a.ldo + gl * EPV;
+    float p[1][V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      float x[EPV], y[EPV];
+      unpack(ldg16(gr + v * G * EPV), x, T());
+      unpack(ldg16(orr + v * G * EPV), y, T());
+      float s = 0.f;
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
+      p[0][v] = s;
+    }
+    head_reduce<G, 1, V>(p, LPH, gmask);
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+      if (head_lead<G>(gl, v, LPH)) a.dlt[(a.L.row_begin + r) * H + ((v * G + gl) * EPV) / a.F] = p[0][v];
+  }
+}
+
+// ---- a7: source-major pass over the CSC ----
+// For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
+// dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
+// dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge.
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
+  __shared__ float s_a[WPB][32][SP];  // alpha, sign = (z > 0)
+  __shared__ float s_d[WPB][32][SP];  // Dlt_i
+  __shared__ float s_z[WPB][32][SP];  // dz out
+  __shared__ int s_i[WPB][32];
+  __shared__ float s_red[1024];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int H = a.H, LPH = a.F / EPV;
+  int hv[V];
+  float arv[V][EPV], dar[V][EPV];
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int col = (v * G + gl) * EPV;
+    hv[v] = col / a.F;
+#pragma unroll
+    for (int k = 0; k < EPV; ++k) { arv[v][k] = a.ar[col + k]; dar[v][k] = 0.f; }
+  }
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *gout = static_cast<const T *>(a.gout);
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
+    const int4 item = a.L.bwd_items[it];
+    const int64_t j = item.x;
+    float whv[V][EPV], acc[V][EPV], derv[V];
+    {
+      const T *rp = feat + j * a.ldf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        unpack(ldg16(rp + v * G * EPV), whv[v], T());
+        derv[v] = 0.f;
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+      }
+    }
+    float erj[MAXH];
+    load_h(a.er + j * H, H, erj);
+    for (int base = item.y; base < item.z; base += G) {
+      const int c = base + gl;
+      const bool valid = c < item.z;
+      const int i = valid ? ld_stream(a.L.cdst + c) : 0;
+      const int64_t gi = a.L.row_begin + i;
+      float eli[MAXH], lsei[MAXH], dli[MAXH];
+      load_h(a.el + gi * H, H, eli);
+      load_h(a.lse + gi * H, H, lsei);
+      load_h(a.dlt + gi * H, H, dli);
+#pragma unroll
+      for (int h = 0; h < MAXH; ++h)
+        if (h < H) {
+          const float z = eli[h] + erj[h];
+          const float al = valid ? expf(leaky(z, a.slope) - lsei[h]) : 0.f;
+          s_a[w][lane][h] = z > 0.f ? al : -al;
+          s_d[w][lane][h] = dli[h];
+        }
+      s_i[w][lane] = i;
+      __syncwarp(gmask);
+      const int cnt = min(G, item.z - base), rb = grp * G;
+      for (int k0 = 0; k0 < cnt; k0 += U) {
+        uint4 raw[U][V];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (k0 + u < cnt) {
+            const T *rp = gout + (int64_t)s_i[w][rb + k0 + u] * a.ldg + gl * EPV;
+#pragma unroll
+            for (int v = 0; v < V; ++v) raw[u][v] = ldg16(rp + v * G * EPV);
+          } else {
+#pragma unroll
+            for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
+          }
+        float p[U][V];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            float x[EPV];
+            unpack(raw[u][v], x, T());
+            float s = 0.f;
+#pragma unroll
+            for (int k = 0; k < EPV; ++k) s = fmaf(x[k], whv[v][k], s);
+            p[u][v] = s;
+          }
+        head_reduce<G, U, V>(p, LPH, gmask);
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+          if (k0 + u < cnt) {
+            const int er_ = rb + k0 + u;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const float sa = s_a[w][er_][hv[v]];
+              const float al = fabsf(sa);
+              const float dz = al * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+              derv[v] += dz;
+              float x[EPV];
+              unpack(raw[u][v], x, T());
+#pragma unroll
+              for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[k], acc[v][k]);
+              if (head_lead<G>(gl, v, LPH)) s_z[w][er_][hv[v]] = dz;
+            }
+          }
+      }
+      __syncwarp(gmask);
+      if (valid) {
+        float *dzp = a.dz + (int64_t)c * H;
+        if ((H & 3) == 0) {
+#pragma unroll
+          for (int q = 0; q < MAXH / 4; ++q)
+            if (4 * q < H)
+              reinterpret_cast<float4 *>(dzp)[q] = make_float4(s_z[w][lane][4 * q], s_z[w][lane][4 * q + 1],
+                                                               s_z[w][lane][4 * q + 2], s_z[w][lane][4 * q + 3]);
+        } else {
+          for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
+        }
+      }
+      __syncwarp(gmask);
+    }
+    if (item.w < 0) {
+      float *orow = a.gfeat + j * a.ldgf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) =
+              make_float4(fmaf(derv[v], arv[v][k], acc[v][k]), fmaf(derv[v], arv[v][k + 1], acc[v][k + 1]),
+                          fmaf(derv[v], arv[v][k + 2], acc[v][k + 2]), fmaf(derv[v], arv[v][k + 3], acc[v][k + 3]));
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) dar[v][k] = fmaf(derv[v], whv[v][k], dar[v][k]);
+      }
+    } else {
+      const int64_t slot = item.w;
+      float *pr = a.ws_bacc + slot * a.D + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+              make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+        if (head_lead<G>(gl, v, LPH)) a.ws_bder[slot * H + hv[v]] = derv[v];
+      }
+    }
+  }
+  block_partial<G, V, EPV>(dar, s_red, a.ws_dar + (int64_t)blockIdx.x * a.D, a.D);
+}
+
+// Split sources: dWh_j = sum_k acc_k + (sum_k der_k) a_r; da_r += der_j Wh_j.
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  __shared__ float s_red[1024];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const int H = a.H;
+  float dar[V][EPV];
+#pragma unroll
+  for (int v = 0; v < V; ++v)
+#pragma unroll
+    for (int k = 0; k < EPV; ++k) dar[v][k] = 0.f;
+  const T *feat = static_cast<const T *>(a.feat);
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_splits; it += stride) {
+    const int64_t j = a.L.bwd_splits[3 * it];
+    const int s0 = a.L.bwd_splits[3 * it + 1], ns = a.L.bwd_splits[3 * it + 2];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const int col = (v * G + gl) * EPV, h = col / a.F;
+      float der = 0.f, y[EPV], wh[EPV];
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) y[k] = 0.f;
+      for (int s = 0; s < ns; ++s) {
+        der += a.ws_bder[(int64_t)(s0 + s) * H + h];
+        const float *pa = a.ws_bacc + (int64_t)(s0 + s) * a.D + col;
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) y[k] += pa[k];
+      }
+      unpack(ldg16(feat + j * a.ldf + col), wh, T());
+      float *orow = a.gfeat + j * a.ldgf + col;
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) {
+        orow[k] = fmaf(der, a.ar[col + k], y[k]);
+        dar[v][k] = fmaf(der, wh[k], dar[v][k]);
+      }
+    }
+  }
+  block_partial<G, V, EPV>(dar, s_red, a.ws_dar2 + (int64_t)blockIdx.x * a.D, a.D);
+}
+
+// ---- a8: destination pass: del_i = sum_In dz; dWh_i += del_i a_l; da_l += del_i Wh_i ----
+template <typename T, int G, int V>
+__global__ void __launch_bounds__(TPB) gat_bwd_dst_kernel(const BwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  __shared__ float s_red[1024];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int H = a.H;
+  int hv[V];
+  float alv[V][EPV], dal[V][EPV];
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int col = (v * G + gl) * EPV;
+    hv[v] = col / a.F;
+#pragma unroll
+    for (int k = 0; k < EPV; ++k) { alv[v][k] = a.al[col + k]; dal[v][k] = 0.f; }
+  }
+  const T *feat = static_cast<const T *>(a.feat);
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
+    const int e0 = a.L.indptr[r], e1 = a.L.indptr[r + 1];
+    float dp[MAXH];
+#pragma unroll
+    for (int h = 0; h < MAXH; ++h) dp[h] = 0.f;
+    for (int e = e0 + gl; e < e1; e += G) {
+      float t[MAXH];
+      load_h(a.dz + (int64_t)ld_stream(a.L.csr2csc + e) * H, H, t);
+#pragma unroll
+      for (int h = 0; h < MAXH; ++h)
+        if (h < H) dp[h] += t[h];
+    }
+    float del[MAXH];
+#pragma unroll
+    for (int h = 0; h < MAXH; ++h) del[h] = h < H ? gsum<G>(dp[h], gmask) : 0.f;
+    const int64_t grow = a.L.row_begin + r;
+    float *gr = a.gfeat + grow * a.ldgf + gl * EPV;
+    const T *wr = feat + grow * a.ldf + gl * EPV;
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const float d = sel(del, hv[v]);
+      float y[EPV], wh[EPV];
+      unpack(ldg16(wr + v * G * EPV), wh, T());
+#pragma unroll
+      for (int k = 0; k < EPV; k += 4) {
+        float4 t = *reinterpret_cast<const float4 *>(gr + v * G * EPV + k);
+        y[k] = fmaf(d, alv[v][k], t.x); y[k + 1] = fmaf(d, alv[v][k + 1], t.y);
+        y[k + 2] = fmaf(d, alv[v][k + 2], t.z); y[k + 3] = fmaf(d, alv[v][k + 3], t.w);
+        *reinterpret_cast<float4 *>(gr + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+      }
+      if (a.gfeat_lp) st16(static_cast<T *>(a.gfeat_lp) + grow * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) dal[v][k] = fmaf(d, wh[k], dal[v][k]);
+    }
+  }
+  block_partial<G, V, EPV>(dal, s_red, a.ws_dal + (int64_t)blockIdx.x * a.D, a.D);
+}
+
+// Second stage of the parameter-gradient reductions (fixed order).
+__global__ void param_reduce_kernel(const float *parts, int nparts, const float *parts2, int nparts2, int D,
+                                    float *out) {
+  for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < D; d += gridDim.x * blockDim.x) {
+    float s = 0.f;
+    for (int b = 0; b < nparts; ++b) s += parts[(int64_t)b * D + d];
+    for (int b = 0; b < nparts2; ++b) s += parts2[(int64_t)b * D + d];
+    out[d] = s;
+  }
+}
+
+}  // namespace kern
+
+// ============================ host side ============================
+namespace {
+using namespace kern;
+
+template <int X> using IC = std::integral_constant<int, X>;
+
+// (G, V) for a row of `nv` 16-byte vectors.
+template <typename Fn>
+bool dispatch_gv(int nv, Fn &&fn) {
+  switch (nv) {
+    case 1: fn(IC<1>(), IC<1>()); return true;
+    case 2: fn(IC<2>(), IC<1>()); return true;
+    case 4: fn(IC<4>(), IC<1>()); return true;
+    case 8: fn(IC<8>(), IC<1>()); return true;
+    case 16: fn(IC<16>(), IC<1>()); return true;
+    case 32: fn(IC<32>(), IC<1>()); return true;
+    case 64: fn(IC<32>(), IC<2>()); return true;
+    case 128: fn(IC<32>(), IC<4>()); return true;
+    case 256: fn(IC<32>(), IC<8>()); return true;
+    default: return false;
+  }
+}
+
+struct DevInfo { int sms = 0; int major = 0; };
+DevInfo dev_info(int dev) {
+  static std::mutex mu;
+  static std::unordered_map<int, DevInfo> cache;
+  std::lock_guard<std::mutex> g(mu);
+  auto it = cache.find(dev);
+  if (it != cache.end()) return it->second;
+  DevInfo d;
+  cudaDeviceGetAttribute(&d.sms, cudaDevAttrMultiProcessorCount, dev);
+  cudaDeviceGetAttribute(&d.major, cudaDevAttrComputeCapabilityMajor, dev);
+  cache[dev] = d;
+  return d;
+}
+
+template <typename K>
+int grid_for(K kernel, int64_t groups, int gpw, int dev) {
+  static std::mutex mu;
+  static std::unordered_map<const void *, int> occ;
+  int per_sm;
+  {
+    std::lock_guard<std::mutex> g(mu);
+    auto it = occ.find((const void *)kernel);
+    if (it == occ.end()) {
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, TPB, 0);
+      occ[(const void *)kernel] = nb > 0 ? nb : 1;
+      per_sm = nb > 0 ? nb : 1;
+    } else {
+      per_sm = it->second;
+    }
+  }
+  const int64_t need = (groups + (int64_t)WPB * gpw - 1) / ((int64_t)WPB * gpw);
+  int64_t g = std::min<int64_t>(need, (int64_t)per_sm * dev_info(dev).sms);
+  g = std::min<int64_t>(g, MAX_GRID);
+  return (int)std::max<int64_t>(g, 1);
+}
+
+bool debug_sync() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_DEBUG_SYNC");
+    v = (e && e[0] == '1') ? 1 : 0;
+  }
+  return v == 1;
+}
+
+mega_status check_launch(cudaStream_t s, const char *what) {
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+  if (debug_sync()) {
+    e = cudaStreamSynchronize(s);
+    if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + " (sync): " + cudaGetErrorString(e));
+  }
+  return MEGA_OK;
+}
+
+size_t align256(size_t x) { return (x + 255) / 256 * 256; }
+
+struct Shape {
+  int H, F, D, epv, nv, G, V;
+};
+
+mega_status check_shape(int heads, int head_dim, mega_dtype dtype, Shape &s) {
+  if (dtype != MEGA_F32 && dtype != MEGA_BF16) return fail(MEGA_ERR_INVALID_ARGUMENT, "dtype must be MEGA_F32 or MEGA_BF16");
+  if (heads < 1 || heads > MAXH) return fail(MEGA_ERR_UNSUPPORTED, "heads must be in [1, 8]");
+  if (head_dim < 1) return fail(MEGA_ERR_INVALID_ARGUMENT, "head_dim must be >= 1");
+  s.H = heads; s.F = head_dim; s.D = heads * head_dim;
+  s.epv = dtype == MEGA_BF16 ? 8 : 4;
+  if (head_dim % s.epv) return fail(MEGA_ERR_UNSUPPORTED, "head_dim must be a multiple of 8 (bf16) / 4 (fp32)");
+  if (s.D > 1024) return fail(MEGA_ERR_UNSUPPORTED, "heads*head_dim must be <= 1024");
+  s.nv = s.D / s.epv;
+  bool ok = dispatch_gv(s.nv, [&](auto g, auto v) { s.G = decltype(g)::value; s.V = decltype(v)::value; });
+  if (!ok) return fail(MEGA_ERR_UNSUPPORTED, "D/EPV must be a power of two <= 32 or 64/128/256");
+  const int lph = s.F / s.epv;
+  if (lph <= s.G) {
+    if ((lph & (lph - 1)) || s.G % lph) return fail(MEGA_ERR_UNSUPPORTED, "head_dim/EPV must be a power of two");
+  } else if (lph % s.G || s.V % (lph / s.G)) {
+    return fail(MEGA_ERR_UNSUPPORTED, "unsupported head_dim for this row width");
+  }
+  return MEGA_OK;
+}
+
+bool al16(const void *p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; }
+
+mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
+  if (!L) return fail(MEGA_ERR_INVALID_ARGUMENT, "null layout");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(e));
+  if (dev_info(dev).major != 10) return fail(MEGA_ERR_UNSUPPORTED, "libmega.so kernels require an sm_100 (B200) device");
+  const Part &P = L->parts[part];
+  if (!P.dev_base) return fail(MEGA_ERR_STATE, "layout part not bound (mega_layout_bind_device)");
+  if (P.device != dev) return fail(MEGA_ERR_STATE, "layout part bound to another device");
+  return MEGA_OK;
+}
+
+struct WsFwd { size_t m, l, acc, total; };
+WsFwd ws_fwd(const DevPart &D, const Shape &s) {
+  WsFwd w;
+  size_t slots = (size_t)std::max(1, D.n_fwd_slots);
+  w.m = 0;
+  w.l = align256(w.m + slots * s.H * 4);
+  w.acc = align256(w.l + slots * s.H * 4);
+  w.total = align256(w.acc + slots * s.D * 4);
+  return w;
+}
+struct WsBwd { size_t dz, bacc, bder, dar, dar2, dal, total; };
+WsBwd ws_bwd(const DevPart &D, const Shape &s) {
+  WsBwd w;
+  size_t slots = (size_t)std::max(1, D.n_bwd_slots);
+  w.dz = 0;
+  w.bacc = align256(w.dz + (size_t)std::max<int64_t>(1, D.edges) * s.H * 4);
+  w.bder = align256(w.bacc + slots * s.D * 4);
+  w.dar = align256(w.bder + slots * s.H * 4);
+  w.dar2 = align256(w.dar + (size_t)MAX_GRID * s.D * 4);
+  w.dal = align256(w.dar2 + (size_t)MAX_GRID * s.D * 4);
+  w.total = align256(w.dal + (size_t)MAX_GRID * s.D * 4);
+  return w;
+}
+DevPart host_counts(const Part &P, int64_t n) {  // sizes without binding
+  DevPart D;
+  D.n = n;
+  D.rows = P.row_end - P.row_begin;
+  D.edges = (int64_t)P.src.size();
+  D.n_fwd_slots = P.n_fwd_slots;
+  D.n_bwd_slots = P.n_bwd_slots;
+  return D;
+}
+
+template <typename T>
+mega_status launch_eler(const void *feat, int64_t ldf, int64_t rows, int64_t row0, const float *al, const float *ar,
+                        const Shape &s, float *el, float *er, cudaStream_t st, int dev) {
+  mega_status rc = MEGA_OK;
+  dispatch_gv(s.nv, [&](auto g, auto v) {
+    constexpr int G = decltype(g)::value, V = decltype(v)::value;
+    auto k = eler_kernel<T, G, V>;
+    const int grid = grid_for(k, rows, 32 / G, dev);
+    k<<<grid, TPB, 0, st>>>(static_cast<const T *>(feat), ldf, rows, row0, al, ar, s.H, s.F, el, er);
+    rc = check_launch(st, "eler_kernel");
+  });
+  return rc;
+}
+
+}  // namespace
+
+// internal entry used by project.cu
+mega_status launch_eler_any(mega_dtype dt, const void *feat, int64_t ldf, int64_t rows, int64_t row0, const float *al,
+                            const float *ar, int heads, int head_dim, float *el, float *er, cudaStream_t st) {
+  Shape s;
+  mega_status rc = check_shape(heads, head_dim, dt, s);
+  if (rc != MEGA_OK) return rc;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  if (rows == 0) return MEGA_OK;
+  return dt == MEGA_BF16 ? launch_eler<__nv_bfloat16>(feat, ldf, rows, row0, al, ar, s, el, er, st, dev)
+                         : launch_eler<float>(feat, ldf, rows, row0, al, ar, s, el, er, st, dev);
+}
+
+namespace {
+template <typename T>
+mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) {
+  mega_status rc = MEGA_OK;
+  dispatch_gv(s.nv, [&](auto g, auto v) {
+    constexpr int G = decltype(g)::value, V = decltype(v)::value;
+    if (a.L.n_fwd_items > 0) {
+      auto k = gat_fwd_kernel<T, G, V>;
+      k<<<grid_for(k, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+      rc = check_launch(st, "gat_fwd_kernel");
+      if (rc != MEGA_OK) return;
+    }
+    if (a.L.n_fwd_splits > 0) {
+      auto k = gat_fwd_merge_kernel<T, G, V>;
+      k<<<grid_for(k, a.L.n_fwd_splits, 32 / G, dev), TPB, 0, st>>>(a);
+      rc = check_launch(st, "gat_fwd_merge_kernel");
+    }
+  });
+  return rc;
+}
+
+template <typename T>
+mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, int dev) {
+  mega_status rc = MEGA_OK;
+  const bool src_phase = (flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) == 0 || (flags & MEGA_BWD_PHASE_SRC);
+  const bool dst_phase = (flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) == 0 || (flags & MEGA_BWD_PHASE_DST);
+  dispatch_gv(s.nv, [&](auto g, auto v) {
+    constexpr int G = decltype(g)::value, V = decltype(v)::value;
+    if (src_phase) {
+      if (a.L.rows > 0) {
+        auto k = dlt_kernel<T, G, V>;
+        k<<<grid_for(k, a.L.rows, 32 / G, dev), TPB, 0, st>>>(a);
+        if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
+      }
+      auto ks = gat_bwd_src_kernel<T, G, V>;
+      a.nb_src = grid_for(ks, std::max(1, a.L.n_bwd_items), 32 / G, dev);
+      ks<<<a.nb_src, TPB, 0, st>>>(a);
+      if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
+      a.nb_merge = 0;
+      if (a.L.n_bwd_splits > 0) {
+        auto km = gat_bwd_src_merge_kernel<T, G, V>;
+        a.nb_merge = grid_for(km, a.L.n_bwd_splits, 32 / G, dev);
+        km<<<a.nb_merge, TPB, 0, st>>>(a);
+        if ((rc = check_launch(st, "gat_bwd_src_merge_kernel")) != MEGA_OK) return;
+      }
+      param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dar, a.nb_src, a.ws_dar2, a.nb_merge, s.D, a.gar);
+      if ((rc = check_launch(st, "param_reduce_kernel(a_r)")) != MEGA_OK) return;
+    }
+    if (dst_phase) {
+      auto kd = gat_bwd_dst_kernel<T, G, V>;
+      a.nb_dst = grid_for(kd, std::max<int64_t>(1, a.L.rows), 32 / G, dev);
+      kd<<<a.nb_dst, TPB, 0, st>>>(a);
+      if ((rc = check_launch(st, "gat_bwd_dst_kernel")) != MEGA_OK) return;
+      param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dal, a.nb_dst, nullptr, 0, s.D, a.gal);
+      rc = check_launch(st, "param_reduce_kernel(a_l)");
+    }
+  });
+  return rc;
+}
+}  // namespace
+}  // namespace mega
+
+using namespace mega;
+
+extern "C" {
+
+mega_status mega_gat_workspace_bytes(const mega_layout *L, int32_t part, int heads, int head_dim, mega_dtype dtype,
+                                     size_t *fwd_ws, size_t *bwd_ws) {
+  clear_error();
+  if (!L || !fwd_ws || !bwd_ws) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  Shape s;
+  mega_status rc = check_shape(heads, head_dim, dtype, s);
+  if (rc != MEGA_OK) return rc;
+  DevPart D = host_counts(L->parts[part], L->n);
+  *fwd_ws = ws_fwd(D, s).total;
+  *bwd_ws = ws_bwd(D, s).total;
+  return MEGA_OK;
+}
+
+mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, int64_t ldf, const float *attn_l,
+                         const float *attn_r, int heads, int head_dim, mega_dtype dtype, float negative_slope,
+                         uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws, size_t ws_bytes,
+                         mega_stream_t stream) {
+  clear_error();
+  int dev = 0;
+  mega_status rc = check_part(L, part, dev);
+  if (rc != MEGA_OK) return rc;
+  Shape s;
+  if ((rc = check_shape(heads, head_dim, dtype, s)) != MEGA_OK) return rc;
+  if (!feat || !attn_l || !attn_r || !out || !ctx || !ws) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  const int esz = dtype == MEGA_BF16 ? 2 : 4;
+  if (ldf < s.D || ldo < s.D || (ldf * esz) % 16 || (ldo * esz) % 16)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "ldf/ldo must be >= D and a multiple of 16 bytes");
+  if (!al16(feat) || !al16(out) || !al16(ctx) || !al16(ws)) return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
+  const Part &P = L->parts[part];
+  const WsFwd w = ws_fwd(P.dev, s);
+  if (ws_bytes < w.total) return fail(MEGA_ERR_OUT_OF_MEMORY, "fwd workspace too small");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t n = L->n, plane = n * s.H;
+  if (!(flags & MEGA_FLAG_ELER_IN_CTX)) {
+    rc = launch_eler_any(dtype, feat, ldf, n, 0, attn_l, attn_r, heads, head_dim, ctx, ctx + plane, st);
+    if (rc != MEGA_OK) return rc;
+  }
+  kern::FwdArgs a;
+  a.L = P.dev;
+  a.feat = feat; a.ldf = ldf;
+  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane;
+  a.H = s.H; a.F = s.F; a.D = s.D; a.slope = negative_slope;
+  a.out = out; a.ldo = ldo;
+  char *wb = static_cast<char *>(ws);
+  a.ws_m = reinterpret_cast<float *>(wb + w.m);
+  a.ws_l = reinterpret_cast<float *>(wb + w.l);
+  a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
+  return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
+}
+
+mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, int64_t ldf, const float *attn_l,
+                         const float *attn_r, int heads, int head_dim, mega_dtype dtype, float negative_slope,
+                         uint32_t flags, const void *out, int64_t ldo, const void *grad_out, int64_t ldg, float *ctx,
+                         float *grad_feat, int64_t ldgf, void *grad_feat_lp, int64_t ldlp, float *grad_attn_l,
+                         float *grad_attn_r, void *ws, size_t ws_bytes, mega_stream_t stream) {
+  clear_error();
+  int dev = 0;
+  mega_status rc = check_part(L, part, dev);
+  if (rc != MEGA_OK) return rc;
+  Shape s;
+  if ((rc = check_shape(heads, head_dim, dtype, s)) != MEGA_OK) return rc;
+  if (!feat || !attn_l || !attn_r || !out || !grad_out || !ctx || !grad_feat || !grad_attn_l || !grad_attn_r || !ws)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  const int esz = dtype == MEGA_BF16 ? 2 : 4;
+  if (ldf < s.D || ldo < s.D || ldg < s.D || ldgf < s.D || (ldf * esz) % 16 || (ldo * esz) % 16 || (ldg * esz) % 16 ||
+      (ldgf * 4) % 16)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "leading dimensions must be >= D and multiples of 16 bytes");
+  if (grad_feat_lp && (ldlp < s.D || (ldlp * esz) % 16 || !al16(grad_feat_lp)))
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "grad_feat_lp: bad ld or alignment");
+  if (!al16(feat) || !al16(out) || !al16(grad_out) || !al16(ctx) || !al16(grad_feat) || !al16(ws))
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
+  const Part &P = L->parts[part];
+  const WsBwd w = ws_bwd(P.dev, s);
+  if (ws_bytes < w.total) return fail(MEGA_ERR_OUT_OF_MEMORY, "bwd workspace too small");
+  const int64_t plane = L->n * s.H;
+  kern::BwdArgs a;
+  a.L = P.dev;
+  a.feat = feat; a.ldf = ldf; a.al = attn_l; a.ar = attn_r;
+  a.H = s.H; a.F = s.F; a.D = s.D; a.slope = negative_slope;
+  a.out = out; a.ldo = ldo; a.gout = grad_out; a.ldg = ldg;
+  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane; a.dlt = ctx + 3 * plane;
+  a.gfeat = grad_feat; a.ldgf = ldgf; a.gfeat_lp = grad_feat_lp; a.ldlp = ldlp;
+  char *wb = static_cast<char *>(ws);
+  a.dz = reinterpret_cast<float *>(wb + w.dz);
+  a.ws_bacc = reinterpret_cast<float *>(wb + w.bacc);
+  a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
+  a.ws_dar = reinterpret_cast<float *>(wb + w.dar);
+  a.ws_dar2 = reinterpret_cast<float *>(wb + w.dar2);
+  a.ws_dal = reinterpret_cast<float *>(wb + w.dal);
+  a.gal = grad_attn_l; a.gar = grad_attn_r;
+  a.nb_src = a.nb_merge = a.nb_dst = 0;
+  cudaStream_t st = (cudaStream_t)stream;
+  return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
+}
+
+}  // extern "C"

@@ -1,0 +1,267 @@
+"""Thin Python binding of libmega.so (include/mega.h) — argument marshalling only.
+
+Every function here has the name of the C entry point it calls.  PyTorch is
+used for device memory and streams only; every step of the hot path runs in
+libmega.so's kernels.  There is no fallback: if libmega.so is missing or the
+device is not an sm_100 GPU the calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libmega.so")
+
+MEGA_F32, MEGA_BF16 = 0, 1
+ORDERS = {"traversal": 0, "identity": 1, "degree": 2, "random": 3}
+MEGA_FLAG_ELER_IN_CTX = 1
+MEGA_BWD_PHASE_SRC = 2
+MEGA_BWD_PHASE_DST = 4
+SLOPE = float(np.float32(0.2))
+
+_c = ctypes
+P = _c.c_void_p
+I64 = _c.c_int64
+
+
+class MegaError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{status_name(status)}: {msg}")
+        self.status = status
+
+
+class mega_csr(_c.Structure):
+    _fields_ = [("num_nodes", _c.c_int64), ("num_edges", _c.c_int64), ("indptr", P), ("indices", P)]
+
+
+class mega_schedule_opts(_c.Structure):
+    _fields_ = [("struct_size", _c.c_uint32), ("window", _c.c_int32), ("candidate_cap", _c.c_int32),
+                ("order", _c.c_int32), ("seg_edges", _c.c_int32), ("num_parts", _c.c_int32),
+                ("seed", _c.c_uint64)]
+
+
+class mega_layout_stats(_c.Structure):
+    _fields_ = [("struct_size", _c.c_uint32)] + [(k, _c.c_int64) for k in (
+        "num_nodes", "num_edges", "num_parts", "window", "candidate_cap", "seg_edges", "order", "path_length",
+        "revisits", "jumps", "tile_unique_sources", "max_in_degree", "max_out_degree")] + [
+        ("preprocess_seconds", _c.c_double)]
+
+
+_VIEW_INTS = ("num_nodes", "num_edges", "row_begin", "row_end", "part_edges", "num_fwd_items", "num_fwd_splits",
+              "num_bwd_items", "num_bwd_splits", "num_parts")
+_VIEW_PTRS = ("perm", "new_of_old", "bounds", "indptr", "src", "eid", "cindptr", "cdst", "cpos", "csr2csc",
+              "fwd_items", "fwd_splits", "bwd_items", "bwd_splits")
+
+
+class mega_layout_view(_c.Structure):
+    _fields_ = [("struct_size", _c.c_uint32)] + [(k, _c.c_int64) for k in _VIEW_INTS] + [
+        (k, _c.POINTER(_c.c_int32)) for k in _VIEW_PTRS]
+
+
+_lib = None
+
+
+def lib():
+    """Load libmega.so (fails loudly if it has not been built)."""
+    global _lib
+    if _lib is None:
+        if not os.path.exists(LIB_PATH):
+            raise ImportError(f"{LIB_PATH} is missing: build it with "
+                              "`python -m paper_conf_icdcs_dengr24_b200.build` (no CPU fallback exists)")
+        L = _c.CDLL(LIB_PATH)
+        S = _c.c_int
+        sig = {
+            "mega_abi_version": (_c.c_int, []),
+            "mega_status_string": (_c.c_char_p, [S]),
+            "mega_last_error": (_c.c_char_p, []),
+            "mega_schedule_opts_init": (None, [P]),
+            "mega_preprocess": (S, [P, P, P]),
+            "mega_layout_destroy": (None, [P]),
+            "mega_layout_stats_get": (S, [P, P]),
+            "mega_layout_view_get": (S, [P, _c.c_int32, P]),
+            "mega_layout_save": (S, [P, _c.c_char_p]),
+            "mega_layout_load": (S, [_c.c_char_p, P]),
+            "mega_layout_device_bytes": (S, [P, _c.c_int32, P]),
+            "mega_layout_bind_device": (S, [P, _c.c_int32, P, _c.c_size_t, P]),
+            "mega_gat_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, _c.c_int, S, P, P]),
+            "mega_project_fwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, P, P, S, P, I64, P, I64, I64, P]),
+            "mega_gat_fwd": (S, [P, _c.c_int32, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64,
+                                 P, P, _c.c_size_t, P]),
+            "mega_gat_bwd": (S, [P, _c.c_int32, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64,
+                                 P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P]),
+            "mega_project_bwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, S, P, I64, P, I64, P, P]),
+        }
+        for name, (res, args) in sig.items():
+            f = getattr(L, name)
+            f.restype = res
+            f.argtypes = args
+        _lib = L
+    return _lib
+
+
+def status_name(s):
+    return lib().mega_status_string(s).decode()
+
+
+def _check(status):
+    if status != 0:
+        raise MegaError(status, lib().mega_last_error().decode())
+
+
+def mega_abi_version():
+    return lib().mega_abi_version()
+
+
+class Layout:
+    """Owns a mega_layout* and the device images bound to it."""
+
+    def __init__(self, handle):
+        self._h = _c.c_void_p(handle)
+        self._dev = {}
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.mega_layout_destroy(self._h)
+            self._h = _c.c_void_p(None)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def stats(self):
+        return mega_layout_stats_get(self)
+
+    def view(self, part=0):
+        return mega_layout_view_get(self, part)
+
+    def bind(self, part=0, stream=None):
+        return mega_layout_bind_device(self, part, stream)
+
+
+def mega_preprocess(indptr, indices, window=0, candidate_cap=0, order="traversal", seg_edges=0, num_parts=1,
+                    seed=0) -> Layout:
+    indptr = np.ascontiguousarray(indptr, dtype=np.int64)
+    indices = np.ascontiguousarray(indices, dtype=np.int32)
+    csr = mega_csr(len(indptr) - 1, len(indices), indptr.ctypes.data, indices.ctypes.data)
+    o = mega_schedule_opts()
+    lib().mega_schedule_opts_init(_c.byref(o))
+    o.window, o.candidate_cap, o.seg_edges, o.num_parts, o.seed = window, candidate_cap, seg_edges, num_parts, seed
+    o.order = ORDERS[order] if isinstance(order, str) else int(order)
+    h = _c.c_void_p()
+    _check(lib().mega_preprocess(_c.byref(csr), _c.byref(o), _c.byref(h)))
+    return Layout(h.value)
+
+
+def mega_layout_stats_get(layout: Layout) -> dict:
+    st = mega_layout_stats()
+    _check(lib().mega_layout_stats_get(layout.handle, _c.byref(st)))
+    return {k: getattr(st, k) for k, _ in mega_layout_stats._fields_ if k != "struct_size"}
+
+
+def mega_layout_view_get(layout: Layout, part: int = 0) -> dict:
+    """Copies of the host arrays of one part (numpy int32)."""
+    v = mega_layout_view()
+    _check(lib().mega_layout_view_get(layout.handle, part, _c.byref(v)))
+    d = {k: getattr(v, k) for k in _VIEW_INTS}
+    n, rows, e = v.num_nodes, v.row_end - v.row_begin, v.part_edges
+    sizes = {"perm": n, "new_of_old": n, "bounds": v.num_parts + 1, "indptr": rows + 1, "src": e, "eid": e,
+             "cindptr": n + 1, "cdst": e, "cpos": e, "csr2csc": e, "fwd_items": 4 * v.num_fwd_items,
+             "fwd_splits": 3 * v.num_fwd_splits, "bwd_items": 4 * v.num_bwd_items,
+             "bwd_splits": 3 * v.num_bwd_splits}
+    for k in _VIEW_PTRS:
+        ptr = getattr(v, k)
+        d[k] = np.ctypeslib.as_array(ptr, shape=(sizes[k],)).copy() if sizes[k] > 0 else np.zeros(0, np.int32)
+    d["fwd_items"] = d["fwd_items"].reshape(-1, 4)
+    d["bwd_items"] = d["bwd_items"].reshape(-1, 4)
+    d["fwd_splits"] = d["fwd_splits"].reshape(-1, 3)
+    d["bwd_splits"] = d["bwd_splits"].reshape(-1, 3)
+    return d
+
+
+def mega_layout_save(layout: Layout, path: str):
+    _check(lib().mega_layout_save(layout.handle, path.encode()))
+
+
+def mega_layout_load(path: str) -> Layout:
+    h = _c.c_void_p()
+    _check(lib().mega_layout_load(path.encode(), _c.byref(h)))
+    return Layout(h.value)
+
+
+def mega_layout_device_bytes(layout: Layout, part: int = 0) -> int:
+    b = _c.c_size_t()
+    _check(lib().mega_layout_device_bytes(layout.handle, part, _c.byref(b)))
+    return b.value
+
+
+def _stream(stream):
+    import torch
+    s = torch.cuda.current_stream() if stream is None else stream
+    return _c.c_void_p(s.cuda_stream)
+
+
+def _ptr(t):
+    return None if t is None else _c.c_void_p(t.data_ptr())
+
+
+def mega_layout_bind_device(layout: Layout, part: int = 0, stream=None):
+    """Allocates the part's device image on the current device (torch) and copies it."""
+    import torch
+    nbytes = mega_layout_device_bytes(layout, part)
+    buf = torch.empty(max(nbytes, 256) + 256, dtype=torch.uint8, device="cuda")
+    off = (-buf.data_ptr()) % 256
+    view = buf[off:off + max(nbytes, 256)]
+    _check(lib().mega_layout_bind_device(layout.handle, part, _c.c_void_p(view.data_ptr()), nbytes, _stream(stream)))
+    layout._dev[part] = buf
+    return buf
+
+
+def _dtype_code(t):
+    import torch
+    if t.dtype == torch.bfloat16:
+        return MEGA_BF16
+    if t.dtype == torch.float32:
+        return MEGA_F32
+    raise TypeError(f"unsupported dtype {t.dtype}")
+
+
+def mega_gat_workspace_bytes(layout: Layout, part: int, heads: int, head_dim: int, dtype: int):
+    f, b = _c.c_size_t(), _c.c_size_t()
+    _check(lib().mega_gat_workspace_bytes(layout.handle, part, heads, head_dim, dtype, _c.byref(f), _c.byref(b)))
+    return f.value, b.value
+
+
+def mega_project_fwd(x, w, attn_l, attn_r, heads, head_dim, feat, ctx, ctx_n, ctx_row0=0, in_dim=None, stream=None):
+    dt = _dtype_code(x)
+    _check(lib().mega_project_fwd(_ptr(x), x.stride(0), x.shape[0], in_dim or w.shape[0], _ptr(w), heads, head_dim,
+                                  _ptr(attn_l), _ptr(attn_r), dt, _ptr(feat), feat.stride(0), _ptr(ctx), ctx_n,
+                                  ctx_row0, _stream(stream)))
+
+
+def mega_gat_fwd(layout: Layout, part, feat, attn_l, attn_r, heads, head_dim, out, ctx, ws,
+                 negative_slope=SLOPE, flags=0, stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_gat_fwd(layout.handle, part, _ptr(feat), feat.stride(0), _ptr(attn_l), _ptr(attn_r), heads,
+                              head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0), _ptr(ctx), _ptr(ws),
+                              ws.numel() * ws.element_size(), _stream(stream)))
+
+
+def mega_gat_bwd(layout: Layout, part, feat, attn_l, attn_r, heads, head_dim, out, grad_out, ctx, grad_feat,
+                 grad_attn_l, grad_attn_r, ws, grad_feat_lp=None, negative_slope=SLOPE, flags=0, stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_gat_bwd(layout.handle, part, _ptr(feat), feat.stride(0), _ptr(attn_l), _ptr(attn_r), heads,
+                              head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0), _ptr(grad_out),
+                              grad_out.stride(0), _ptr(ctx), _ptr(grad_feat), grad_feat.stride(0),
+                              _ptr(grad_feat_lp), grad_feat_lp.stride(0) if grad_feat_lp is not None else 0,
+                              _ptr(grad_attn_l), _ptr(grad_attn_r), _ptr(ws), ws.numel() * ws.element_size(),
+                              _stream(stream)))
+
+
+def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_dim=None, stream=None):
+    dt = _dtype_code(x)
+    _check(lib().mega_project_bwd(_ptr(x), x.stride(0), x.shape[0], in_dim or w.shape[0], _ptr(w), heads, head_dim,
+                                  dt, _ptr(grad_feat), grad_feat.stride(0), _ptr(grad_x),
+                                  grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _stream(stream)))

@@ -1,0 +1,132 @@
+"""Shared driver for the GPU parity tests: run the product (libmega.so via the
+binding) and the oracle on the same seeded inputs, in old node ids."""
+from __future__ import annotations
+
+import numpy as np
+import torch
+
+import synth
+from paper_conf_icdcs_dengr24_b200 import mega as M
+from paper_conf_icdcs_dengr24_b200.layer import GATLayer
+
+DT = {"fp32": torch.float32, "bf16": torch.bfloat16}
+
+
+def inputs(seed, n, H, F, bf16):
+    rng = np.random.default_rng(seed)
+    Wh = rng.standard_normal((n, H, F)).astype(np.float32)
+    a_l = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
+    a_r = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
+    g = rng.standard_normal((n, H, F)).astype(np.float32)
+    if bf16:
+        Wh, g = synth.bf16_round(Wh), synth.bf16_round(g)
+    return Wh, a_l, a_r, g
+
+
+def run_attention(layout, Wh_old, a_l, a_r, g_old, dtype, slope=M.SLOPE, parts=None, dev="cuda"):
+    """mega_gat_fwd + mega_gat_bwd on every part of `layout` (parts run one after
+    another on this GPU; partial grad_feat of the source phase is summed over
+    parts before the destination phase, as the k-GPU reduce-scatter does).
+    Returns old-order numpy arrays."""
+    n, H, F = Wh_old.shape
+    D = H * F
+    v0 = layout.view(0)
+    perm = v0["perm"].astype(np.int64)
+    k = v0["num_parts"]
+    tdt = DT[dtype]
+    feat = torch.tensor(Wh_old.reshape(n, D)[perm], dtype=torch.float32, device=dev).to(tdt).contiguous()
+    g_new = torch.tensor(g_old.reshape(n, D)[perm], dtype=torch.float32, device=dev).to(tdt).contiguous()
+    al = torch.tensor(a_l.reshape(-1), device=dev)
+    ar = torch.tensor(a_r.reshape(-1), device=dev)
+    ctx = torch.zeros(4, n, H, dtype=torch.float32, device=dev)
+    out_full = torch.empty(n, D, dtype=tdt, device=dev)
+    gfeat = torch.zeros(n, D, dtype=torch.float32, device=dev)
+    gal = torch.zeros(D, device=dev)
+    gar = torch.zeros(D, device=dev)
+    part_ids = range(k) if parts is None else parts
+    states = []
+    for p in part_ids:
+        layout.bind(p)
+        v = layout.view(p)
+        b0, b1 = v["row_begin"], v["row_end"]
+        fws, bws = M.mega_gat_workspace_bytes(layout, p, H, F, M._dtype_code(feat))
+        wsf = torch.empty(max(fws, 256), dtype=torch.uint8, device=dev)
+        wsb = torch.empty(max(bws, 256), dtype=torch.uint8, device=dev)
+        out = out_full[b0:b1]
+        M.mega_gat_fwd(layout, p, feat, al, ar, H, F, out, ctx, wsf, negative_slope=slope)
+        states.append((p, b0, b1, wsb))
+    # source phase per part -> partial grad_feat; sum over parts
+    partial = []
+    gar_sum = torch.zeros(D, device=dev)
+    for p, b0, b1, wsb in states:
+        gf = torch.zeros(n, D, dtype=torch.float32, device=dev)
+        tmp_l = torch.zeros(D, device=dev)
+        tmp_r = torch.zeros(D, device=dev)
+        flags = M.MEGA_BWD_PHASE_SRC if k > 1 else 0
+        M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gf, tmp_l, tmp_r, wsb,
+                       negative_slope=slope, flags=flags)
+        partial.append(gf)
+        gar_sum += tmp_r
+        if k == 1:
+            gal = tmp_l
+    if k == 1:
+        gfeat = partial[0]
+        gar = gar_sum
+    else:
+        gfeat = torch.stack(partial).sum(0)
+        gar = gar_sum
+        for p, b0, b1, wsb in states:
+            tmp_l = torch.zeros(D, device=dev)
+            M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gfeat, tmp_l,
+                           torch.zeros(D, device=dev), wsb, negative_slope=slope, flags=M.MEGA_BWD_PHASE_DST)
+            gal += tmp_l
+    torch.cuda.synchronize()
+    inv = np.empty(n, np.int64)
+    inv[perm] = np.arange(n)
+
+    def old(t, shape):
+        a = t.float().cpu().numpy()
+        return a[inv].reshape(shape)
+
+    return {"out": old(out_full, (n, H, F)), "lse": old(ctx[2], (n, H)), "el": old(ctx[0], (n, H)),
+            "er": old(ctx[1], (n, H)), "grad_feat": old(gfeat, (n, H, F)),
+            "grad_attn_l": gal.cpu().numpy().reshape(H, F), "grad_attn_r": gar.cpu().numpy().reshape(H, F)}
+
+
+def assert_fp32_close(got, ref, name):
+    """north_star fp32 bar: |gpu - ref| <= 1e-4 + 1e-5 |ref| elementwise."""
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    fin = np.isfinite(ref)
+    assert np.array_equal(fin, np.isfinite(got)), f"{name}: finiteness differs"
+    assert np.all(got[~fin] == ref[~fin]), f"{name}: infinities differ"
+    err = np.abs(got[fin] - ref[fin])
+    tol = 1e-4 + 1e-5 * np.abs(ref[fin])
+    bad = err > tol
+    assert not bad.any(), f"{name}: {bad.sum()} elements out of tolerance, max err {err.max():.3e}"
+
+
+def assert_bf16_close(got, ref, name):
+    """north_star bf16 bar: max|gpu - ref| <= 2e-2 max|ref| per tensor."""
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    fin = np.isfinite(ref)
+    assert np.array_equal(fin, np.isfinite(got)), f"{name}: finiteness differs"
+    scale = np.max(np.abs(ref[fin])) if fin.any() else 0.0
+    err = np.max(np.abs(got[fin] - ref[fin])) if fin.any() else 0.0
+    assert err <= 2e-2 * scale + 1e-30, f"{name}: max err {err:.3e} > 2e-2 * {scale:.3e}"
+
+
+def check(got, ref, dtype, keys=("out", "lse", "grad_feat", "grad_attn_l", "grad_attn_r")):
+    for k in keys:
+        (assert_fp32_close if dtype == "fp32" else assert_bf16_close)(got[k], ref[k], k)
+
+
+def layer(layout, x_new, w, a_l, a_r, H, F, dtype, want_grad_x=True):
+    tdt = DT[dtype]
+    dev = "cuda"
+    xt = torch.tensor(x_new, device=dev).to(tdt).contiguous()
+    wt = torch.tensor(w, device=dev).to(tdt).contiguous()
+    L = GATLayer(layout, xt, wt, torch.tensor(a_l, device=dev), torch.tensor(a_r, device=dev), H, F,
+                 want_grad_x=want_grad_x)
+    return L
