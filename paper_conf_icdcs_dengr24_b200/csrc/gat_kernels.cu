@@ -139,9 +139,10 @@ __device__ __forceinline__ bool head_lead(int gl, int v, int LPH) {
 }
 
 // Reduce per-lane [V][EPV] accumulators over all groups of the block and
-// store the block's [D] partial (fixed order -> deterministic).
+// store the block's [D] partial (fixed order -> deterministic; the cross-warp
+// sum is carried in fp64 because these are long reductions with cancellation).
 template <int G, int V, int EPV>
-__device__ void block_partial(float (&acc)[V][EPV], float *s_red, float *dst, int D) {
+__device__ void block_partial(float (&acc)[V][EPV], double *s_red, double *dst, int D) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G;
 #pragma unroll
   for (int o = G; o < 32; o <<= 1)
@@ -157,7 +158,7 @@ __device__ void block_partial(float (&acc)[V][EPV], float *s_red, float *dst, in
 #pragma unroll
         for (int k = 0; k < EPV; ++k) {
           const int col = (v * G + gl) * EPV + k;
-          s_red[col] = (ww == 0 ? 0.f : s_red[col]) + acc[v][k];
+          s_red[col] = (ww == 0 ? 0.0 : s_red[col]) + (double)acc[v][k];
         }
     }
     __syncthreads();
@@ -393,7 +394,8 @@ struct BwdArgs {
   int64_t ldgf;
   void *gfeat_lp;
   int64_t ldlp;
-  float *dz, *ws_bacc, *ws_bder, *ws_dar, *ws_dar2, *ws_dal;
+  float *dz, *ws_bacc, *ws_bder;
+  double *ws_dar, *ws_dar2, *ws_dal;
   float *gal, *gar;
   int nb_src, nb_merge, nb_dst;
 };
@@ -439,7 +441,7 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
   __shared__ int s_i[WPB][32];
-  __shared__ float s_red[1024];
+  __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H, LPH = a.F / EPV;
@@ -581,7 +583,7 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
 template <typename T, int G, int V>
 __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
-  __shared__ float s_red[1024];
+  __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const int H = a.H;
   float dar[V][EPV];
@@ -622,7 +624,7 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
 template <typename T, int G, int V>
 __global__ void __launch_bounds__(TPB) gat_bwd_dst_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
-  __shared__ float s_red[1024];
+  __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H;
@@ -675,14 +677,14 @@ __global__ void __launch_bounds__(TPB) gat_bwd_dst_kernel(const BwdArgs a) {
   block_partial<G, V, EPV>(dal, s_red, a.ws_dal + (int64_t)blockIdx.x * a.D, a.D);
 }
 
-// Second stage of the parameter-gradient reductions (fixed order).
-__global__ void param_reduce_kernel(const float *parts, int nparts, const float *parts2, int nparts2, int D,
+// Second stage of the parameter-gradient reductions (fixed order, fp64).
+__global__ void param_reduce_kernel(const double *parts, int nparts, const double *parts2, int nparts2, int D,
                                     float *out) {
   for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < D; d += gridDim.x * blockDim.x) {
-    float s = 0.f;
+    double s = 0.0;
     for (int b = 0; b < nparts; ++b) s += parts[(int64_t)b * D + d];
     for (int b = 0; b < nparts2; ++b) s += parts2[(int64_t)b * D + d];
-    out[d] = s;
+    out[d] = (float)s;
   }
 }
 
@@ -825,9 +827,9 @@ WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   w.bacc = align256(w.dz + (size_t)std::max<int64_t>(1, D.edges) * s.H * 4);
   w.bder = align256(w.bacc + slots * s.D * 4);
   w.dar = align256(w.bder + slots * s.H * 4);
-  w.dar2 = align256(w.dar + (size_t)MAX_GRID * s.D * 4);
-  w.dal = align256(w.dar2 + (size_t)MAX_GRID * s.D * 4);
-  w.total = align256(w.dal + (size_t)MAX_GRID * s.D * 4);
+  w.dar2 = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
+  w.dal = align256(w.dar2 + (size_t)MAX_GRID * s.D * 8);
+  w.total = align256(w.dal + (size_t)MAX_GRID * s.D * 8);
   return w;
 }
 DevPart host_counts(const Part &P, int64_t n) {  // sizes without binding
@@ -1022,9 +1024,9 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.dz = reinterpret_cast<float *>(wb + w.dz);
   a.ws_bacc = reinterpret_cast<float *>(wb + w.bacc);
   a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
-  a.ws_dar = reinterpret_cast<float *>(wb + w.dar);
-  a.ws_dar2 = reinterpret_cast<float *>(wb + w.dar2);
-  a.ws_dal = reinterpret_cast<float *>(wb + w.dal);
+  a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
+  a.ws_dar2 = reinterpret_cast<double *>(wb + w.dar2);
+  a.ws_dal = reinterpret_cast<double *>(wb + w.dal);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_src = a.nb_merge = a.nb_dst = 0;
   cudaStream_t st = (cudaStream_t)stream;

@@ -142,6 +142,10 @@ def test_whole_layer(cuda_device, dtype, name):
     inv = np.empty(n, np.int64)
     inv[perm] = np.arange(n)
     Wh = og.project_forward(x, w).reshape(n, H, F)
+    if dtype == "bf16":
+        # DESIGN.md R-prec: the oracle consumes the values the GPU stores — Wh is held in bf16
+        # (the rounding alone moves grad_attn_l by ~8% on these graphs)
+        Wh = synth.bf16_round(Wh.astype(np.float32)).astype(np.float64)
     f = og.gat_forward(ip, ix, Wh, inp["a_l"], inp["a_r"])
     b = og.gat_backward(ip, ix, Wh, inp["a_l"], inp["a_r"], g.reshape(n, H, F), fwd=f)
     pb = og.project_backward(x, w, b["grad_feat"].reshape(n, D))
@@ -151,13 +155,5 @@ def test_whole_layer(cuda_device, dtype, name):
     ref = {"out": f["out"].reshape(n, D), "grad_attn_l": b["grad_attn_l"].reshape(-1),
            "grad_attn_r": b["grad_attn_r"].reshape(-1), "grad_w": pb["grad_w"], "grad_x": pb["grad_x"],
            "grad_feat": b["grad_feat"].reshape(n, D)}
-    if dtype == "fp32":
-        # whole-layer fp32: GEMM reassociation over K = in_dim adds ~K*eps relative error; the
-        # north_star bar is applied to the attention part above, here we use the same form scaled by K
-        for k in ref:
-            err = np.abs(got[k] - ref[k])
-            tol = 1e-4 + 1e-5 * np.abs(ref[k]) + 1e-6 * np.sqrt(x.shape[1]) * np.max(np.abs(ref[k]))
-            assert np.all(err <= tol), (k, float(err.max()))
-    else:
-        for k in ref:
-            hz.assert_bf16_close(got[k], ref[k], k)
+    for k in ref:
+        (hz.assert_fp32_close if dtype == "fp32" else hz.assert_bf16_close)(got[k], ref[k], k)
