@@ -28,9 +28,11 @@
  *   - Features are row-major [rows][ld] with D = heads*head_dim used columns,
  *     heads concatenated (column h*head_dim + f).  attn_l/attn_r are fp32
  *     [heads*head_dim] in the same column order.
- *   - ctx is an fp32 block of four planes [4][ctx_n][heads]: el, er, lse,
- *     Dlt, indexed by GLOBAL new node id (ctx_n = num_nodes).  lse = -inf for
- *     rows with no in-edges (whose out row is 0) (R6).
+ *   - ctx is an fp32 block of five planes [MEGA_CTX_PLANES][ctx_n][heads]:
+ *     el, er, lse, Dlt, der, indexed by GLOBAL new node id (ctx_n =
+ *     num_nodes).  lse = -inf for rows with no in-edges (whose out row is 0)
+ *     (R6).  Dlt_i = g_i.out_i and der_j = sum over out-edges of
+ *     dz are backward intermediates (der is a per-part partial for k > 1).
  *   - Multi-part layouts (num_parts = k > 1, destination-partitioned across k
  *     GPUs): part p owns rows [bounds[p], bounds[p+1]).  For
  *     part p, `out`, `grad_out` are LOCAL row arrays [rows_p][ld]; `feat`,
@@ -145,13 +147,17 @@ typedef struct {
   const int32_t *bwd_splits; /* [num_bwd_splits][3] */
 } mega_layout_view;
 
+#define MEGA_CTX_PLANES 5 /* el, er, lse, Dlt, der */
+
 /* Flags */
 #define MEGA_FLAG_ELER_IN_CTX 1u /* mega_gat_fwd: el/er planes of ctx are already valid (from
                                     mega_project_fwd); otherwise they are computed from feat */
-#define MEGA_BWD_PHASE_SRC 2u    /* mega_gat_bwd: Dlt + source-major pass -> partial grad_feat for
-                                    ALL sources (k > 1: reduce over ranks before PHASE_DST), grad_attn_r */
-#define MEGA_BWD_PHASE_DST 4u    /* mega_gat_bwd: destination pass -> adds del_i a_l to this part's rows
-                                    of grad_feat, grad_attn_l.  Neither phase flag = both. */
+#define MEGA_BWD_PHASE_SRC 2u    /* mega_gat_bwd: Dlt + source-major pass -> partial grad_feat and the
+                                    der plane of ctx for ALL sources (k > 1: sum both over ranks onto
+                                    the owners' rows before PHASE_DST) */
+#define MEGA_BWD_PHASE_DST 4u    /* mega_gat_bwd: destination pass over this part's rows -> adds
+                                    del_i a_l to grad_feat, writes grad_feat_lp, grad_attn_l and
+                                    grad_attn_r (partials of this part for k > 1).  Neither flag = both. */
 
 int mega_abi_version(void);
 const char *mega_status_string(mega_status s);
@@ -192,7 +198,7 @@ mega_status mega_gat_workspace_bytes(const mega_layout *layout, int32_t part, in
  * cores (bf16 inputs, fp32 accumulation; MEGA_F32 = true fp32, no TF32),
  * then el/er of every projected row into ctx rows [ctx_row0, ctx_row0+rows).
  *   x    device [rows][ldx] dtype, w device [in_dim][heads*head_dim] dtype,
- *   feat device [rows][ldf] dtype, ctx device fp32 [4][ctx_n][heads].
+ *   feat device [rows][ldf] dtype, ctx device fp32 [MEGA_CTX_PLANES][ctx_n][heads].
  * Errors: INVALID_ARGUMENT, UNSUPPORTED, CUDA. */
 mega_status mega_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
                              int head_dim, const float *attn_l, const float *attn_r, mega_dtype dtype, void *feat,
@@ -203,8 +209,8 @@ mega_status mega_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_di
  * (PAPER.md:7, 84 — the irregular graph op the paper targets).
  *   feat  device [num_nodes][ldf] dtype (all sources, new order)
  *   out   device [rows_p][ldo] dtype  (written; 0 for rows without in-edges)
- *   ctx   device fp32 [4][num_nodes][heads]: writes lse (and el/er unless
- *         MEGA_FLAG_ELER_IN_CTX)
+ *   ctx   device fp32 [MEGA_CTX_PLANES][num_nodes][heads]: writes lse (and
+ *         el/er unless MEGA_FLAG_ELER_IN_CTX)
  *   ws    device, >= fwd_ws bytes from mega_gat_workspace_bytes.
  * Supported shapes: heads <= 8; head_dim a multiple of 8 (bf16) / 4 (fp32);
  * D/8 (bf16) or D/4 (fp32) a power of two <= 32 or a multiple of 32 up to 256;

@@ -1,7 +1,9 @@
 // C ABI: errors, options, layout lifetime, views, persistence and device binding.
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdio>
+#include <functional>
 #include <cstring>
 #include <new>
 
@@ -292,6 +294,13 @@ mega_status mega_layout_load(const char *path, mega_layout **out) {
       r.vec(P.indptr); r.vec(P.src); r.vec(P.eid); r.vec(P.cindptr); r.vec(P.cdst); r.vec(P.cpos);
       r.vec(P.csr2csc); r.vec(P.fwd_items); r.vec(P.fwd_splits); r.vec(P.bwd_items); r.vec(P.bwd_splits);
       if (!r.ok) throw 0;
+      if (P.cindptr.size() != (size_t)L->n + 1 || P.indptr.empty()) throw 0;
+      P.out_deg_desc.resize(L->n);
+      for (int64_t v = 0; v < L->n; ++v) P.out_deg_desc[v] = P.cindptr[v + 1] - P.cindptr[v];
+      std::sort(P.out_deg_desc.begin(), P.out_deg_desc.end(), std::greater<int32_t>());
+      P.in_deg_desc.resize(P.indptr.size() - 1);
+      for (size_t q = 0; q + 1 < P.indptr.size(); ++q) P.in_deg_desc[q] = P.indptr[q + 1] - P.indptr[q];
+      std::sort(P.in_deg_desc.begin(), P.in_deg_desc.end(), std::greater<int32_t>());
     }
   } catch (...) {
     fclose(f); delete L;

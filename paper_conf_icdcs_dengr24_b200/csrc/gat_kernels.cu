@@ -1,24 +1,28 @@
 // a3-a8: the GAT attention kernels for sm_100a and their C-ABI entry points.
 //
 // Memory-bound graph operators: no tensor cores here
-// (north_star).  Design (DESIGN.md "Kernels"):
-//   * a "group" of G lanes owns one work item (a destination row or a
+// (north_star).  Design (DESIGN.md §5):
+//   * a "group" of G lanes owns one work item (a destination row, or a
 //     segment of one); each lane holds V 16-byte vectors of a feature row, so
 //     one source row is fetched with G*V coalesced 128-bit loads;
 //   * scores are computed once per (edge, head): in the score phase lane l
-//     handles edge base+l for all heads, then the group's online softmax
-//     state (running max, per-lane partial sums) is updated with shuffles;
-//   * probabilities and source ids are staged in shared memory and the
-//     aggregation loop keeps U rows in flight per lane;
+//     takes edge base+l for all heads and the group updates the online
+//     softmax state with shuffles; the first U source rows of the chunk are
+//     requested before the scores are evaluated (their addresses only need
+//     the source ids), later batches follow from shared memory;
+//   * L2 residency: rows of high-degree nodes ("hot": gathered often) are
+//     loaded with an L2 evict_last policy, the rest with evict_first, so the
+//     126 MB L2 keeps the rows that the power-law degree distribution makes
+//     most reused; the threshold comes from the layout's degree histogram;
 //   * rows/sources longer than S edges were split by mega_preprocess into
-//     segments whose partial softmax states are merged deterministically
+//     segments whose partial softmax states are merged in fixed order
 //     (no atomics anywhere on the value path);
-//   * items are assigned grid-stride in path order, so concurrently running
-//     groups work on neighbouring rows of the MEGA order and share sources
-//     in L1/L2 (the locality the traversal creates).
+//   * items are taken grid-stride in path order, so co-resident groups work
+//     on neighbouring rows of the MEGA order.
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
+#include <climits>
 #include <cmath>
 #include <cstdlib>
 #include <mutex>
@@ -34,16 +38,34 @@ constexpr int MAXH = 8;
 constexpr int WPB = 8;
 constexpr int TPB = WPB * 32;
 constexpr int MAX_GRID = 4096;  // upper bound for per-block partial buffers
-constexpr int SP = MAXH + 1;    // smem row pitch (bank-conflict free)
 
 template <typename T> struct Tr;
 template <> struct Tr<float> { static constexpr int EPV = 4; };
 template <> struct Tr<__nv_bfloat16> { static constexpr int EPV = 8; };
 
+// ---------------------------------------------------------------- loads
+__device__ __forceinline__ uint64_t policy_last() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policy_first() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
 __device__ __forceinline__ uint4 ldg16(const void *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
-__device__ __forceinline__ int ld_stream(const int32_t *p) {
+__device__ __forceinline__ uint4 ldg16_pol(const void *p, uint64_t pol) {
+  uint4 r;
+  asm("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+// streamed index arrays: no L1 allocation, L2 evict_first
+__device__ __forceinline__ int ld_stream(const int32_t *p, uint64_t pol) {
   int v;
-  asm("ld.global.nc.L1::no_allocate.b32 %0, [%1];" : "=r"(v) : "l"(p));
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
   return v;
 }
 __device__ __forceinline__ void st16(void *p, uint4 v) { *reinterpret_cast<uint4 *>(p) = v; }
@@ -79,25 +101,25 @@ template <int G> __device__ __forceinline__ float gsum(float v, unsigned mask) {
   for (int o = G / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, G);
   return v;
 }
-__device__ __forceinline__ float sel(const float (&a)[MAXH], int i) {
+template <int HT> __device__ __forceinline__ float sel(const float (&a)[HT], int i) {
   float r = a[0];
 #pragma unroll
-  for (int h = 1; h < MAXH; ++h)
+  for (int h = 1; h < HT; ++h)
     if (i == h) r = a[h];
   return r;
 }
-// H consecutive fp32 values (16-byte vectors when H % 4 == 0)
-__device__ __forceinline__ void load_h(const float *p, int H, float (&v)[MAXH]) {
-  if ((H & 3) == 0) {
+// H (<= HT) consecutive fp32 values; 16-byte vectors when H % 4 == 0
+template <int HT> __device__ __forceinline__ void load_h(const float *p, int H, float (&v)[HT]) {
+  if (HT >= 4 && (H & 3) == 0) {
 #pragma unroll
-    for (int q = 0; q < MAXH / 4; ++q)
+    for (int q = 0; q < HT / 4; ++q)
       if (4 * q < H) {
         float4 t = __ldg(reinterpret_cast<const float4 *>(p) + q);
         v[4 * q] = t.x; v[4 * q + 1] = t.y; v[4 * q + 2] = t.z; v[4 * q + 3] = t.w;
       }
   } else {
 #pragma unroll
-    for (int h = 0; h < MAXH; ++h)
+    for (int h = 0; h < HT; ++h)
       if (h < H) v[h] = __ldg(p + h);
   }
 }
@@ -138,9 +160,9 @@ __device__ __forceinline__ bool head_lead(int gl, int v, int LPH) {
   return LPH <= G ? (gl % LPH) == 0 : (gl == 0 && (v % (LPH / G)) == 0);
 }
 
-// Reduce per-lane [V][EPV] accumulators over all groups of the block and
-// store the block's [D] partial (fixed order -> deterministic; the cross-warp
-// sum is carried in fp64 because these are long reductions with cancellation).
+// Reduce per-lane [V][EPV] accumulators over all groups of the block and store
+// the block's [D] partial (fixed order -> deterministic; the cross-warp sum is
+// carried in fp64 because these are long reductions with cancellation).
 template <int G, int V, int EPV>
 __device__ void block_partial(float (&acc)[V][EPV], double *s_red, double *dst, int D) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G;
@@ -164,6 +186,7 @@ __device__ void block_partial(float (&acc)[V][EPV], double *s_red, double *dst, 
     __syncthreads();
   }
   for (int d = threadIdx.x; d < D; d += TPB) dst[d] = s_red[d];
+  __syncthreads();
 }
 
 struct FwdArgs {
@@ -177,18 +200,20 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
+  int hot_deg;  // source rows with >= hot_deg gathers (out-degree in this part) are kept in L2
 };
 
 // ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
-template <typename T, int G, int V>
-__global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+template <typename T, int G, int V, int HT>
+__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_kernel(const FwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
   constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
   __shared__ float s_p[WPB][32][SP];
-  __shared__ int s_j[WPB][32];
+  __shared__ int s_j[WPB][32];  // source id, bit 31 = hot
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H;
+  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
@@ -197,10 +222,10 @@ __global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
     const int4 item = a.L.fwd_items[it];
     const int64_t grow = a.L.row_begin + item.x;
-    float elr[MAXH], mrun[MAXH], lrun[MAXH];
-    load_h(a.el + grow * H, H, elr);
+    float elr[HT], mrun[HT], lrun[HT];
+    load_h<HT>(a.el + grow * H, H, elr);
 #pragma unroll
-    for (int h = 0; h < MAXH; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
+    for (int h = 0; h < HT; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
     float acc[V][EPV];
 #pragma unroll
     for (int v = 0; v < V; ++v)
@@ -209,11 +234,25 @@ __global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + gl;
       const bool valid = e < item.z;
-      const int j = valid ? ld_stream(a.L.src + e) : 0;
-      float erj[MAXH], sc[MAXH];
-      load_h(a.er + (int64_t)j * H, H, erj);
+      const int j = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
+      const int cnt = min(G, item.z - base), rb = grp * G;
+      int hot = 0;
+      if (valid && a.hot_deg != INT_MAX) hot = (__ldg(a.L.cindptr + j + 1) - __ldg(a.L.cindptr + j)) >= a.hot_deg;
+      float erj[HT];
+      load_h<HT>(a.er + (int64_t)j * H, H, erj);
+      // first batch of source rows: addresses only need the ids
+      uint4 raw[U][V];
 #pragma unroll
-      for (int h = 0; h < MAXH; ++h) {
+      for (int u = 0; u < U; ++u)
+        if (u < cnt) {
+          const int jj = __shfl_sync(gmask, j, u, G), hh = __shfl_sync(gmask, hot, u, G);
+          const T *rp = feat + (int64_t)jj * a.ldf + gl * EPV;
+#pragma unroll
+          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, hh ? pol_hot : pol_cold);
+        }
+      float sc[HT];
+#pragma unroll
+      for (int h = 0; h < HT; ++h) {
         sc[h] = 1.f;
         if (h < H) {
           const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
@@ -225,24 +264,25 @@ __global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
           s_p[w][lane][h] = p;
         }
       }
-      s_j[w][lane] = j;
+      s_j[w][lane] = j | (hot << 31);
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float f = sel(sc, hv[v]);
+        const float f = sel<HT>(sc, hv[v]);
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
       }
       __syncwarp(gmask);
-      const int cnt = min(G, item.z - base), rb = grp * G;
       for (int k0 = 0; k0 < cnt; k0 += U) {
-        uint4 raw[U][V];
+        if (k0 > 0) {
 #pragma unroll
-        for (int u = 0; u < U; ++u)
-          if (k0 + u < cnt) {
-            const T *rp = feat + (int64_t)s_j[w][rb + k0 + u] * a.ldf + gl * EPV;
+          for (int u = 0; u < U; ++u)
+            if (k0 + u < cnt) {
+              const int jh = s_j[w][rb + k0 + u];
+              const T *rp = feat + (int64_t)(jh & 0x7fffffff) * a.ldf + gl * EPV;
 #pragma unroll
-            for (int v = 0; v < V; ++v) raw[u][v] = ldg16(rp + v * G * EPV);
-          }
+              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, jh < 0 ? pol_hot : pol_cold);
+            }
+        }
 #pragma unroll
         for (int u = 0; u < U; ++u)
           if (k0 + u < cnt) {
@@ -258,14 +298,14 @@ __global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
       }
       __syncwarp(gmask);
     }
-    float lt[MAXH];
+    float lt[HT];
 #pragma unroll
-    for (int h = 0; h < MAXH; ++h) lt[h] = h < H ? gsum<G>(lrun[h], gmask) : 0.f;
+    for (int h = 0; h < HT; ++h) lt[h] = h < H ? gsum<G>(lrun[h], gmask) : 0.f;
     if (item.w < 0) {
       T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float Lh = sel(lt, hv[v]);
+        const float Lh = sel<HT>(lt, hv[v]);
         const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
         float y[EPV];
 #pragma unroll
@@ -273,14 +313,14 @@ __global__ void __launch_bounds__(TPB) gat_fwd_kernel(const FwdArgs a) {
         st16(orow + v * G * EPV, pack(y, T()));
       }
       for (int h = gl; h < H; h += G) {
-        const float Lh = sel(lt, h);
-        a.lse[grow * H + h] = Lh > 0.f ? sel(mrun, h) + logf(Lh) : -INFINITY;
+        const float Lh = sel<HT>(lt, h);
+        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + logf(Lh) : -INFINITY;
       }
     } else {
       const int64_t slot = item.w;
       for (int h = gl; h < H; h += G) {
-        a.ws_m[slot * H + h] = sel(mrun, h);
-        a.ws_l[slot * H + h] = sel(lt, h);
+        a.ws_m[slot * H + h] = sel<HT>(mrun, h);
+        a.ws_l[slot * H + h] = sel<HT>(lt, h);
       }
       float *pr = a.ws_acc + slot * a.D + gl * EPV;
 #pragma unroll
@@ -389,15 +429,16 @@ struct BwdArgs {
   const void *gout;
   int64_t ldg;
   const float *el, *er, *lse;
-  float *dlt;
+  float *dlt, *der;
   float *gfeat;
   int64_t ldgf;
   void *gfeat_lp;
   int64_t ldlp;
   float *dz, *ws_bacc, *ws_bder;
-  double *ws_dar, *ws_dar2, *ws_dal;
+  double *ws_dal, *ws_dar;
   float *gal, *gar;
-  int nb_src, nb_merge, nb_dst;
+  int nb_dst;
+  int hot_deg;  // destination rows with >= hot_deg in-edges: their g rows are kept in L2
 };
 
 // ---- a6: Dlt_i = g_i . out_i ----
@@ -432,89 +473,102 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // ---- a7: source-major pass over the CSC ----
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
-// dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge.
-template <typename T, int G, int V>
-__global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+// dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
+// der_j into the der plane of ctx.
+template <typename T, int G, int V, int HT>
+__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
   constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
-  __shared__ float s_a[WPB][32][SP];  // alpha, sign = (z > 0)
+  __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
-  __shared__ int s_i[WPB][32];
-  __shared__ double s_red[1024];
+  __shared__ int s_i[WPB][32];        // destination row, bit 31 = hot
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H, LPH = a.F / EPV;
+  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
-  float arv[V][EPV], dar[V][EPV];
 #pragma unroll
-  for (int v = 0; v < V; ++v) {
-    const int col = (v * G + gl) * EPV;
-    hv[v] = col / a.F;
-#pragma unroll
-    for (int k = 0; k < EPV; ++k) { arv[v][k] = a.ar[col + k]; dar[v][k] = 0.f; }
-  }
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
   const T *gout = static_cast<const T *>(a.gout);
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
-    float whv[V][EPV], acc[V][EPV], derv[V];
+    uint4 whp[V];  // Wh_j, packed
+    float acc[V][EPV], derv[V];
     {
       const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        unpack(ldg16(rp + v * G * EPV), whv[v], T());
+        whp[v] = ldg16(rp + v * G * EPV);
         derv[v] = 0.f;
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
       }
     }
-    float erj[MAXH];
-    load_h(a.er + j * H, H, erj);
+    float erj[HT];
+    load_h<HT>(a.er + j * H, H, erj);
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
-      const int i = valid ? ld_stream(a.L.cdst + c) : 0;
+      const int i = valid ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+      const int cnt = min(G, item.z - base), rb = grp * G;
+      int hot = 0;
+      if (valid && a.hot_deg != INT_MAX) hot = (__ldg(a.L.indptr + i + 1) - __ldg(a.L.indptr + i)) >= a.hot_deg;
       const int64_t gi = a.L.row_begin + i;
-      float eli[MAXH], lsei[MAXH], dli[MAXH];
-      load_h(a.el + gi * H, H, eli);
-      load_h(a.lse + gi * H, H, lsei);
-      load_h(a.dlt + gi * H, H, dli);
+      float eli[HT], lsei[HT], dli[HT];
+      load_h<HT>(a.el + gi * H, H, eli);
+      load_h<HT>(a.lse + gi * H, H, lsei);
+      load_h<HT>(a.dlt + gi * H, H, dli);
+      uint4 raw[U][V];
 #pragma unroll
-      for (int h = 0; h < MAXH; ++h)
+      for (int u = 0; u < U; ++u)
+        if (u < cnt) {
+          const int ii = __shfl_sync(gmask, i, u, G), hh = __shfl_sync(gmask, hot, u, G);
+          const T *rp = gout + (int64_t)ii * a.ldg + gl * EPV;
+#pragma unroll
+          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, hh ? pol_hot : pol_cold);
+        } else {
+#pragma unroll
+          for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
+        }
+#pragma unroll
+      for (int h = 0; h < HT; ++h)
         if (h < H) {
           const float z = eli[h] + erj[h];
           const float al = valid ? expf(leaky(z, a.slope) - lsei[h]) : 0.f;
           s_a[w][lane][h] = z > 0.f ? al : -al;
           s_d[w][lane][h] = dli[h];
         }
-      s_i[w][lane] = i;
+      s_i[w][lane] = i | (hot << 31);
       __syncwarp(gmask);
-      const int cnt = min(G, item.z - base), rb = grp * G;
       for (int k0 = 0; k0 < cnt; k0 += U) {
-        uint4 raw[U][V];
+        if (k0 > 0) {
 #pragma unroll
-        for (int u = 0; u < U; ++u)
-          if (k0 + u < cnt) {
-            const T *rp = gout + (int64_t)s_i[w][rb + k0 + u] * a.ldg + gl * EPV;
+          for (int u = 0; u < U; ++u)
+            if (k0 + u < cnt) {
+              const int ih = s_i[w][rb + k0 + u];
+              const T *rp = gout + (int64_t)(ih & 0x7fffffff) * a.ldg + gl * EPV;
 #pragma unroll
-            for (int v = 0; v < V; ++v) raw[u][v] = ldg16(rp + v * G * EPV);
-          } else {
+              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, ih < 0 ? pol_hot : pol_cold);
+            } else {
 #pragma unroll
-            for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
-          }
+              for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
+            }
+        }
         float p[U][V];
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
           for (int v = 0; v < V; ++v) {
-            float x[EPV];
+            float x[EPV], y[EPV];
             unpack(raw[u][v], x, T());
+            unpack(whp[v], y, T());
             float s = 0.f;
 #pragma unroll
-            for (int k = 0; k < EPV; ++k) s = fmaf(x[k], whv[v][k], s);
+            for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
             p[u][v] = s;
           }
         head_reduce<G, U, V>(p, LPH, gmask);
@@ -539,9 +593,9 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
       __syncwarp(gmask);
       if (valid) {
         float *dzp = a.dz + (int64_t)c * H;
-        if ((H & 3) == 0) {
+        if (HT >= 4 && (H & 3) == 0) {
 #pragma unroll
-          for (int q = 0; q < MAXH / 4; ++q)
+          for (int q = 0; q < HT / 4; ++q)
             if (4 * q < H)
               reinterpret_cast<float4 *>(dzp)[q] = make_float4(s_z[w][lane][4 * q], s_z[w][lane][4 * q + 1],
                                                                s_z[w][lane][4 * q + 2], s_z[w][lane][4 * q + 3]);
@@ -555,13 +609,15 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
       float *orow = a.gfeat + j * a.ldgf + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
+        const float *arp = a.ar + (v * G + gl) * EPV;
 #pragma unroll
-        for (int k = 0; k < EPV; k += 4)
+        for (int k = 0; k < EPV; k += 4) {
+          const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           *reinterpret_cast<float4 *>(orow + v * G * EPV + k) =
-              make_float4(fmaf(derv[v], arv[v][k], acc[v][k]), fmaf(derv[v], arv[v][k + 1], acc[v][k + 1]),
-                          fmaf(derv[v], arv[v][k + 2], acc[v][k + 2]), fmaf(derv[v], arv[v][k + 3], acc[v][k + 3]));
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) dar[v][k] = fmaf(derv[v], whv[v][k], dar[v][k]);
+              make_float4(fmaf(derv[v], r4.x, acc[v][k]), fmaf(derv[v], r4.y, acc[v][k + 1]),
+                          fmaf(derv[v], r4.z, acc[v][k + 2]), fmaf(derv[v], r4.w, acc[v][k + 3]));
+        }
+        if (head_lead<G>(gl, v, LPH)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
       const int64_t slot = item.w;
@@ -576,30 +632,27 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_kernel(const BwdArgs a) {
       }
     }
   }
-  block_partial<G, V, EPV>(dar, s_red, a.ws_dar + (int64_t)blockIdx.x * a.D, a.D);
 }
 
-// Split sources: dWh_j = sum_k acc_k + (sum_k der_k) a_r; da_r += der_j Wh_j.
+// Split sources: dWh_j = sum_k acc_k + der_j a_r, der_j = sum_k der_k.
 template <typename T, int G, int V>
 __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
-  __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const int H = a.H;
-  float dar[V][EPV];
-#pragma unroll
-  for (int v = 0; v < V; ++v)
-#pragma unroll
-    for (int k = 0; k < EPV; ++k) dar[v][k] = 0.f;
-  const T *feat = static_cast<const T *>(a.feat);
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_splits; it += stride) {
     const int64_t j = a.L.bwd_splits[3 * it];
     const int s0 = a.L.bwd_splits[3 * it + 1], ns = a.L.bwd_splits[3 * it + 2];
+    for (int h = gl; h < H; h += G) {
+      float der = 0.f;
+      for (int s = 0; s < ns; ++s) der += a.ws_bder[(int64_t)(s0 + s) * H + h];
+      a.der[j * H + h] = der;
+    }
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       const int col = (v * G + gl) * EPV, h = col / a.F;
-      float der = 0.f, y[EPV], wh[EPV];
+      float der = 0.f, y[EPV];
 #pragma unroll
       for (int k = 0; k < EPV; ++k) y[k] = 0.f;
       for (int s = 0; s < ns; ++s) {
@@ -608,82 +661,84 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
 #pragma unroll
         for (int k = 0; k < EPV; ++k) y[k] += pa[k];
       }
-      unpack(ldg16(feat + j * a.ldf + col), wh, T());
       float *orow = a.gfeat + j * a.ldgf + col;
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) {
-        orow[k] = fmaf(der, a.ar[col + k], y[k]);
-        dar[v][k] = fmaf(der, wh[k], dar[v][k]);
-      }
+      for (int k = 0; k < EPV; ++k) orow[k] = fmaf(der, a.ar[col + k], y[k]);
     }
   }
-  block_partial<G, V, EPV>(dar, s_red, a.ws_dar2 + (int64_t)blockIdx.x * a.D, a.D);
 }
 
-// ---- a8: destination pass: del_i = sum_In dz; dWh_i += del_i a_l; da_l += del_i Wh_i ----
-template <typename T, int G, int V>
-__global__ void __launch_bounds__(TPB) gat_bwd_dst_kernel(const BwdArgs a) {
+// ---- a8: destination pass over this part's rows ----
+// del_i = sum_In dz; dWh_i += del_i a_l; da_l += del_i Wh_i; da_r += der_i Wh_i.
+template <typename T, int G, int V, int HT>
+__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_dst_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
   __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H;
+  const uint64_t pol_cold = policy_first();
   int hv[V];
-  float alv[V][EPV], dal[V][EPV];
+  float dal[V][EPV], dar[V][EPV];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
-    const int col = (v * G + gl) * EPV;
-    hv[v] = col / a.F;
+    hv[v] = ((v * G + gl) * EPV) / a.F;
 #pragma unroll
-    for (int k = 0; k < EPV; ++k) { alv[v][k] = a.al[col + k]; dal[v][k] = 0.f; }
+    for (int k = 0; k < EPV; ++k) { dal[v][k] = 0.f; dar[v][k] = 0.f; }
   }
   const T *feat = static_cast<const T *>(a.feat);
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
     const int e0 = a.L.indptr[r], e1 = a.L.indptr[r + 1];
-    float dp[MAXH];
+    float dp[HT];
 #pragma unroll
-    for (int h = 0; h < MAXH; ++h) dp[h] = 0.f;
+    for (int h = 0; h < HT; ++h) dp[h] = 0.f;
     for (int e = e0 + gl; e < e1; e += G) {
-      float t[MAXH];
-      load_h(a.dz + (int64_t)ld_stream(a.L.csr2csc + e) * H, H, t);
+      float t[HT];
+      load_h<HT>(a.dz + (int64_t)ld_stream(a.L.csr2csc + e, pol_cold) * H, H, t);
 #pragma unroll
-      for (int h = 0; h < MAXH; ++h)
+      for (int h = 0; h < HT; ++h)
         if (h < H) dp[h] += t[h];
     }
-    float del[MAXH];
+    float del[HT];
 #pragma unroll
-    for (int h = 0; h < MAXH; ++h) del[h] = h < H ? gsum<G>(dp[h], gmask) : 0.f;
+    for (int h = 0; h < HT; ++h) del[h] = h < H ? gsum<G>(dp[h], gmask) : 0.f;
     const int64_t grow = a.L.row_begin + r;
+    float derr[HT];
+    load_h<HT>(a.der + grow * H, H, derr);
     float *gr = a.gfeat + grow * a.ldgf + gl * EPV;
     const T *wr = feat + grow * a.ldf + gl * EPV;
 #pragma unroll
     for (int v = 0; v < V; ++v) {
-      const float d = sel(del, hv[v]);
+      const float d = sel<HT>(del, hv[v]), dr = sel<HT>(derr, hv[v]);
+      const float *alp = a.al + (v * G + gl) * EPV;
       float y[EPV], wh[EPV];
       unpack(ldg16(wr + v * G * EPV), wh, T());
 #pragma unroll
       for (int k = 0; k < EPV; k += 4) {
-        float4 t = *reinterpret_cast<const float4 *>(gr + v * G * EPV + k);
-        y[k] = fmaf(d, alv[v][k], t.x); y[k + 1] = fmaf(d, alv[v][k + 1], t.y);
-        y[k + 2] = fmaf(d, alv[v][k + 2], t.z); y[k + 3] = fmaf(d, alv[v][k + 3], t.w);
+        const float4 t = *reinterpret_cast<const float4 *>(gr + v * G * EPV + k);
+        const float4 l4 = __ldg(reinterpret_cast<const float4 *>(alp + k));
+        y[k] = fmaf(d, l4.x, t.x); y[k + 1] = fmaf(d, l4.y, t.y);
+        y[k + 2] = fmaf(d, l4.z, t.z); y[k + 3] = fmaf(d, l4.w, t.w);
         *reinterpret_cast<float4 *>(gr + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
       }
       if (a.gfeat_lp) st16(static_cast<T *>(a.gfeat_lp) + grow * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) dal[v][k] = fmaf(d, wh[k], dal[v][k]);
+      for (int k = 0; k < EPV; ++k) {
+        dal[v][k] = fmaf(d, wh[k], dal[v][k]);
+        dar[v][k] = fmaf(dr, wh[k], dar[v][k]);
+      }
     }
   }
   block_partial<G, V, EPV>(dal, s_red, a.ws_dal + (int64_t)blockIdx.x * a.D, a.D);
+  block_partial<G, V, EPV>(dar, s_red, a.ws_dar + (int64_t)blockIdx.x * a.D, a.D);
 }
 
 // Second stage of the parameter-gradient reductions (fixed order, fp64).
-__global__ void param_reduce_kernel(const double *parts, int nparts, const double *parts2, int nparts2, int D,
-                                    float *out) {
+__global__ void param_reduce_kernel(const double *parts, int nparts, int D, float *out) {
   for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < D; d += gridDim.x * blockDim.x) {
     double s = 0.0;
     for (int b = 0; b < nparts; ++b) s += parts[(int64_t)b * D + d];
-    for (int b = 0; b < nparts2; ++b) s += parts2[(int64_t)b * D + d];
     out[d] = (float)s;
   }
 }
@@ -712,6 +767,14 @@ bool dispatch_gv(int nv, Fn &&fn) {
     default: return false;
   }
 }
+// HT = heads rounded up to a power of two (<= 8)
+template <typename Fn>
+void dispatch_h(int H, Fn &&fn) {
+  if (H <= 1) fn(IC<1>());
+  else if (H <= 2) fn(IC<2>());
+  else if (H <= 4) fn(IC<4>());
+  else fn(IC<8>());
+}
 
 struct DevInfo { int sms = 0; int major = 0; };
 DevInfo dev_info(int dev) {
@@ -738,8 +801,8 @@ int grid_for(K kernel, int64_t groups, int gpw, int dev) {
     if (it == occ.end()) {
       int nb = 0;
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, kernel, TPB, 0);
-      occ[(const void *)kernel] = nb > 0 ? nb : 1;
       per_sm = nb > 0 ? nb : 1;
+      occ[(const void *)kernel] = per_sm;
     } else {
       per_sm = it->second;
     }
@@ -757,6 +820,28 @@ bool debug_sync() {
     v = (e && e[0] == '1') ? 1 : 0;
   }
   return v == 1;
+}
+
+// L2 budget (MB) for rows pinned with evict_last; 0 disables the hints.
+double l2_hot_mb() {
+  static double v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_L2_HOT_MB");
+    v = e ? std::atof(e) : 64.0;
+  }
+  return v;
+}
+
+// Degree threshold so that the rows gathered at least T times fit the L2 hot
+// budget (rows gathered once have no reuse and are never "hot").
+int hot_threshold(const std::vector<int32_t> &desc, size_t row_bytes) {
+  const double mb = l2_hot_mb();
+  if (mb <= 0 || desc.empty()) return INT_MAX;
+  const size_t budget_rows = (size_t)(mb * 1024.0 * 1024.0 / (double)row_bytes);
+  if (budget_rows == 0) return INT_MAX;
+  if (budget_rows >= desc.size()) return 2;
+  const int t = desc[budget_rows - 1] + 1;
+  return t >= 2 ? t : 2;
 }
 
 mega_status check_launch(cudaStream_t s, const char *what) {
@@ -819,17 +904,16 @@ WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   w.total = align256(w.acc + slots * s.D * 4);
   return w;
 }
-struct WsBwd { size_t dz, bacc, bder, dar, dar2, dal, total; };
+struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
 WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   WsBwd w;
   size_t slots = (size_t)std::max(1, D.n_bwd_slots);
   w.dz = 0;
   w.bacc = align256(w.dz + (size_t)std::max<int64_t>(1, D.edges) * s.H * 4);
   w.bder = align256(w.bacc + slots * s.D * 4);
-  w.dar = align256(w.bder + slots * s.H * 4);
-  w.dar2 = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
-  w.dal = align256(w.dar2 + (size_t)MAX_GRID * s.D * 8);
-  w.total = align256(w.dal + (size_t)MAX_GRID * s.D * 8);
+  w.dal = align256(w.bder + slots * s.H * 4);
+  w.dar = align256(w.dal + (size_t)MAX_GRID * s.D * 8);
+  w.total = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
   return w;
 }
 DevPart host_counts(const Part &P, int64_t n) {  // sizes without binding
@@ -878,9 +962,11 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
   dispatch_gv(s.nv, [&](auto g, auto v) {
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
     if (a.L.n_fwd_items > 0) {
-      auto k = gat_fwd_kernel<T, G, V>;
-      k<<<grid_for(k, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
-      rc = check_launch(st, "gat_fwd_kernel");
+      dispatch_h(s.H, [&](auto ht) {
+        auto k = gat_fwd_kernel<T, G, V, decltype(ht)::value>;
+        k<<<grid_for(k, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+        rc = check_launch(st, "gat_fwd_kernel");
+      });
       if (rc != MEGA_OK) return;
     }
     if (a.L.n_fwd_splits > 0) {
@@ -895,38 +981,41 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
 template <typename T>
 mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, int dev) {
   mega_status rc = MEGA_OK;
-  const bool src_phase = (flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) == 0 || (flags & MEGA_BWD_PHASE_SRC);
-  const bool dst_phase = (flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) == 0 || (flags & MEGA_BWD_PHASE_DST);
+  const uint32_t ph = flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST);
+  const bool src_phase = ph == 0 || (ph & MEGA_BWD_PHASE_SRC);
+  const bool dst_phase = ph == 0 || (ph & MEGA_BWD_PHASE_DST);
   dispatch_gv(s.nv, [&](auto g, auto v) {
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
-    if (src_phase) {
-      if (a.L.rows > 0) {
-        auto k = dlt_kernel<T, G, V>;
-        k<<<grid_for(k, a.L.rows, 32 / G, dev), TPB, 0, st>>>(a);
-        if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
+    dispatch_h(s.H, [&](auto ht) {
+      constexpr int HT = decltype(ht)::value;
+      if (src_phase) {
+        if (a.L.rows > 0) {
+          auto k = dlt_kernel<T, G, V>;
+          k<<<grid_for(k, a.L.rows, 32 / G, dev), TPB, 0, st>>>(a);
+          if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
+        }
+        if (a.L.n_bwd_items > 0) {
+          auto ks = gat_bwd_src_kernel<T, G, V, HT>;
+          ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+          if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
+        }
+        if (a.L.n_bwd_splits > 0) {
+          auto km = gat_bwd_src_merge_kernel<T, G, V>;
+          km<<<grid_for(km, a.L.n_bwd_splits, 32 / G, dev), TPB, 0, st>>>(a);
+          if ((rc = check_launch(st, "gat_bwd_src_merge_kernel")) != MEGA_OK) return;
+        }
       }
-      auto ks = gat_bwd_src_kernel<T, G, V>;
-      a.nb_src = grid_for(ks, std::max(1, a.L.n_bwd_items), 32 / G, dev);
-      ks<<<a.nb_src, TPB, 0, st>>>(a);
-      if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
-      a.nb_merge = 0;
-      if (a.L.n_bwd_splits > 0) {
-        auto km = gat_bwd_src_merge_kernel<T, G, V>;
-        a.nb_merge = grid_for(km, a.L.n_bwd_splits, 32 / G, dev);
-        km<<<a.nb_merge, TPB, 0, st>>>(a);
-        if ((rc = check_launch(st, "gat_bwd_src_merge_kernel")) != MEGA_OK) return;
+      if (dst_phase) {
+        auto kd = gat_bwd_dst_kernel<T, G, V, HT>;
+        a.nb_dst = grid_for(kd, std::max<int64_t>(1, a.L.rows), 32 / G, dev);
+        kd<<<a.nb_dst, TPB, 0, st>>>(a);
+        if ((rc = check_launch(st, "gat_bwd_dst_kernel")) != MEGA_OK) return;
+        param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dal, a.nb_dst, s.D, a.gal);
+        if ((rc = check_launch(st, "param_reduce_kernel(a_l)")) != MEGA_OK) return;
+        param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dar, a.nb_dst, s.D, a.gar);
+        rc = check_launch(st, "param_reduce_kernel(a_r)");
       }
-      param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dar, a.nb_src, a.ws_dar2, a.nb_merge, s.D, a.gar);
-      if ((rc = check_launch(st, "param_reduce_kernel(a_r)")) != MEGA_OK) return;
-    }
-    if (dst_phase) {
-      auto kd = gat_bwd_dst_kernel<T, G, V>;
-      a.nb_dst = grid_for(kd, std::max<int64_t>(1, a.L.rows), 32 / G, dev);
-      kd<<<a.nb_dst, TPB, 0, st>>>(a);
-      if ((rc = check_launch(st, "gat_bwd_dst_kernel")) != MEGA_OK) return;
-      param_reduce_kernel<<<(s.D + 255) / 256, 256, 0, st>>>(a.ws_dal, a.nb_dst, nullptr, 0, s.D, a.gal);
-      rc = check_launch(st, "param_reduce_kernel(a_l)");
-    }
+    });
   });
   return rc;
 }
@@ -985,6 +1074,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
+  a.hot_deg = hot_threshold(P.out_deg_desc, (size_t)s.D * esz);
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1007,7 +1097,8 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
     return fail(MEGA_ERR_INVALID_ARGUMENT, "leading dimensions must be >= D and multiples of 16 bytes");
   if (grad_feat_lp && (ldlp < s.D || (ldlp * esz) % 16 || !al16(grad_feat_lp)))
     return fail(MEGA_ERR_INVALID_ARGUMENT, "grad_feat_lp: bad ld or alignment");
-  if (!al16(feat) || !al16(out) || !al16(grad_out) || !al16(ctx) || !al16(grad_feat) || !al16(ws))
+  if (!al16(feat) || !al16(out) || !al16(grad_out) || !al16(ctx) || !al16(grad_feat) || !al16(ws) ||
+      !al16(attn_l) || !al16(attn_r))
     return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
   const Part &P = L->parts[part];
   const WsBwd w = ws_bwd(P.dev, s);
@@ -1018,17 +1109,17 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.feat = feat; a.ldf = ldf; a.al = attn_l; a.ar = attn_r;
   a.H = s.H; a.F = s.F; a.D = s.D; a.slope = negative_slope;
   a.out = out; a.ldo = ldo; a.gout = grad_out; a.ldg = ldg;
-  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane; a.dlt = ctx + 3 * plane;
+  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane; a.dlt = ctx + 3 * plane; a.der = ctx + 4 * plane;
   a.gfeat = grad_feat; a.ldgf = ldgf; a.gfeat_lp = grad_feat_lp; a.ldlp = ldlp;
   char *wb = static_cast<char *>(ws);
   a.dz = reinterpret_cast<float *>(wb + w.dz);
   a.ws_bacc = reinterpret_cast<float *>(wb + w.bacc);
   a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
-  a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
-  a.ws_dar2 = reinterpret_cast<double *>(wb + w.dar2);
   a.ws_dal = reinterpret_cast<double *>(wb + w.dal);
+  a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
-  a.nb_src = a.nb_merge = a.nb_dst = 0;
+  a.nb_dst = 0;
+  a.hot_deg = hot_threshold(P.in_deg_desc, (size_t)s.D * esz);
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }

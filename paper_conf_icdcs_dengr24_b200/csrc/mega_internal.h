@@ -35,6 +35,9 @@ struct Part {
   std::vector<int32_t> indptr, src, eid, cindptr, cdst, cpos, csr2csc;
   std::vector<int32_t> fwd_items, fwd_splits, bwd_items, bwd_splits;
   int32_t n_fwd_slots = 0, n_bwd_slots = 0;
+  // degrees sorted descending (host only): gather counts of source rows (out-degree in
+  // this part) and destination rows (in-degree); used to pick L2-resident "hot" rows
+  std::vector<int32_t> out_deg_desc, in_deg_desc;
   // binding
   int device = -1;
   void *dev_base = nullptr;

@@ -16,6 +16,7 @@
 // dropped at most once.
 #include <algorithm>
 #include <chrono>
+#include <functional>
 #include <cstring>
 #include <new>
 #include <thread>
@@ -310,6 +311,12 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
         P.cpos[c] = q;
         P.csr2csc[q] = c;
       }
+    P.out_deg_desc.resize(n);
+    for (int64_t v = 0; v < n; ++v) P.out_deg_desc[v] = P.cindptr[v + 1] - P.cindptr[v];
+    std::sort(P.out_deg_desc.begin(), P.out_deg_desc.end(), std::greater<int32_t>());
+    P.in_deg_desc.resize(rows);
+    for (int64_t r = 0; r < rows; ++r) P.in_deg_desc[r] = P.indptr[r + 1] - P.indptr[r];
+    std::sort(P.in_deg_desc.begin(), P.in_deg_desc.end(), std::greater<int32_t>());
     items_for(P.indptr, S, P.fwd_items, P.fwd_splits, P.n_fwd_slots);
     items_for(P.cindptr, S, P.bwd_items, P.bwd_splits, P.n_bwd_slots);
   }

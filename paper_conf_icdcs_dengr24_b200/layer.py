@@ -32,7 +32,7 @@ class GATLayer:
         dev = x.device
         D, n = self.D, self.n
         self.feat = torch.empty(n, D, dtype=self.dtype, device=dev)
-        self.ctx = torch.zeros(4, n, heads, dtype=torch.float32, device=dev)
+        self.ctx = torch.zeros(M.MEGA_CTX_PLANES, n, heads, dtype=torch.float32, device=dev)
         self.out = torch.empty(self.rows, D, dtype=self.dtype, device=dev)
         fws, bws = M.mega_gat_workspace_bytes(layout, part, heads, head_dim, M._dtype_code(x))
         self.ws_f = torch.empty(max(fws, 256), dtype=torch.uint8, device=dev)

@@ -18,6 +18,7 @@ LIB_PATH = os.path.join(_HERE, "libmega.so")
 MEGA_F32, MEGA_BF16 = 0, 1
 ORDERS = {"traversal": 0, "identity": 1, "degree": 2, "random": 3}
 MEGA_FLAG_ELER_IN_CTX = 1
+MEGA_CTX_PLANES = 5  # el, er, lse, Dlt, der
 MEGA_BWD_PHASE_SRC = 2
 MEGA_BWD_PHASE_DST = 4
 SLOPE = float(np.float32(0.2))

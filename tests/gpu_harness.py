@@ -38,9 +38,8 @@ def run_attention(layout, Wh_old, a_l, a_r, g_old, dtype, slope=M.SLOPE, parts=N
     g_new = torch.tensor(g_old.reshape(n, D)[perm], dtype=torch.float32, device=dev).to(tdt).contiguous()
     al = torch.tensor(a_l.reshape(-1), device=dev)
     ar = torch.tensor(a_r.reshape(-1), device=dev)
-    ctx = torch.zeros(4, n, H, dtype=torch.float32, device=dev)
+    ctx = torch.zeros(M.MEGA_CTX_PLANES, n, H, dtype=torch.float32, device=dev)
     out_full = torch.empty(n, D, dtype=tdt, device=dev)
-    gfeat = torch.zeros(n, D, dtype=torch.float32, device=dev)
     gal = torch.zeros(D, device=dev)
     gar = torch.zeros(D, device=dev)
     part_ids = range(k) if parts is None else parts
@@ -55,31 +54,32 @@ def run_attention(layout, Wh_old, a_l, a_r, g_old, dtype, slope=M.SLOPE, parts=N
         out = out_full[b0:b1]
         M.mega_gat_fwd(layout, p, feat, al, ar, H, F, out, ctx, wsf, negative_slope=slope)
         states.append((p, b0, b1, wsb))
-    # source phase per part -> partial grad_feat; sum over parts
-    partial = []
-    gar_sum = torch.zeros(D, device=dev)
+    # source phase per part -> partial grad_feat and der plane; sum over parts (the k-GPU
+    # reduce-scatter), then the destination phase per part on its own rows
+    partial, der_parts = [], []
     for p, b0, b1, wsb in states:
         gf = torch.zeros(n, D, dtype=torch.float32, device=dev)
+        M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gf,
+                       torch.zeros(D, device=dev), torch.zeros(D, device=dev), wsb, negative_slope=slope,
+                       flags=M.MEGA_BWD_PHASE_SRC)
+        partial.append(gf)
+        der_parts.append(ctx[4].clone())
+    gfeat = torch.stack(partial).sum(0)
+    ctx[4] = torch.stack(der_parts).sum(0)
+    for p, b0, b1, wsb in states:
         tmp_l = torch.zeros(D, device=dev)
         tmp_r = torch.zeros(D, device=dev)
-        flags = M.MEGA_BWD_PHASE_SRC if k > 1 else 0
-        M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gf, tmp_l, tmp_r, wsb,
-                       negative_slope=slope, flags=flags)
-        partial.append(gf)
-        gar_sum += tmp_r
-        if k == 1:
-            gal = tmp_l
-    if k == 1:
-        gfeat = partial[0]
-        gar = gar_sum
-    else:
-        gfeat = torch.stack(partial).sum(0)
-        gar = gar_sum
-        for p, b0, b1, wsb in states:
-            tmp_l = torch.zeros(D, device=dev)
-            M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gfeat, tmp_l,
-                           torch.zeros(D, device=dev), wsb, negative_slope=slope, flags=M.MEGA_BWD_PHASE_DST)
-            gal += tmp_l
+        M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gfeat, tmp_l, tmp_r,
+                       wsb, negative_slope=slope, flags=M.MEGA_BWD_PHASE_DST)
+        gal += tmp_l
+        gar += tmp_r
+    if k == 1:   # the single-call path (both phases) must agree with the split one
+        gf1 = torch.zeros(n, D, dtype=torch.float32, device=dev)
+        l1, r1 = torch.zeros(D, device=dev), torch.zeros(D, device=dev)
+        p, b0, b1, wsb = states[0]
+        M.mega_gat_bwd(layout, p, feat, al, ar, H, F, out_full[b0:b1], g_new[b0:b1], ctx, gf1, l1, r1, wsb,
+                       negative_slope=slope)
+        assert torch.equal(gf1, gfeat) and torch.equal(l1, gal) and torch.equal(r1, gar)
     torch.cuda.synchronize()
     inv = np.empty(n, np.int64)
     inv[perm] = np.arange(n)
