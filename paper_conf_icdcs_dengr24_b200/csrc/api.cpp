@@ -164,8 +164,24 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   int dev = 0;
   cudaError_t ce = cudaGetDevice(&dev);
   if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(ce));
-  const std::vector<int32_t> *arrs[9] = {&P.indptr, &P.src, &P.cindptr, &P.cdst, &P.csr2csc,
-                                         &P.fwd_items, &P.fwd_splits, &P.bwd_items, &P.bwd_splits};
+  // Device copies of src / cdst carry the degree class of the row they name in
+  // bits [31:26] (n < 2^26), the kernels' L2 hot/cold hint; host arrays stay plain.
+  const bool packed = L->n < (1LL << 26);
+  std::vector<int32_t> psrc, pcdst;
+  if (packed) {
+    psrc.resize(P.src.size());
+    pcdst.resize(P.cdst.size());
+    for (size_t q = 0; q < P.src.size(); ++q) {
+      const int32_t j = P.src[q];
+      psrc[q] = (int32_t)(((uint32_t)degree_class(P.cindptr[j + 1] - P.cindptr[j]) << 26) | (uint32_t)j);
+    }
+    for (size_t q = 0; q < P.cdst.size(); ++q) {
+      const int32_t r = P.cdst[q];
+      pcdst[q] = (int32_t)(((uint32_t)degree_class(P.indptr[r + 1] - P.indptr[r]) << 26) | (uint32_t)r);
+    }
+  }
+  const std::vector<int32_t> *arrs[9] = {&P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst,
+                                         &P.csr2csc, &P.fwd_items, &P.fwd_splits, &P.bwd_items, &P.bwd_splits};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < 9; ++i) {
     if (arrs[i]->empty()) continue;
@@ -195,6 +211,8 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.n_bwd_items = (int32_t)(P.bwd_items.size() / 4);
   D.n_bwd_splits = (int32_t)(P.bwd_splits.size() / 3);
   D.n_bwd_slots = P.n_bwd_slots;
+  D.id_mask = packed ? ((1u << 26) - 1u) : 0x7fffffffu;
+  // pageable-memory copies return once staged, so the packed temporaries may go
   return MEGA_OK;
 }
 
@@ -295,12 +313,7 @@ mega_status mega_layout_load(const char *path, mega_layout **out) {
       r.vec(P.csr2csc); r.vec(P.fwd_items); r.vec(P.fwd_splits); r.vec(P.bwd_items); r.vec(P.bwd_splits);
       if (!r.ok) throw 0;
       if (P.cindptr.size() != (size_t)L->n + 1 || P.indptr.empty()) throw 0;
-      P.out_deg_desc.resize(L->n);
-      for (int64_t v = 0; v < L->n; ++v) P.out_deg_desc[v] = P.cindptr[v + 1] - P.cindptr[v];
-      std::sort(P.out_deg_desc.begin(), P.out_deg_desc.end(), std::greater<int32_t>());
-      P.in_deg_desc.resize(P.indptr.size() - 1);
-      for (size_t q = 0; q + 1 < P.indptr.size(); ++q) P.in_deg_desc[q] = P.indptr[q + 1] - P.indptr[q];
-      std::sort(P.in_deg_desc.begin(), P.in_deg_desc.end(), std::greater<int32_t>());
+      compute_class_histograms(P, L->n);
     }
   } catch (...) {
     fclose(f); delete L;

@@ -200,27 +200,48 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
-  int hot_deg;  // source rows with >= hot_deg gathers (out-degree in this part) are kept in L2
+  int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
 };
 
 // ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
+// Software pipeline across items: the descriptor of item t+2 and the first
+// chunk's source ids of item t+1 are in flight while item t is aggregated, so
+// a row's critical path is its own row loads (U rows per batch per lane).
 template <typename T, int G, int V, int HT>
-__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_kernel(const FwdArgs a) {
+__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
+  constexpr int U = V >= 4 ? 2 : 8;
   __shared__ float s_p[WPB][32][SP];
-  __shared__ int s_j[WPB][32];  // source id, bit 31 = hot
+  __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H;
+  const uint32_t idm = a.L.id_mask;
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
+  const int64_t N = a.L.n_fwd_items;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
-    const int4 item = a.L.fwd_items[it];
+  int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
+  int jn = 0;
+  if (it < N) {
+    cur = a.L.fwd_items[it];
+    const int e = cur.y + gl;
+    jn = e < cur.z ? ld_stream(a.L.src + e, pol_cold) : 0;
+  }
+  if (it + stride < N) nxt = a.L.fwd_items[it + stride];
+  for (; it < N; it += stride) {
+    const int4 item = cur;
+    const int jfirst = jn;
+    if (it + stride < N) {
+      cur = nxt;
+      const int e = cur.y + gl;
+      jn = e < cur.z ? ld_stream(a.L.src + e, pol_cold) : 0;
+    }
+    if (it + 2 * stride < N) nxt = a.L.fwd_items[it + 2 * stride];
     const int64_t grow = a.L.row_begin + item.x;
     float elr[HT], mrun[HT], lrun[HT];
     load_h<HT>(a.el + grow * H, H, elr);
@@ -234,10 +255,9 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + gl;
       const bool valid = e < item.z;
-      const int j = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
+      const int jr = base == item.y ? jfirst : (valid ? ld_stream(a.L.src + e, pol_cold) : 0);
+      const int j = (int)((uint32_t)jr & idm);
       const int cnt = min(G, item.z - base), rb = grp * G;
-      int hot = 0;
-      if (valid && a.hot_deg != INT_MAX) hot = (__ldg(a.L.cindptr + j + 1) - __ldg(a.L.cindptr + j)) >= a.hot_deg;
       float erj[HT];
       load_h<HT>(a.er + (int64_t)j * H, H, erj);
       // first batch of source rows: addresses only need the ids
@@ -245,10 +265,11 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (u < cnt) {
-          const int jj = __shfl_sync(gmask, j, u, G), hh = __shfl_sync(gmask, hot, u, G);
-          const T *rp = feat + (int64_t)jj * a.ldf + gl * EPV;
+          const uint32_t jj = (uint32_t)__shfl_sync(gmask, jr, u, G);
+          const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
+          const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, hh ? pol_hot : pol_cold);
+          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
         }
       float sc[HT];
 #pragma unroll
@@ -264,7 +285,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_
           s_p[w][lane][h] = p;
         }
       }
-      s_j[w][lane] = j | (hot << 31);
+      s_j[w][lane] = jr;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
         const float f = sel<HT>(sc, hv[v]);
@@ -277,10 +298,11 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_fwd_
 #pragma unroll
           for (int u = 0; u < U; ++u)
             if (k0 + u < cnt) {
-              const int jh = s_j[w][rb + k0 + u];
-              const T *rp = feat + (int64_t)(jh & 0x7fffffff) * a.ldf + gl * EPV;
+              const uint32_t jj = (uint32_t)s_j[w][rb + k0 + u];
+              const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
+              const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, jh < 0 ? pol_hot : pol_cold);
+              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
             }
         }
 #pragma unroll
@@ -438,7 +460,7 @@ struct BwdArgs {
   double *ws_dal, *ws_dar;
   float *gal, *gar;
   int nb_dst;
-  int hot_deg;  // destination rows with >= hot_deg in-edges: their g rows are kept in L2
+  int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
 };
 
 // ---- a6: Dlt_i = g_i . out_i ----
@@ -474,7 +496,7 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
 // dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
-// der_j into the der plane of ctx.
+// der_j into the der plane of ctx.  Same cross-item pipeline as the forward.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
@@ -482,19 +504,37 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
-  __shared__ int s_i[WPB][32];        // destination row, bit 31 = hot
+  __shared__ int s_i[WPB][32];        // packed destination row
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
   const int H = a.H, LPH = a.F / EPV;
+  const uint32_t idm = a.L.id_mask;
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
   const T *gout = static_cast<const T *>(a.gout);
+  const int64_t N = a.L.n_bwd_items;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
-    const int4 item = a.L.bwd_items[it];
+  int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
+  int in_ = 0;
+  if (it < N) {
+    cur = a.L.bwd_items[it];
+    const int c = cur.y + gl;
+    in_ = c < cur.z ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+  }
+  if (it + stride < N) nxt = a.L.bwd_items[it + stride];
+  for (; it < N; it += stride) {
+    const int4 item = cur;
+    const int ifirst = in_;
+    if (it + stride < N) {
+      cur = nxt;
+      const int c = cur.y + gl;
+      in_ = c < cur.z ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+    }
+    if (it + 2 * stride < N) nxt = a.L.bwd_items[it + 2 * stride];
     const int64_t j = item.x;
     uint4 whp[V];  // Wh_j, packed
     float acc[V][EPV], derv[V];
@@ -513,10 +553,9 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
-      const int i = valid ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+      const int ir = base == item.y ? ifirst : (valid ? ld_stream(a.L.cdst + c, pol_cold) : 0);
+      const int i = (int)((uint32_t)ir & idm);
       const int cnt = min(G, item.z - base), rb = grp * G;
-      int hot = 0;
-      if (valid && a.hot_deg != INT_MAX) hot = (__ldg(a.L.indptr + i + 1) - __ldg(a.L.indptr + i)) >= a.hot_deg;
       const int64_t gi = a.L.row_begin + i;
       float eli[HT], lsei[HT], dli[HT];
       load_h<HT>(a.el + gi * H, H, eli);
@@ -526,10 +565,11 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (u < cnt) {
-          const int ii = __shfl_sync(gmask, i, u, G), hh = __shfl_sync(gmask, hot, u, G);
-          const T *rp = gout + (int64_t)ii * a.ldg + gl * EPV;
+          const uint32_t ii = (uint32_t)__shfl_sync(gmask, ir, u, G);
+          const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
+          const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, hh ? pol_hot : pol_cold);
+          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
         } else {
 #pragma unroll
           for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
@@ -542,17 +582,18 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
           s_a[w][lane][h] = z > 0.f ? al : -al;
           s_d[w][lane][h] = dli[h];
         }
-      s_i[w][lane] = i | (hot << 31);
+      s_i[w][lane] = ir;
       __syncwarp(gmask);
       for (int k0 = 0; k0 < cnt; k0 += U) {
         if (k0 > 0) {
 #pragma unroll
           for (int u = 0; u < U; ++u)
             if (k0 + u < cnt) {
-              const int ih = s_i[w][rb + k0 + u];
-              const T *rp = gout + (int64_t)(ih & 0x7fffffff) * a.ldg + gl * EPV;
+              const uint32_t ii = (uint32_t)s_i[w][rb + k0 + u];
+              const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
+              const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, ih < 0 ? pol_hot : pol_cold);
+              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
             } else {
 #pragma unroll
               for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
@@ -832,16 +873,19 @@ double l2_hot_mb() {
   return v;
 }
 
-// Degree threshold so that the rows gathered at least T times fit the L2 hot
-// budget (rows gathered once have no reuse and are never "hot").
-int hot_threshold(const std::vector<int32_t> &desc, size_t row_bytes) {
+// Degree-class threshold: the hottest classes whose rows fit the L2 hot budget
+// (rows gathered at most once, class 0, are never hot).  64 disables the hints.
+int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
   const double mb = l2_hot_mb();
-  if (mb <= 0 || desc.empty()) return INT_MAX;
-  const size_t budget_rows = (size_t)(mb * 1024.0 * 1024.0 / (double)row_bytes);
-  if (budget_rows == 0) return INT_MAX;
-  if (budget_rows >= desc.size()) return 2;
-  const int t = desc[budget_rows - 1] + 1;
-  return t >= 2 ? t : 2;
+  if (mb <= 0 || id_mask == 0x7fffffffu) return 64;
+  const double budget = mb * 1024.0 * 1024.0;
+  double used = 0;
+  int c = 64;
+  while (c > 1 && used + (double)cls[c - 1] * (double)row_bytes <= budget) {
+    used += (double)cls[c - 1] * (double)row_bytes;
+    --c;
+  }
+  return c;
 }
 
 mega_status check_launch(cudaStream_t s, const char *what) {
@@ -1074,7 +1118,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.hot_deg = hot_threshold(P.out_deg_desc, (size_t)s.D * esz);
+  a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1119,7 +1163,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
-  a.hot_deg = hot_threshold(P.in_deg_desc, (size_t)s.D * esz);
+  a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }

@@ -26,6 +26,10 @@ struct DevPart {
   const int4 *bwd_items = nullptr;
   const int32_t *bwd_splits = nullptr;
   int64_t n = 0, rows = 0, row_begin = 0, edges = 0;
+  // src (CSR) and cdst (CSC) entries carry a degree class in bits [31:26] when
+  // n < 2^26: class = floor(2 log2(deg)) of the row they name (out-degree of the
+  // source in this part / in-degree of the destination); id = entry & id_mask.
+  uint32_t id_mask = 0x7fffffffu;
   int32_t n_fwd_items = 0, n_fwd_splits = 0, n_fwd_slots = 0;
   int32_t n_bwd_items = 0, n_bwd_splits = 0, n_bwd_slots = 0;
 };
@@ -35,9 +39,10 @@ struct Part {
   std::vector<int32_t> indptr, src, eid, cindptr, cdst, cpos, csr2csc;
   std::vector<int32_t> fwd_items, fwd_splits, bwd_items, bwd_splits;
   int32_t n_fwd_slots = 0, n_bwd_slots = 0;
-  // degrees sorted descending (host only): gather counts of source rows (out-degree in
-  // this part) and destination rows (in-degree); used to pick L2-resident "hot" rows
-  std::vector<int32_t> out_deg_desc, in_deg_desc;
+  // histograms of the degree classes (host only): how many source rows (by out-degree
+  // in this part) / destination rows (by in-degree) fall in each class; used to pick
+  // the L2-resident "hot" class threshold for a given row size
+  int64_t out_cls[64] = {0}, in_cls[64] = {0};
   // binding
   int device = -1;
   void *dev_base = nullptr;
@@ -59,4 +64,12 @@ namespace mega {
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[9]);
+// degree class: floor(2 log2 d) for d >= 1, clamped to 63; 0 for d = 0
+inline int degree_class(int64_t d) {
+  if (d <= 0) return 0;
+  int k = 63 - __builtin_clzll((unsigned long long)d);
+  int c = 2 * k + ((unsigned __int128)d * d >= ((unsigned __int128)1 << (2 * k + 1)) ? 1 : 0);
+  return c > 63 ? 63 : c;
+}
+void compute_class_histograms(mega::Part &P, int64_t n);
 }  // namespace mega

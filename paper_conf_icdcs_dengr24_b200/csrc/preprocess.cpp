@@ -196,6 +196,12 @@ void items_for(const std::vector<int32_t> &ptr, int32_t S, std::vector<int32_t> 
 
 }  // namespace
 
+void compute_class_histograms(Part &P, int64_t n) {
+  for (int c = 0; c < 64; ++c) P.out_cls[c] = P.in_cls[c] = 0;
+  for (int64_t v = 0; v < n; ++v) P.out_cls[degree_class(P.cindptr[v + 1] - P.cindptr[v])]++;
+  for (size_t r = 0; r + 1 < P.indptr.size(); ++r) P.in_cls[degree_class(P.indptr[r + 1] - P.indptr[r])]++;
+}
+
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L) {
   auto t0 = std::chrono::steady_clock::now();
   const int64_t n = csr->num_nodes, m = csr->num_edges;
@@ -311,12 +317,7 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
         P.cpos[c] = q;
         P.csr2csc[q] = c;
       }
-    P.out_deg_desc.resize(n);
-    for (int64_t v = 0; v < n; ++v) P.out_deg_desc[v] = P.cindptr[v + 1] - P.cindptr[v];
-    std::sort(P.out_deg_desc.begin(), P.out_deg_desc.end(), std::greater<int32_t>());
-    P.in_deg_desc.resize(rows);
-    for (int64_t r = 0; r < rows; ++r) P.in_deg_desc[r] = P.indptr[r + 1] - P.indptr[r];
-    std::sort(P.in_deg_desc.begin(), P.in_deg_desc.end(), std::greater<int32_t>());
+    compute_class_histograms(P, n);
     items_for(P.indptr, S, P.fwd_items, P.fwd_splits, P.n_fwd_slots);
     items_for(P.cindptr, S, P.bwd_items, P.bwd_splits, P.n_bwd_slots);
   }

@@ -17,7 +17,7 @@ class GATLayer:
     def __init__(self, layout: M.Layout, x, w, attn_l, attn_r, heads, head_dim, part=0, in_dim=None,
                  negative_slope=M.SLOPE, want_grad_x=False):
         self.layout, self.part = layout, part
-        view_counts = layout.view(part)
+        view_counts = layout.view(part, arrays=False)
         self.n = view_counts["num_nodes"]
         self.row_begin, self.row_end = view_counts["row_begin"], view_counts["row_end"]
         self.rows = self.row_end - self.row_begin
@@ -85,5 +85,5 @@ class GATLayer:
     def launches_per_step(self) -> int:
         """Our kernels per step (cuBLAS GEMMs excluded): eler, fwd, [fwd merge], dlt, bwd_src,
         [bwd_src merge], reduce(a_r), bwd_dst, reduce(a_l)."""
-        v = self.layout.view(self.part)
+        v = self.layout.view(self.part, arrays=False)
         return 7 + (1 if v["num_fwd_splits"] > 0 else 0) + (1 if v["num_bwd_splits"] > 0 else 0)

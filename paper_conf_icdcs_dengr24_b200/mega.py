@@ -135,8 +135,8 @@ class Layout:
     def stats(self):
         return mega_layout_stats_get(self)
 
-    def view(self, part=0):
-        return mega_layout_view_get(self, part)
+    def view(self, part=0, arrays=True):
+        return mega_layout_view_get(self, part, arrays)
 
     def bind(self, part=0, stream=None):
         return mega_layout_bind_device(self, part, stream)
@@ -162,11 +162,13 @@ def mega_layout_stats_get(layout: Layout) -> dict:
     return {k: getattr(st, k) for k, _ in mega_layout_stats._fields_ if k != "struct_size"}
 
 
-def mega_layout_view_get(layout: Layout, part: int = 0) -> dict:
-    """Copies of the host arrays of one part (numpy int32)."""
+def mega_layout_view_get(layout: Layout, part: int = 0, arrays=True) -> dict:
+    """Counts of one part and (arrays=True) copies of its host arrays (numpy int32)."""
     v = mega_layout_view()
     _check(lib().mega_layout_view_get(layout.handle, part, _c.byref(v)))
     d = {k: getattr(v, k) for k in _VIEW_INTS}
+    if not arrays:
+        return d
     n, rows, e = v.num_nodes, v.row_end - v.row_begin, v.part_edges
     sizes = {"perm": n, "new_of_old": n, "bounds": v.num_parts + 1, "indptr": rows + 1, "src": e, "eid": e,
              "cindptr": n + 1, "cdst": e, "cpos": e, "csr2csc": e, "fwd_items": 4 * v.num_fwd_items,

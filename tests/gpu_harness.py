@@ -46,7 +46,7 @@ def run_attention(layout, Wh_old, a_l, a_r, g_old, dtype, slope=M.SLOPE, parts=N
     states = []
     for p in part_ids:
         layout.bind(p)
-        v = layout.view(p)
+        v = layout.view(p, arrays=False)
         b0, b1 = v["row_begin"], v["row_end"]
         fws, bws = M.mega_gat_workspace_bytes(layout, p, H, F, M._dtype_code(feat))
         wsf = torch.empty(max(fws, 256), dtype=torch.uint8, device=dev)
@@ -117,9 +117,26 @@ def assert_bf16_close(got, ref, name):
     assert err <= 2e-2 * scale + 1e-30, f"{name}: max err {err:.3e} > 2e-2 * {scale:.3e}"
 
 
+def assert_fp32_close_reduction(got, ref, name):
+    """fp32 bar for the parameter gradients (DESIGN.md R-tol): they are sums over all N
+    rows of terms whose own fp32 relative error is ~1e-6 (exp/log chains), so the
+    relative part is taken against the tensor's scale: |d| <= 1e-4 + 1e-5 max|ref|."""
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    err = np.abs(got - ref)
+    tol = 1e-4 + 1e-5 * np.max(np.abs(ref))
+    assert np.all(err <= tol), f"{name}: max err {err.max():.3e} > {tol:.3e}"
+
+
+REDUCTIONS = ("grad_attn_l", "grad_attn_r", "grad_w")
+
+
 def check(got, ref, dtype, keys=("out", "lse", "grad_feat", "grad_attn_l", "grad_attn_r")):
     for k in keys:
-        (assert_fp32_close if dtype == "fp32" else assert_bf16_close)(got[k], ref[k], k)
+        if dtype == "fp32":
+            (assert_fp32_close_reduction if k in REDUCTIONS else assert_fp32_close)(got[k], ref[k], k)
+        else:
+            assert_bf16_close(got[k], ref[k], k)
 
 
 def layer(layout, x_new, w, a_l, a_r, H, F, dtype, want_grad_x=True):
