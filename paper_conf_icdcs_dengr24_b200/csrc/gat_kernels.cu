@@ -123,6 +123,36 @@ template <int HT> __device__ __forceinline__ void load_h(const float *p, int H, 
       if (h < H) v[h] = __ldg(p + h);
   }
 }
+// volatile loads: issued exactly where written (software-pipelined prefetches)
+__device__ __forceinline__ int ldv_i32(const int32_t *p, uint64_t pol) {
+  int v;
+  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+  return v;
+}
+__device__ __forceinline__ int4 ldv_i4(const int4 *p) {
+  int4 r;
+  asm volatile("ld.global.nc.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ uint4 ldv16(const void *p) {
+  uint4 r;
+  asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
+  return r;
+}
+template <int HT> __device__ __forceinline__ void load_h_v(const float *p, int H, float (&v)[HT]) {
+  if (HT >= 4 && (H & 3) == 0) {
+#pragma unroll
+    for (int q = 0; q < HT / 4; ++q)
+      if (4 * q < H)
+        asm volatile("ld.global.nc.v4.f32 {%0, %1, %2, %3}, [%4];"
+                     : "=f"(v[4 * q]), "=f"(v[4 * q + 1]), "=f"(v[4 * q + 2]), "=f"(v[4 * q + 3])
+                     : "l"(p + 4 * q));
+  } else {
+#pragma unroll
+    for (int h = 0; h < HT; ++h)
+      if (h < H) asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v[h]) : "l"(p + h));
+  }
+}
 __device__ __forceinline__ float leaky(float z, float slope) { return z > 0.f ? z : slope * z; }
 
 // Sum per-vector partial dot products over the lanes (and vectors) of a head.
@@ -204,13 +234,15 @@ struct FwdArgs {
 };
 
 // ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
-// Software pipeline across items: the descriptor of item t+2 and the first
-// chunk's source ids of item t+1 are in flight while item t is aggregated, so
-// a row's critical path is its own row loads (U rows per batch per lane).
+// Software pipeline across items: while item t is aggregated, the descriptor
+// of item t+2, the first-chunk source ids of item t+1 and (once those ids
+// have landed) their er / the row's el are in flight (volatile loads so the
+// compiler cannot sink them to their use), so each row's critical path is
+// its own source-row loads, U rows per batch per lane.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = V >= 4 ? 2 : 8;
+  constexpr int U = V >= 4 ? 2 : (V == 2 ? 4 : 8);
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
@@ -227,24 +259,32 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
   int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
   int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
   int jn = 0;
+  float ern[HT], eln[HT];
+#pragma unroll
+  for (int h = 0; h < HT; ++h) { ern[h] = 0.f; eln[h] = 0.f; }
   if (it < N) {
-    cur = a.L.fwd_items[it];
+    cur = ldv_i4(a.L.fwd_items + it);
     const int e = cur.y + gl;
-    jn = e < cur.z ? ld_stream(a.L.src + e, pol_cold) : 0;
+    jn = e < cur.z ? ldv_i32(a.L.src + e, pol_cold) : 0;
+    load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
+    load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
   }
-  if (it + stride < N) nxt = a.L.fwd_items[it + stride];
+  if (it + stride < N) nxt = ldv_i4(a.L.fwd_items + it + stride);
   for (; it < N; it += stride) {
     const int4 item = cur;
     const int jfirst = jn;
-    if (it + stride < N) {
+    float erf[HT], elr[HT];
+#pragma unroll
+    for (int h = 0; h < HT; ++h) { erf[h] = ern[h]; elr[h] = eln[h]; }
+    const bool has_next = it + stride < N;
+    if (has_next) {
       cur = nxt;
       const int e = cur.y + gl;
-      jn = e < cur.z ? ld_stream(a.L.src + e, pol_cold) : 0;
+      jn = e < cur.z ? ldv_i32(a.L.src + e, pol_cold) : 0;
     }
-    if (it + 2 * stride < N) nxt = a.L.fwd_items[it + 2 * stride];
+    if (it + 2 * stride < N) nxt = ldv_i4(a.L.fwd_items + it + 2 * stride);
     const int64_t grow = a.L.row_begin + item.x;
-    float elr[HT], mrun[HT], lrun[HT];
-    load_h<HT>(a.el + grow * H, H, elr);
+    float mrun[HT], lrun[HT];
 #pragma unroll
     for (int h = 0; h < HT; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
     float acc[V][EPV];
@@ -255,11 +295,9 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + gl;
       const bool valid = e < item.z;
-      const int jr = base == item.y ? jfirst : (valid ? ld_stream(a.L.src + e, pol_cold) : 0);
-      const int j = (int)((uint32_t)jr & idm);
+      const bool first = base == item.y;
+      const int jr = first ? jfirst : (valid ? ld_stream(a.L.src + e, pol_cold) : 0);
       const int cnt = min(G, item.z - base), rb = grp * G;
-      float erj[HT];
-      load_h<HT>(a.er + (int64_t)j * H, H, erj);
       // first batch of source rows: addresses only need the ids
       uint4 raw[U][V];
 #pragma unroll
@@ -271,6 +309,13 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
 #pragma unroll
           for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
         }
+      float erj[HT];
+      if (first) {
+#pragma unroll
+        for (int h = 0; h < HT; ++h) erj[h] = erf[h];
+      } else {
+        load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
+      }
       float sc[HT];
 #pragma unroll
       for (int h = 0; h < HT; ++h) {
@@ -293,6 +338,10 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
         for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
       }
       __syncwarp(gmask);
+      if (first && has_next) {  // next item's ids have landed by now: fetch its er / el
+        load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
+        load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
+      }
       for (int k0 = 0; k0 < cnt; k0 += U) {
         if (k0 > 0) {
 #pragma unroll
@@ -319,6 +368,10 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
           }
       }
       __syncwarp(gmask);
+    }
+    if (item.z == item.y && has_next) {  // empty row: still prefetch the next item's scores
+      load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
+      load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
     }
     float lt[HT];
 #pragma unroll
@@ -496,11 +549,13 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
 // dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
-// der_j into the der plane of ctx.  Same cross-item pipeline as the forward.
+// der_j into the der plane of ctx.  Same cross-item pipeline as the forward:
+// the next item's destination ids, their (el, lse, Dlt) and er_j are in
+// flight while the current item is processed.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = (8 / V) > 1 ? (8 / V) : 1;
+  constexpr int U = V >= 4 ? 1 : (V == 2 ? 2 : 4);
   __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
@@ -520,47 +575,56 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
   int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
   int in_ = 0;
+  float eln[HT], lsen[HT], dln[HT], ern[HT];
+#pragma unroll
+  for (int h = 0; h < HT; ++h) { eln[h] = lsen[h] = dln[h] = ern[h] = 0.f; }
+  auto fetch_next = [&](const int4 &nit, int nir) {
+    const int64_t gi = a.L.row_begin + (int)((uint32_t)nir & idm);
+    load_h_v<HT>(a.el + gi * H, H, eln);
+    load_h_v<HT>(a.lse + gi * H, H, lsen);
+    load_h_v<HT>(a.dlt + gi * H, H, dln);
+    load_h_v<HT>(a.er + (int64_t)nit.x * H, H, ern);
+  };
   if (it < N) {
-    cur = a.L.bwd_items[it];
+    cur = ldv_i4(a.L.bwd_items + it);
     const int c = cur.y + gl;
-    in_ = c < cur.z ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+    in_ = c < cur.z ? ldv_i32(a.L.cdst + c, pol_cold) : 0;
+    fetch_next(cur, in_);
   }
-  if (it + stride < N) nxt = a.L.bwd_items[it + stride];
+  if (it + stride < N) nxt = ldv_i4(a.L.bwd_items + it + stride);
   for (; it < N; it += stride) {
     const int4 item = cur;
     const int ifirst = in_;
-    if (it + stride < N) {
+    float elf[HT], lsef[HT], dlf[HT], erj[HT];
+#pragma unroll
+    for (int h = 0; h < HT; ++h) { elf[h] = eln[h]; lsef[h] = lsen[h]; dlf[h] = dln[h]; erj[h] = ern[h]; }
+    uint4 whp[V];  // Wh_j: needed only once the g rows arrive, so loaded here
+    {
+      const T *rp = feat + (int64_t)item.x * a.ldf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) whp[v] = ldg16(rp + v * G * EPV);
+    }
+    const bool has_next = it + stride < N;
+    if (has_next) {
       cur = nxt;
       const int c = cur.y + gl;
-      in_ = c < cur.z ? ld_stream(a.L.cdst + c, pol_cold) : 0;
+      in_ = c < cur.z ? ldv_i32(a.L.cdst + c, pol_cold) : 0;
     }
-    if (it + 2 * stride < N) nxt = a.L.bwd_items[it + 2 * stride];
+    if (it + 2 * stride < N) nxt = ldv_i4(a.L.bwd_items + it + 2 * stride);
     const int64_t j = item.x;
-    uint4 whp[V];  // Wh_j, packed
     float acc[V][EPV], derv[V];
-    {
-      const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
-      for (int v = 0; v < V; ++v) {
-        whp[v] = ldg16(rp + v * G * EPV);
-        derv[v] = 0.f;
+    for (int v = 0; v < V; ++v) {
+      derv[v] = 0.f;
 #pragma unroll
-        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
-      }
+      for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
     }
-    float erj[HT];
-    load_h<HT>(a.er + j * H, H, erj);
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
-      const int ir = base == item.y ? ifirst : (valid ? ld_stream(a.L.cdst + c, pol_cold) : 0);
-      const int i = (int)((uint32_t)ir & idm);
+      const bool first = base == item.y;
+      const int ir = first ? ifirst : (valid ? ld_stream(a.L.cdst + c, pol_cold) : 0);
       const int cnt = min(G, item.z - base), rb = grp * G;
-      const int64_t gi = a.L.row_begin + i;
-      float eli[HT], lsei[HT], dli[HT];
-      load_h<HT>(a.el + gi * H, H, eli);
-      load_h<HT>(a.lse + gi * H, H, lsei);
-      load_h<HT>(a.dlt + gi * H, H, dli);
       uint4 raw[U][V];
 #pragma unroll
       for (int u = 0; u < U; ++u)
@@ -574,6 +638,16 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
 #pragma unroll
           for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
         }
+      float eli[HT], lsei[HT], dli[HT];
+      if (first) {
+#pragma unroll
+        for (int h = 0; h < HT; ++h) { eli[h] = elf[h]; lsei[h] = lsef[h]; dli[h] = dlf[h]; }
+      } else {
+        const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
+        load_h<HT>(a.el + gi * H, H, eli);
+        load_h<HT>(a.lse + gi * H, H, lsei);
+        load_h<HT>(a.dlt + gi * H, H, dli);
+      }
 #pragma unroll
       for (int h = 0; h < HT; ++h)
         if (h < H) {
@@ -584,6 +658,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
         }
       s_i[w][lane] = ir;
       __syncwarp(gmask);
+      if (first && has_next) fetch_next(cur, in_);
       for (int k0 = 0; k0 < cnt; k0 += U) {
         if (k0 > 0) {
 #pragma unroll
@@ -646,6 +721,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
       }
       __syncwarp(gmask);
     }
+    if (item.z == item.y && has_next) fetch_next(cur, in_);
     if (item.w < 0) {
       float *orow = a.gfeat + j * a.ldgf + gl * EPV;
 #pragma unroll
