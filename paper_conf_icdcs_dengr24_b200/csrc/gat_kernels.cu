@@ -234,15 +234,14 @@ struct FwdArgs {
 };
 
 // ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
-// Software pipeline across items: while item t is aggregated, the descriptor
-// of item t+2, the first-chunk source ids of item t+1 and (once those ids
-// have landed) their er / the row's el are in flight (volatile loads so the
-// compiler cannot sink them to their use), so each row's critical path is
-// its own source-row loads, U rows per batch per lane.
+// Per chunk of G edges: lane l scores edge base+l for all heads (online
+// softmax state updated with shuffles); source rows stream through two
+// register batches of U rows (batch b+1 is requested before batch b is
+// accumulated), so 2U rows per lane are in flight.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = V >= 4 ? 2 : (V == 2 ? 4 : 8);
+  constexpr int U = V >= 4 ? 1 : (V == 2 ? 4 : 8);
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
@@ -254,37 +253,23 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
-  const int64_t N = a.L.n_fwd_items;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
-  int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
-  int jn = 0;
-  float ern[HT], eln[HT];
+  auto issue = [&](uint4 (&raw)[U][V], int k0, int cnt, int rb) {
 #pragma unroll
-  for (int h = 0; h < HT; ++h) { ern[h] = 0.f; eln[h] = 0.f; }
-  if (it < N) {
-    cur = ldv_i4(a.L.fwd_items + it);
-    const int e = cur.y + gl;
-    jn = e < cur.z ? ldv_i32(a.L.src + e, pol_cold) : 0;
-    load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
-    load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
-  }
-  if (it + stride < N) nxt = ldv_i4(a.L.fwd_items + it + stride);
-  for (; it < N; it += stride) {
-    const int4 item = cur;
-    const int jfirst = jn;
-    float erf[HT], elr[HT];
+    for (int u = 0; u < U; ++u)
+      if (k0 + u < cnt) {
+        const uint32_t jj = (uint32_t)s_j[w][rb + k0 + u];
+        const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
+        const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-    for (int h = 0; h < HT; ++h) { erf[h] = ern[h]; elr[h] = eln[h]; }
-    const bool has_next = it + stride < N;
-    if (has_next) {
-      cur = nxt;
-      const int e = cur.y + gl;
-      jn = e < cur.z ? ldv_i32(a.L.src + e, pol_cold) : 0;
-    }
-    if (it + 2 * stride < N) nxt = ldv_i4(a.L.fwd_items + it + 2 * stride);
+        for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
+      }
+  };
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
+    const int4 item = a.L.fwd_items[it];
     const int64_t grow = a.L.row_begin + item.x;
-    float mrun[HT], lrun[HT];
+    float elr[HT], mrun[HT], lrun[HT];
+    load_h<HT>(a.el + grow * H, H, elr);
 #pragma unroll
     for (int h = 0; h < HT; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
     float acc[V][EPV];
@@ -292,14 +277,29 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
     for (int v = 0; v < V; ++v)
 #pragma unroll
       for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+    auto consume = [&](const uint4 (&raw)[U][V], int k0, int cnt, int rb) {
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (k0 + u < cnt) {
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float pw = s_p[w][rb + k0 + u][hv[v]];
+            float x[EPV];
+            unpack(raw[u][v], x, T());
+#pragma unroll
+            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
+          }
+        }
+    };
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + gl;
       const bool valid = e < item.z;
-      const bool first = base == item.y;
-      const int jr = first ? jfirst : (valid ? ld_stream(a.L.src + e, pol_cold) : 0);
+      const int jr = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
       const int cnt = min(G, item.z - base), rb = grp * G;
-      // first batch of source rows: addresses only need the ids
-      uint4 raw[U][V];
+      float erj[HT];
+      load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
+      // first batch: addresses only need the ids (shuffled, before the scores)
+      uint4 ra[U][V], rz[U][V];
 #pragma unroll
       for (int u = 0; u < U; ++u)
         if (u < cnt) {
@@ -307,15 +307,11 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
           const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
           const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
+          for (int v = 0; v < V; ++v) ra[u][v] = ldg16_pol(rp + v * G * EPV, pol);
         }
-      float erj[HT];
-      if (first) {
-#pragma unroll
-        for (int h = 0; h < HT; ++h) erj[h] = erf[h];
-      } else {
-        load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
-      }
+      s_j[w][lane] = jr;
+      __syncwarp(gmask);
+      if (U < cnt) issue(rz, U, cnt, rb);
       float sc[HT];
 #pragma unroll
       for (int h = 0; h < HT; ++h) {
@@ -330,7 +326,6 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
           s_p[w][lane][h] = p;
         }
       }
-      s_j[w][lane] = jr;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
         const float f = sel<HT>(sc, hv[v]);
@@ -338,40 +333,15 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
         for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
       }
       __syncwarp(gmask);
-      if (first && has_next) {  // next item's ids have landed by now: fetch its er / el
-        load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
-        load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
-      }
-      for (int k0 = 0; k0 < cnt; k0 += U) {
-        if (k0 > 0) {
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-            if (k0 + u < cnt) {
-              const uint32_t jj = (uint32_t)s_j[w][rb + k0 + u];
-              const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
-              const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-            }
+      for (int k0 = 0; k0 < cnt; k0 += 2 * U) {
+        consume(ra, k0, cnt, rb);
+        if (k0 + 2 * U < cnt) issue(ra, k0 + 2 * U, cnt, rb);
+        if (k0 + U < cnt) {
+          consume(rz, k0 + U, cnt, rb);
+          if (k0 + 3 * U < cnt) issue(rz, k0 + 3 * U, cnt, rb);
         }
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-          if (k0 + u < cnt) {
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-              const float pw = s_p[w][rb + k0 + u][hv[v]];
-              float x[EPV];
-              unpack(raw[u][v], x, T());
-#pragma unroll
-              for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
-            }
-          }
       }
       __syncwarp(gmask);
-    }
-    if (item.z == item.y && has_next) {  // empty row: still prefetch the next item's scores
-      load_h_v<HT>(a.er + (int64_t)((uint32_t)jn & idm) * H, H, ern);
-      load_h_v<HT>(a.el + (a.L.row_begin + cur.x) * H, H, eln);
     }
     float lt[HT];
 #pragma unroll
@@ -549,9 +519,7 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
 // dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
-// der_j into the der plane of ctx.  Same cross-item pipeline as the forward:
-// the next item's destination ids, their (el, lse, Dlt) and er_j are in
-// flight while the current item is processed.
+// der_j into the der plane of ctx.  g rows stream through two register batches.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
@@ -570,84 +538,86 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
   const T *gout = static_cast<const T *>(a.gout);
-  const int64_t N = a.L.n_bwd_items;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
-  int4 cur = make_int4(0, 0, 0, -1), nxt = make_int4(0, 0, 0, -1);
-  int in_ = 0;
-  float eln[HT], lsen[HT], dln[HT], ern[HT];
+  auto issue = [&](uint4 (&raw)[U][V], int k0, int cnt, int rb) {
 #pragma unroll
-  for (int h = 0; h < HT; ++h) { eln[h] = lsen[h] = dln[h] = ern[h] = 0.f; }
-  auto fetch_next = [&](const int4 &nit, int nir) {
-    const int64_t gi = a.L.row_begin + (int)((uint32_t)nir & idm);
-    load_h_v<HT>(a.el + gi * H, H, eln);
-    load_h_v<HT>(a.lse + gi * H, H, lsen);
-    load_h_v<HT>(a.dlt + gi * H, H, dln);
-    load_h_v<HT>(a.er + (int64_t)nit.x * H, H, ern);
+    for (int u = 0; u < U; ++u)
+      if (k0 + u < cnt) {
+        const uint32_t ii = (uint32_t)s_i[w][rb + k0 + u];
+        const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
+        const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
+#pragma unroll
+        for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
+      } else {
+#pragma unroll
+        for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
+      }
   };
-  if (it < N) {
-    cur = ldv_i4(a.L.bwd_items + it);
-    const int c = cur.y + gl;
-    in_ = c < cur.z ? ldv_i32(a.L.cdst + c, pol_cold) : 0;
-    fetch_next(cur, in_);
-  }
-  if (it + stride < N) nxt = ldv_i4(a.L.bwd_items + it + stride);
-  for (; it < N; it += stride) {
-    const int4 item = cur;
-    const int ifirst = in_;
-    float elf[HT], lsef[HT], dlf[HT], erj[HT];
-#pragma unroll
-    for (int h = 0; h < HT; ++h) { elf[h] = eln[h]; lsef[h] = lsen[h]; dlf[h] = dln[h]; erj[h] = ern[h]; }
-    uint4 whp[V];  // Wh_j: needed only once the g rows arrive, so loaded here
-    {
-      const T *rp = feat + (int64_t)item.x * a.ldf + gl * EPV;
-#pragma unroll
-      for (int v = 0; v < V; ++v) whp[v] = ldg16(rp + v * G * EPV);
-    }
-    const bool has_next = it + stride < N;
-    if (has_next) {
-      cur = nxt;
-      const int c = cur.y + gl;
-      in_ = c < cur.z ? ldv_i32(a.L.cdst + c, pol_cold) : 0;
-    }
-    if (it + 2 * stride < N) nxt = ldv_i4(a.L.bwd_items + it + 2 * stride);
+  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
+    const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
+    uint4 whp[V];  // Wh_j, packed
     float acc[V][EPV], derv[V];
+    {
+      const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
-    for (int v = 0; v < V; ++v) {
-      derv[v] = 0.f;
+      for (int v = 0; v < V; ++v) {
+        whp[v] = ldg16(rp + v * G * EPV);
+        derv[v] = 0.f;
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+      }
     }
+    float erj[HT];
+    load_h<HT>(a.er + j * H, H, erj);
+    auto consume = [&](const uint4 (&raw)[U][V], int k0, int cnt, int rb) {
+      float p[U][V];
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          float x[EPV], y[EPV];
+          unpack(raw[u][v], x, T());
+          unpack(whp[v], y, T());
+          float s = 0.f;
+#pragma unroll
+          for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
+          p[u][v] = s;
+        }
+      head_reduce<G, U, V>(p, LPH, gmask);
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+        if (k0 + u < cnt) {
+          const int er_ = rb + k0 + u;
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float sa = s_a[w][er_][hv[v]];
+            const float al = fabsf(sa);
+            const float dz = al * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+            derv[v] += dz;
+            float x[EPV];
+            unpack(raw[u][v], x, T());
+#pragma unroll
+            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[k], acc[v][k]);
+            if (head_lead<G>(gl, v, LPH)) s_z[w][er_][hv[v]] = dz;
+          }
+        }
+    };
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
-      const bool first = base == item.y;
-      const int ir = first ? ifirst : (valid ? ld_stream(a.L.cdst + c, pol_cold) : 0);
+      const int ir = valid ? ld_stream(a.L.cdst + c, pol_cold) : 0;
       const int cnt = min(G, item.z - base), rb = grp * G;
-      uint4 raw[U][V];
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-        if (u < cnt) {
-          const uint32_t ii = (uint32_t)__shfl_sync(gmask, ir, u, G);
-          const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
-          const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-          for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-        } else {
-#pragma unroll
-          for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
-        }
+      const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
       float eli[HT], lsei[HT], dli[HT];
-      if (first) {
-#pragma unroll
-        for (int h = 0; h < HT; ++h) { eli[h] = elf[h]; lsei[h] = lsef[h]; dli[h] = dlf[h]; }
-      } else {
-        const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
-        load_h<HT>(a.el + gi * H, H, eli);
-        load_h<HT>(a.lse + gi * H, H, lsei);
-        load_h<HT>(a.dlt + gi * H, H, dli);
-      }
+      load_h<HT>(a.el + gi * H, H, eli);
+      load_h<HT>(a.lse + gi * H, H, lsei);
+      load_h<HT>(a.dlt + gi * H, H, dli);
+      s_i[w][lane] = ir;
+      __syncwarp(gmask);
+      uint4 ra[U][V], rz[U][V];
+      issue(ra, 0, cnt, rb);
+      if (U < cnt) issue(rz, U, cnt, rb);
 #pragma unroll
       for (int h = 0; h < HT; ++h)
         if (h < H) {
@@ -656,55 +626,14 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
           s_a[w][lane][h] = z > 0.f ? al : -al;
           s_d[w][lane][h] = dli[h];
         }
-      s_i[w][lane] = ir;
       __syncwarp(gmask);
-      if (first && has_next) fetch_next(cur, in_);
-      for (int k0 = 0; k0 < cnt; k0 += U) {
-        if (k0 > 0) {
-#pragma unroll
-          for (int u = 0; u < U; ++u)
-            if (k0 + u < cnt) {
-              const uint32_t ii = (uint32_t)s_i[w][rb + k0 + u];
-              const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
-              const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-              for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-            } else {
-#pragma unroll
-              for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
-            }
+      for (int k0 = 0; k0 < cnt; k0 += 2 * U) {
+        consume(ra, k0, cnt, rb);
+        if (k0 + 2 * U < cnt) issue(ra, k0 + 2 * U, cnt, rb);
+        if (k0 + U < cnt) {
+          consume(rz, k0 + U, cnt, rb);
+          if (k0 + 3 * U < cnt) issue(rz, k0 + 3 * U, cnt, rb);
         }
-        float p[U][V];
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-#pragma unroll
-          for (int v = 0; v < V; ++v) {
-            float x[EPV], y[EPV];
-            unpack(raw[u][v], x, T());
-            unpack(whp[v], y, T());
-            float s = 0.f;
-#pragma unroll
-            for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
-            p[u][v] = s;
-          }
-        head_reduce<G, U, V>(p, LPH, gmask);
-#pragma unroll
-        for (int u = 0; u < U; ++u)
-          if (k0 + u < cnt) {
-            const int er_ = rb + k0 + u;
-#pragma unroll
-            for (int v = 0; v < V; ++v) {
-              const float sa = s_a[w][er_][hv[v]];
-              const float al = fabsf(sa);
-              const float dz = al * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
-              derv[v] += dz;
-              float x[EPV];
-              unpack(raw[u][v], x, T());
-#pragma unroll
-              for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[k], acc[v][k]);
-              if (head_lead<G>(gl, v, LPH)) s_z[w][er_][hv[v]] = dz;
-            }
-          }
       }
       __syncwarp(gmask);
       if (valid) {
@@ -721,7 +650,6 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
       }
       __syncwarp(gmask);
     }
-    if (item.z == item.y && has_next) fetch_next(cur, in_);
     if (item.w < 0) {
       float *orow = a.gfeat + j * a.ldgf + gl * EPV;
 #pragma unroll
