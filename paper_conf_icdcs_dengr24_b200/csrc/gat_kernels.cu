@@ -378,6 +378,157 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
   }
 }
 
+// ---- a3+a4+a5 for wide rows (G = 32 lanes per row): cp.async ring pipeline ----
+// Each warp streams its source rows through a private shared-memory ring of P
+// quads (4 rows each) with cp.async (LDGSTS, L2 cache-policy hints): every lane
+// copies and later reads back exactly its own 16-byte pieces, so the ring
+// needs no barriers; P quads stay in flight without holding registers.
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, uint64_t pol) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
+template <typename T, int V, int HT, int P>
+__global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, SP = HT + 1, RSLOT = 4 * P;
+  extern __shared__ uint4 ring_all[];   // [WPB][RSLOT][V][32]
+  __shared__ float s_p[WPB][32][SP];
+  __shared__ int s_j[WPB][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  uint4 *ring = ring_all + (size_t)w * RSLOT * V * 32;
+  const int H = a.H;
+  const uint32_t idm = a.L.id_mask;
+  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / a.F;
+  const T *feat = static_cast<const T *>(a.feat);
+  const int64_t stride = (int64_t)gridDim.x * WPB;
+  auto issue_quad = [&](int q, int cnt) {
+#pragma unroll
+    for (int r = 0; r < 4; ++r) {
+      const int k = 4 * q + r;
+      if (k < cnt) {
+        const uint32_t jj = (uint32_t)s_j[w][k];
+        const T *rp = feat + (int64_t)(jj & idm) * a.ldf + lane * EPV;
+        const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
+        uint4 *dst = ring + ((q % P) * 4 + r) * V * 32 + lane;
+#pragma unroll
+        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
+      }
+    }
+    cp_async_commit();
+  };
+  for (int64_t it = (int64_t)blockIdx.x * WPB + w; it < a.L.n_fwd_items; it += stride) {
+    const int4 item = a.L.fwd_items[it];
+    const int64_t grow = a.L.row_begin + item.x;
+    float elr[HT], mrun[HT], lrun[HT];
+    load_h<HT>(a.el + grow * H, H, elr);
+#pragma unroll
+    for (int h = 0; h < HT; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
+    float acc[V][EPV];
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+    for (int base = item.y; base < item.z; base += G) {
+      const int e = base + lane;
+      const bool valid = e < item.z;
+      const int jr = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
+      const int cnt = min(G, item.z - base), nq = (cnt + 3) >> 2;
+      float erj[HT];
+      load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
+      s_j[w][lane] = jr;
+      __syncwarp();
+#pragma unroll
+      for (int q = 0; q < P; ++q) {
+        if (q < nq) issue_quad(q, cnt);
+        else cp_async_commit();
+      }
+      float sc[HT];
+#pragma unroll
+      for (int h = 0; h < HT; ++h) {
+        sc[h] = 1.f;
+        if (h < H) {
+          const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
+          const float mn = fmaxf(mrun[h], gmax<G>(s, 0xffffffffu));
+          sc[h] = expf(mrun[h] - mn);
+          const float p = valid ? expf(s - mn) : 0.f;
+          lrun[h] = fmaf(lrun[h], sc[h], p);
+          mrun[h] = mn;
+          s_p[w][lane][h] = p;
+        }
+      }
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const float f = sel<HT>(sc, hv[v]);
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
+      }
+      __syncwarp();
+      for (int q = 0; q < nq; ++q) {
+        cp_async_wait<P - 1>();
+#pragma unroll
+        for (int r = 0; r < 4; ++r) {
+          const int k = 4 * q + r;
+          if (k < cnt) {
+            const uint4 *src = ring + ((q % P) * 4 + r) * V * 32 + lane;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const float pw = s_p[w][k][hv[v]];
+              float x[EPV];
+              unpack(src[v * 32], x, T());
+#pragma unroll
+              for (int kk = 0; kk < EPV; ++kk) acc[v][kk] = fmaf(pw, x[kk], acc[v][kk]);
+            }
+          }
+        }
+        if (q + P < nq) issue_quad(q + P, cnt);
+        else cp_async_commit();
+      }
+      __syncwarp();
+    }
+    float lt[HT];
+#pragma unroll
+    for (int h = 0; h < HT; ++h) lt[h] = h < H ? gsum<G>(lrun[h], 0xffffffffu) : 0.f;
+    if (item.w < 0) {
+      T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + lane * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const float Lh = sel<HT>(lt, hv[v]);
+        const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
+        float y[EPV];
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) y[k] = acc[v][k] * inv;
+        st16(orow + v * G * EPV, pack(y, T()));
+      }
+      for (int h = lane; h < H; h += G) {
+        const float Lh = sel<HT>(lt, h);
+        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + logf(Lh) : -INFINITY;
+      }
+    } else {
+      const int64_t slot = item.w;
+      for (int h = lane; h < H; h += G) {
+        a.ws_m[slot * H + h] = sel<HT>(mrun, h);
+        a.ws_l[slot * H + h] = sel<HT>(lt, h);
+      }
+      float *pr = a.ws_acc + slot * a.D + lane * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+              make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+    }
+  }
+  cp_async_wait<0>();
+}
+
 // Merge the partial softmax states of split rows: M = max m_k,
 // L = sum l_k e^{m_k - M}, out = sum acc_k e^{m_k - M} / L, lse = M + log L.
 template <typename T, int G, int V>
@@ -892,6 +1043,20 @@ int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
   return c;
 }
 
+// cp.async ring kernels for wide rows (MEGA_RING=0 selects the register-batch kernels)
+bool use_ring() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_RING");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
+int ring_blocks(size_t smem) {
+  const size_t per_sm = 227 * 1024;
+  return (int)std::max<size_t>(1, per_sm / (smem + 12 * 1024));
+}
+
 mega_status check_launch(cudaStream_t s, const char *what) {
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
@@ -1011,7 +1176,26 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
     if (a.L.n_fwd_items > 0) {
       dispatch_h(s.H, [&](auto ht) {
-        auto k = gat_fwd_kernel<T, G, V, decltype(ht)::value>;
+        constexpr int HT = decltype(ht)::value;
+        if constexpr (G == 32) {
+          if (use_ring()) {
+            constexpr int RB = 32 * V * 16;                       // bytes per row
+            constexpr int P = RB >= 4096 ? 1 : (RB >= 2048 ? 3 : (RB >= 1024 ? 6 : 8));  // <= 192 KB ring
+            auto k = gat_fwd_ring_kernel<T, V, HT, P>;
+            const size_t smem = (size_t)WPB * 4 * P * RB;
+            static bool attr = false;
+            if (!attr) {
+              cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+              attr = true;
+            }
+            const int grid = (int)std::min<int64_t>((a.L.n_fwd_items + WPB - 1) / WPB,
+                                                    (int64_t)dev_info(dev).sms * ring_blocks(smem));
+            k<<<std::max(grid, 1), TPB, smem, st>>>(a);
+            rc = check_launch(st, "gat_fwd_ring_kernel");
+            return;
+          }
+        }
+        auto k = gat_fwd_kernel<T, G, V, HT>;
         k<<<grid_for(k, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
         rc = check_launch(st, "gat_fwd_kernel");
       });
