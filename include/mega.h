@@ -246,6 +246,15 @@ mega_status mega_project_bwd(const void *x, int64_t ldx, int64_t rows, int in_di
                              int head_dim, mega_dtype dtype, const void *grad_feat, int64_t ldgf, void *grad_x,
                              int64_t ldgx, float *grad_w, mega_stream_t stream);
 
+/* Measurement helper (SURVEY §8(d)-d2 calibration; not part of the GAT path):
+ * gathers the rows idx[0..n) of a device table [rows][row_bytes] (row_bytes in
+ * {512, 1024, 2048}) on `stream`, XOR-folding them into `sink` (device fp32,
+ * >= 64 * SM-count entries) so the loads cannot be elided.  Time it with CUDA
+ * events to get the achievable row-gather bandwidth for an index pattern.
+ * Errors: INVALID_ARGUMENT, UNSUPPORTED, OUT_OF_MEMORY (sink), CUDA. */
+mega_status mega_calib_gather(const void *table, int64_t rows, int row_bytes, const int32_t *idx, int64_t n,
+                              float *sink, int64_t sink_len, mega_stream_t stream);
+
 #ifdef __cplusplus
 }
 #endif
