@@ -19,7 +19,7 @@ __global__ void __launch_bounds__(256) gather_kernel(const uint4 *table, int64_t
   uint32_t acc = 0;
   for (int64_t b = warp * 32; b < n; b += nwarps * 32) {
     const int my = b + lane < n ? __ldg(idx + b + lane) : -1;
-    const int cnt = (int)min<int64_t>(32, n - b);
+    const int cnt = (n - b) < 32 ? (int)(n - b) : 32;
     for (int k0 = 0; k0 < cnt; k0 += U) {
       uint4 r[U][V];
 #pragma unroll
