@@ -237,33 +237,31 @@ struct FwdArgs {
 // Per chunk of G edges: lane l scores edge base+l for all heads (online
 // softmax state updated with shuffles); source rows stream through two
 // register batches of U rows (batch b+1 is requested before batch b is
-// accumulated), so 2U rows per lane are in flight.
+// accumulated).  Batches are branch-free: the tail of a chunk re-reads its
+// last row (an L1 hit) with weight p = 0.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = V >= 4 ? 1 : (V == 2 ? 4 : 8);
+  constexpr int U = V >= 4 ? 1 : (V == 2 ? 4 : (G >= 16 ? 8 : 4));
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H;
-  const uint32_t idm = a.L.id_mask;
+  const int H = a.H, rb = grp * G;
+  const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
+  const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
-  int hv[V];
+  const float *sp_v[V];
 #pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
-  const T *feat = static_cast<const T *>(a.feat);
+  for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / a.F];
+  const T *featl = static_cast<const T *>(a.feat) + gl * EPV;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  auto issue = [&](uint4 (&raw)[U][V], int k0, int cnt, int rb) {
+  // element offsets fit in 32 bits (checked on the host: n * ldf < 2^32)
+  auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
+    const T *rp = featl + (jj & idm) * ldf;
+    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (k0 + u < cnt) {
-        const uint32_t jj = (uint32_t)s_j[w][rb + k0 + u];
-        const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
-        const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-        for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-      }
+    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
     const int4 item = a.L.fwd_items[it];
@@ -277,41 +275,22 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
     for (int v = 0; v < V; ++v)
 #pragma unroll
       for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
-    auto consume = [&](const uint4 (&raw)[U][V], int k0, int cnt, int rb) {
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-        if (k0 + u < cnt) {
-#pragma unroll
-          for (int v = 0; v < V; ++v) {
-            const float pw = s_p[w][rb + k0 + u][hv[v]];
-            float x[EPV];
-            unpack(raw[u][v], x, T());
-#pragma unroll
-            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
-          }
-        }
-    };
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + gl;
       const bool valid = e < item.z;
-      const int jr = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
-      const int cnt = min(G, item.z - base), rb = grp * G;
+      const int cnt = min(G, item.z - base), nb = (cnt + U - 1) / U;
+      const int jr = ld_stream(a.L.src + min(e, item.z - 1), pol_cold);
       float erj[HT];
       load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
-      // first batch: addresses only need the ids (shuffled, before the scores)
       uint4 ra[U][V], rz[U][V];
 #pragma unroll
-      for (int u = 0; u < U; ++u)
-        if (u < cnt) {
-          const uint32_t jj = (uint32_t)__shfl_sync(gmask, jr, u, G);
-          const T *rp = feat + (int64_t)(jj & idm) * a.ldf + gl * EPV;
-          const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-          for (int v = 0; v < V; ++v) ra[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-        }
+      for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)__shfl_sync(gmask, jr, min(u, cnt - 1), G));
       s_j[w][lane] = jr;
       __syncwarp(gmask);
-      if (U < cnt) issue(rz, U, cnt, rb);
+      if (nb > 1) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_j[w][rb + min(U + u, cnt - 1)]);
+      }
       float sc[HT];
 #pragma unroll
       for (int h = 0; h < HT; ++h) {
@@ -328,17 +307,35 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       }
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float f = sel<HT>(sc, hv[v]);
+        const float f = sel<HT>(sc, ((v * G + gl) * EPV) / a.F);
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
       }
       __syncwarp(gmask);
-      for (int k0 = 0; k0 < cnt; k0 += 2 * U) {
-        consume(ra, k0, cnt, rb);
-        if (k0 + 2 * U < cnt) issue(ra, k0 + 2 * U, cnt, rb);
-        if (k0 + U < cnt) {
-          consume(rz, k0 + U, cnt, rb);
-          if (k0 + 3 * U < cnt) issue(rz, k0 + 3 * U, cnt, rb);
+      auto consume = [&](const uint4 (&raw)[U][V], int k0) {
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float pw = sp_v[v][(k0 + u) * SP];
+            float x[EPV];
+            unpack(raw[u][v], x, T());
+#pragma unroll
+            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
+          }
+      };
+      for (int b = 0; b < nb; b += 2) {
+        consume(ra, b * U);
+        if (b + 2 < nb) {
+#pragma unroll
+          for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_j[w][rb + min((b + 2) * U + u, cnt - 1)]);
+        }
+        if (b + 1 < nb) {
+          consume(rz, (b + 1) * U);
+          if (b + 3 < nb) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_j[w][rb + min((b + 3) * U + u, cnt - 1)]);
+          }
         }
       }
       __syncwarp(gmask);
@@ -350,7 +347,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float Lh = sel<HT>(lt, hv[v]);
+        const float Lh = sel<HT>(lt, ((v * G + gl) * EPV) / a.F);
         const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
         float y[EPV];
 #pragma unroll
@@ -1043,12 +1040,12 @@ int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
   return c;
 }
 
-// cp.async ring kernels for wide rows (MEGA_RING=0 selects the register-batch kernels)
+// cp.async ring kernels for wide rows (opt-in with MEGA_RING=1; the register-batch kernels measure faster)
 bool use_ring() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_RING");
-    v = (e && e[0] == '0') ? 0 : 1;
+    v = (e && e[0] == '1') ? 1 : 0;
   }
   return v == 1;
 }
@@ -1286,6 +1283,8 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   const int esz = dtype == MEGA_BF16 ? 2 : 4;
   if (ldf < s.D || ldo < s.D || (ldf * esz) % 16 || (ldo * esz) % 16)
     return fail(MEGA_ERR_INVALID_ARGUMENT, "ldf/ldo must be >= D and a multiple of 16 bytes");
+  if ((uint64_t)L->n * (uint64_t)ldf >= (1ULL << 32))
+    return fail(MEGA_ERR_UNSUPPORTED, "num_nodes * ldf must be < 2^32 elements (32-bit row offsets)");
   if (!al16(feat) || !al16(out) || !al16(ctx) || !al16(ws)) return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
   const Part &P = L->parts[part];
   const WsFwd w = ws_fwd(P.dev, s);
@@ -1327,6 +1326,8 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   if (ldf < s.D || ldo < s.D || ldg < s.D || ldgf < s.D || (ldf * esz) % 16 || (ldo * esz) % 16 || (ldg * esz) % 16 ||
       (ldgf * 4) % 16)
     return fail(MEGA_ERR_INVALID_ARGUMENT, "leading dimensions must be >= D and multiples of 16 bytes");
+  if ((uint64_t)L->n * (uint64_t)std::max(ldf, ldg) >= (1ULL << 32))
+    return fail(MEGA_ERR_UNSUPPORTED, "num_nodes * ld must be < 2^32 elements (32-bit row offsets)");
   if (grad_feat_lp && (ldlp < s.D || (ldlp * esz) % 16 || !al16(grad_feat_lp)))
     return fail(MEGA_ERR_INVALID_ARGUMENT, "grad_feat_lp: bad ld or alignment");
   if (!al16(feat) || !al16(out) || !al16(grad_out) || !al16(ctx) || !al16(grad_feat) || !al16(ws) ||
