@@ -153,6 +153,18 @@ template <int HT> __device__ __forceinline__ void load_h_v(const float *p, int H
       if (h < H) asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v[h]) : "l"(p + h));
   }
 }
+// exp / log on the SFU: ex2.approx / lg2.approx (max rel. error ~2^-22; the
+// x*log2(e) rounding adds ~1e-7 |x| relative, within the fp32 parity bar)
+__device__ __forceinline__ float fexp(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x * 1.4426950408889634f));
+  return y;
+}
+__device__ __forceinline__ float flog(float x) {
+  float y;
+  asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y * 0.6931471805599453f;
+}
 __device__ __forceinline__ float leaky(float z, float slope) { return z > 0.f ? z : slope * z; }
 
 // Sum per-vector partial dot products over the lanes (and vectors) of a head.
@@ -242,7 +254,7 @@ struct FwdArgs {
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = V >= 4 ? 1 : (V == 2 ? 4 : (G >= 16 ? 8 : 4));
+  constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 4 : 8), U = U0 < G ? U0 : G;  // U divides G
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
@@ -298,8 +310,8 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
         if (h < H) {
           const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
           const float mn = fmaxf(mrun[h], gmax<G>(s, gmask));
-          sc[h] = expf(mrun[h] - mn);
-          const float p = valid ? expf(s - mn) : 0.f;
+          sc[h] = fexp(mrun[h] - mn);
+          const float p = valid ? fexp(s - mn) : 0.f;
           lrun[h] = fmaf(lrun[h], sc[h], p);
           mrun[h] = mn;
           s_p[w][lane][h] = p;
@@ -356,7 +368,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       }
       for (int h = gl; h < H; h += G) {
         const float Lh = sel<HT>(lt, h);
-        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + logf(Lh) : -INFINITY;
+        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + flog(Lh) : -INFINITY;
       }
     } else {
       const int64_t slot = item.w;
@@ -454,8 +466,8 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
         if (h < H) {
           const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
           const float mn = fmaxf(mrun[h], gmax<G>(s, 0xffffffffu));
-          sc[h] = expf(mrun[h] - mn);
-          const float p = valid ? expf(s - mn) : 0.f;
+          sc[h] = fexp(mrun[h] - mn);
+          const float p = valid ? fexp(s - mn) : 0.f;
           lrun[h] = fmaf(lrun[h], sc[h], p);
           mrun[h] = mn;
           s_p[w][lane][h] = p;
@@ -506,7 +518,7 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
       }
       for (int h = lane; h < H; h += G) {
         const float Lh = sel<HT>(lt, h);
-        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + logf(Lh) : -INFINITY;
+        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + flog(Lh) : -INFINITY;
       }
     } else {
       const int64_t slot = item.w;
@@ -541,8 +553,8 @@ __global__ void __launch_bounds__(TPB) gat_fwd_merge_kernel(const FwdArgs a) {
       float M = -INFINITY;
       for (int k = 0; k < ns; ++k) M = fmaxf(M, a.ws_m[(int64_t)(s0 + k) * H + h]);
       float Ls = 0.f;
-      for (int k = 0; k < ns; ++k) Ls += a.ws_l[(int64_t)(s0 + k) * H + h] * expf(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
-      a.lse[grow * H + h] = M + logf(Ls);
+      for (int k = 0; k < ns; ++k) Ls += a.ws_l[(int64_t)(s0 + k) * H + h] * fexp(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
+      a.lse[grow * H + h] = M + flog(Ls);
     }
     T *orow = static_cast<T *>(a.out) + (int64_t)r * a.ldo;
 #pragma unroll
@@ -554,7 +566,7 @@ __global__ void __launch_bounds__(TPB) gat_fwd_merge_kernel(const FwdArgs a) {
 #pragma unroll
       for (int q = 0; q < EPV; ++q) y[q] = 0.f;
       for (int k = 0; k < ns; ++k) {
-        const float f = expf(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
+        const float f = fexp(a.ws_m[(int64_t)(s0 + k) * H + h] - M);
         Ls += a.ws_l[(int64_t)(s0 + k) * H + h] * f;
         const float *pa = a.ws_acc + (int64_t)(s0 + k) * a.D + col;
 #pragma unroll
@@ -667,50 +679,44 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
 // dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
-// der_j into the der plane of ctx.  g rows stream through two register batches.
+// der_j into the der plane of ctx.  g rows stream through two register
+// batches; batches are branch-free (the chunk tail re-reads its last row with
+// alpha = 0).
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U = V >= 4 ? 1 : (V == 2 ? 2 : 4);
+  constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U0 < G ? U0 : G;
   __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
   __shared__ int s_i[WPB][32];        // packed destination row
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, LPH = a.F / EPV;
-  const uint32_t idm = a.L.id_mask;
+  const int H = a.H, LPH = a.F / EPV, rb = grp * G;
+  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
+  const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
   const T *feat = static_cast<const T *>(a.feat);
-  const T *gout = static_cast<const T *>(a.gout);
+  const T *goutl = static_cast<const T *>(a.gout) + gl * EPV;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  auto issue = [&](uint4 (&raw)[U][V], int k0, int cnt, int rb) {
+  auto row_load = [&](uint4 (&r)[V], uint32_t ii) {
+    const T *rp = goutl + (ii & idm) * ldg;
+    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_cold;
 #pragma unroll
-    for (int u = 0; u < U; ++u)
-      if (k0 + u < cnt) {
-        const uint32_t ii = (uint32_t)s_i[w][rb + k0 + u];
-        const T *rp = gout + (int64_t)(ii & idm) * a.ldg + gl * EPV;
-        const uint64_t pol = (int)(ii >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-#pragma unroll
-        for (int v = 0; v < V; ++v) raw[u][v] = ldg16_pol(rp + v * G * EPV, pol);
-      } else {
-#pragma unroll
-        for (int v = 0; v < V; ++v) raw[u][v] = make_uint4(0, 0, 0, 0);
-      }
+    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
-    uint4 whp[V];  // Wh_j, packed
-    float acc[V][EPV], derv[V];
+    float whf[V][EPV], acc[V][EPV], derv[V];
     {
       const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        whp[v] = ldg16(rp + v * G * EPV);
+        unpack(ldg16(rp + v * G * EPV), whf[v], T());
         derv[v] = 0.f;
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
@@ -718,24 +724,49 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
     }
     float erj[HT];
     load_h<HT>(a.er + j * H, H, erj);
-    auto consume = [&](const uint4 (&raw)[U][V], int k0, int cnt, int rb) {
-      float p[U][V];
+    for (int base = item.y; base < item.z; base += G) {
+      const int c = base + gl;
+      const bool valid = c < item.z;
+      const int cnt = min(G, item.z - base), nb = (cnt + U - 1) / U;
+      const int ir = ld_stream(a.L.cdst + min(c, item.z - 1), pol_cold);
+      const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
+      float eli[HT], lsei[HT], dli[HT];
+      load_h<HT>(a.el + gi * H, H, eli);
+      load_h<HT>(a.lse + gi * H, H, lsei);
+      load_h<HT>(a.dlt + gi * H, H, dli);
+      uint4 ra[U][V], rz[U][V];
 #pragma unroll
-      for (int u = 0; u < U; ++u)
+      for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)__shfl_sync(gmask, ir, min(u, cnt - 1), G));
+      s_i[w][lane] = ir;
+      __syncwarp(gmask);
+      if (nb > 1) {
 #pragma unroll
-        for (int v = 0; v < V; ++v) {
-          float x[EPV], y[EPV];
-          unpack(raw[u][v], x, T());
-          unpack(whp[v], y, T());
-          float s = 0.f;
+        for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_i[w][rb + min(U + u, cnt - 1)]);
+      }
 #pragma unroll
-          for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
-          p[u][v] = s;
+      for (int h = 0; h < HT; ++h)
+        if (h < H) {
+          const float z = eli[h] + erj[h];
+          const float al = valid ? fexp(leaky(z, a.slope) - lsei[h]) : 0.f;
+          s_a[w][lane][h] = z > 0.f ? al : -al;
+          s_d[w][lane][h] = dli[h];
         }
-      head_reduce<G, U, V>(p, LPH, gmask);
+      __syncwarp(gmask);
+      auto consume = [&](const uint4 (&raw)[U][V], int k0) {
+        float p[U][V], x[U][V][EPV];
 #pragma unroll
-      for (int u = 0; u < U; ++u)
-        if (k0 + u < cnt) {
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            unpack(raw[u][v], x[u][v], T());
+            float s = 0.f;
+#pragma unroll
+            for (int k = 0; k < EPV; ++k) s = fmaf(x[u][v][k], whf[v][k], s);
+            p[u][v] = s;
+          }
+        head_reduce<G, U, V>(p, LPH, gmask);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
           const int er_ = rb + k0 + u;
 #pragma unroll
           for (int v = 0; v < V; ++v) {
@@ -743,44 +774,24 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
             const float al = fabsf(sa);
             const float dz = al * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
             derv[v] += dz;
-            float x[EPV];
-            unpack(raw[u][v], x, T());
 #pragma unroll
-            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[k], acc[v][k]);
+            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[u][v][k], acc[v][k]);
             if (head_lead<G>(gl, v, LPH)) s_z[w][er_][hv[v]] = dz;
           }
         }
-    };
-    for (int base = item.y; base < item.z; base += G) {
-      const int c = base + gl;
-      const bool valid = c < item.z;
-      const int ir = valid ? ld_stream(a.L.cdst + c, pol_cold) : 0;
-      const int cnt = min(G, item.z - base), rb = grp * G;
-      const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
-      float eli[HT], lsei[HT], dli[HT];
-      load_h<HT>(a.el + gi * H, H, eli);
-      load_h<HT>(a.lse + gi * H, H, lsei);
-      load_h<HT>(a.dlt + gi * H, H, dli);
-      s_i[w][lane] = ir;
-      __syncwarp(gmask);
-      uint4 ra[U][V], rz[U][V];
-      issue(ra, 0, cnt, rb);
-      if (U < cnt) issue(rz, U, cnt, rb);
+      };
+      for (int b = 0; b < nb; b += 2) {
+        consume(ra, b * U);
+        if (b + 2 < nb) {
 #pragma unroll
-      for (int h = 0; h < HT; ++h)
-        if (h < H) {
-          const float z = eli[h] + erj[h];
-          const float al = valid ? expf(leaky(z, a.slope) - lsei[h]) : 0.f;
-          s_a[w][lane][h] = z > 0.f ? al : -al;
-          s_d[w][lane][h] = dli[h];
+          for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_i[w][rb + min((b + 2) * U + u, cnt - 1)]);
         }
-      __syncwarp(gmask);
-      for (int k0 = 0; k0 < cnt; k0 += 2 * U) {
-        consume(ra, k0, cnt, rb);
-        if (k0 + 2 * U < cnt) issue(ra, k0 + 2 * U, cnt, rb);
-        if (k0 + U < cnt) {
-          consume(rz, k0 + U, cnt, rb);
-          if (k0 + 3 * U < cnt) issue(rz, k0 + 3 * U, cnt, rb);
+        if (b + 1 < nb) {
+          consume(rz, (b + 1) * U);
+          if (b + 3 < nb) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_i[w][rb + min((b + 3) * U + u, cnt - 1)]);
+          }
         }
       }
       __syncwarp(gmask);
