@@ -168,10 +168,12 @@ __device__ __forceinline__ float flog(float x) {
 __device__ __forceinline__ float leaky(float z, float slope) { return z > 0.f ? z : slope * z; }
 
 // Sum per-vector partial dot products over the lanes (and vectors) of a head.
-// LPH = lanes per head within one vector (F / EPV).
-template <int G, int U, int V>
-__device__ __forceinline__ void head_reduce(float (&p)[U][V], int LPH, unsigned mask) {
-  if (LPH <= G) {
+// LPH = lanes per head within one vector (head_dim / EPV), a compile-time
+// power of two (heads is a power of two for every supported row width).
+template <int G, int U, int V, int LPH>
+__device__ __forceinline__ void head_reduce(float (&p)[U][V], unsigned mask) {
+  if constexpr (LPH <= G) {
+#pragma unroll
     for (int o = LPH >> 1; o > 0; o >>= 1) {
 #pragma unroll
       for (int u = 0; u < U; ++u)
@@ -179,7 +181,7 @@ __device__ __forceinline__ void head_reduce(float (&p)[U][V], int LPH, unsigned 
         for (int v = 0; v < V; ++v) p[u][v] += __shfl_xor_sync(mask, p[u][v], o, G);
     }
   } else {
-    const int VPH = LPH / G;
+    constexpr int VPH = LPH / G;
 #pragma unroll
     for (int u = 0; u < U; ++u) {
       float q[V];
@@ -197,9 +199,10 @@ __device__ __forceinline__ void head_reduce(float (&p)[U][V], int LPH, unsigned 
   }
 }
 // Does this lane write the (reduced) value of vector v's head?
-template <int G>
-__device__ __forceinline__ bool head_lead(int gl, int v, int LPH) {
-  return LPH <= G ? (gl % LPH) == 0 : (gl == 0 && (v % (LPH / G)) == 0);
+template <int G, int LPH>
+__device__ __forceinline__ bool head_lead(int gl, int v) {
+  if constexpr (LPH <= G) return (gl & (LPH - 1)) == 0;
+  else return gl == 0 && (v % (LPH / G)) == 0;
 }
 
 // Reduce per-lane [V][EPV] accumulators over all groups of the block and store
@@ -253,7 +256,7 @@ struct FwdArgs {
 // last row (an L1 hit) with weight p = 0.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
+  constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G, SP = HT + 1;
   constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 4 : 8), U = U0 < G ? U0 : G;  // U divides G
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
@@ -265,7 +268,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   const float *sp_v[V];
 #pragma unroll
-  for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / a.F];
+  for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
   const T *featl = static_cast<const T *>(a.feat) + gl * EPV;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   // element offsets fit in 32 bits (checked on the host: n * ldf < 2^32)
@@ -319,7 +322,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       }
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float f = sel<HT>(sc, ((v * G + gl) * EPV) / a.F);
+        const float f = sel<HT>(sc, ((v * G + gl) * EPV) / FF);
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
       }
@@ -359,7 +362,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        const float Lh = sel<HT>(lt, ((v * G + gl) * EPV) / a.F);
+        const float Lh = sel<HT>(lt, ((v * G + gl) * EPV) / FF);
         const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
         float y[EPV];
 #pragma unroll
@@ -404,7 +407,7 @@ template <int N> __device__ __forceinline__ void cp_async_wait() {
 
 template <typename T, int V, int HT, int P>
 __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
-  constexpr int G = 32, EPV = Tr<T>::EPV, SP = HT + 1, RSLOT = 4 * P;
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, SP = HT + 1, RSLOT = 4 * P;
   extern __shared__ uint4 ring_all[];   // [WPB][RSLOT][V][32]
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];
@@ -415,7 +418,7 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / a.F;
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / FF;
   const T *feat = static_cast<const T *>(a.feat);
   const int64_t stride = (int64_t)gridDim.x * WPB;
   auto issue_quad = [&](int q, int cnt) {
@@ -581,20 +584,19 @@ __global__ void __launch_bounds__(TPB) gat_fwd_merge_kernel(const FwdArgs a) {
 }
 
 // ---- a2 epilogue (when features did not come from mega_project_fwd): el, er ----
-template <typename T, int G, int V>
+template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB) eler_kernel(const T *feat, int64_t ldf, int64_t rows, int64_t row0,
                                                    const float *al, const float *ar, int H, int F, float *el,
                                                    float *er) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, FF = G * V * EPV / HT, LPH = FF / EPV;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int LPH = F / EPV;
   float cl[V][EPV], cr[V][EPV];
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
     const int col = (v * G + gl) * EPV;
-    hv[v] = col / F;
+    hv[v] = col / FF;
 #pragma unroll
     for (int k = 0; k < EPV; ++k) { cl[v][k] = al[col + k]; cr[v][k] = ar[col + k]; }
   }
@@ -611,11 +613,11 @@ __global__ void __launch_bounds__(TPB) eler_kernel(const T *feat, int64_t ldf, i
       for (int k = 0; k < EPV; ++k) { sl = fmaf(cl[v][k], x[k], sl); sr = fmaf(cr[v][k], x[k], sr); }
       pl[0][v] = sl; pr[0][v] = sr;
     }
-    head_reduce<G, 1, V>(pl, LPH, gmask);
-    head_reduce<G, 1, V>(pr, LPH, gmask);
+    head_reduce<G, 1, V, LPH>(pl, gmask);
+    head_reduce<G, 1, V, LPH>(pr, gmask);
 #pragma unroll
     for (int v = 0; v < V; ++v)
-      if (head_lead<G>(gl, v, LPH)) {
+      if (head_lead<G, LPH>(gl, v)) {
         el[(row0 + r) * H + hv[v]] = pl[0][v];
         er[(row0 + r) * H + hv[v]] = pr[0][v];
       }
@@ -647,12 +649,12 @@ struct BwdArgs {
 };
 
 // ---- a6: Dlt_i = g_i . out_i ----
-template <typename T, int G, int V>
+template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, FF = G * V * EPV / HT, LPH = FF / EPV;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int LPH = a.F / EPV, H = a.H;
+  const int H = a.H;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
     const T *gr = static_cast<const T *>(a.gout) + r * a.ldg + gl * EPV;
@@ -668,10 +670,10 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
       for (int k = 0; k < EPV; ++k) s = fmaf(x[k], y[k], s);
       p[0][v] = s;
     }
-    head_reduce<G, 1, V>(p, LPH, gmask);
+    head_reduce<G, 1, V, LPH>(p, gmask);
 #pragma unroll
     for (int v = 0; v < V; ++v)
-      if (head_lead<G>(gl, v, LPH)) a.dlt[(a.L.row_begin + r) * H + ((v * G + gl) * EPV) / a.F] = p[0][v];
+      if (head_lead<G, LPH>(gl, v)) a.dlt[(a.L.row_begin + r) * H + ((v * G + gl) * EPV) / FF] = p[0][v];
   }
 }
 
@@ -684,7 +686,7 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // alpha = 0).
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, SP = HT + 1;
+  constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G, SP = HT + 1;
   constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U0 < G ? U0 : G;
   __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
@@ -692,13 +694,13 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   __shared__ int s_i[WPB][32];        // packed destination row
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, LPH = a.F / EPV, rb = grp * G;
+  const int H = a.H, rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
   const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / a.F;
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
   const T *feat = static_cast<const T *>(a.feat);
   const T *goutl = static_cast<const T *>(a.gout) + gl * EPV;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
@@ -753,30 +755,33 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
         }
       __syncwarp(gmask);
       auto consume = [&](const uint4 (&raw)[U][V], int k0) {
-        float p[U][V], x[U][V][EPV];
+        float p[U][V];
 #pragma unroll
         for (int u = 0; u < U; ++u)
 #pragma unroll
           for (int v = 0; v < V; ++v) {
-            unpack(raw[u][v], x[u][v], T());
+            // alpha is known before the dot product: accumulate alpha g_i and g_i . Wh_j in one pass
+            const float al = fabsf(s_a[w][rb + k0 + u][hv[v]]);
+            float x[EPV];
+            unpack(raw[u][v], x, T());
             float s = 0.f;
 #pragma unroll
-            for (int k = 0; k < EPV; ++k) s = fmaf(x[u][v][k], whf[v][k], s);
+            for (int k = 0; k < EPV; ++k) {
+              s = fmaf(x[k], whf[v][k], s);
+              acc[v][k] = fmaf(al, x[k], acc[v][k]);
+            }
             p[u][v] = s;
           }
-        head_reduce<G, U, V>(p, LPH, gmask);
+        head_reduce<G, U, V, LPH>(p, gmask);
 #pragma unroll
         for (int u = 0; u < U; ++u) {
           const int er_ = rb + k0 + u;
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             const float sa = s_a[w][er_][hv[v]];
-            const float al = fabsf(sa);
-            const float dz = al * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+            const float dz = fabsf(sa) * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
             derv[v] += dz;
-#pragma unroll
-            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(al, x[u][v][k], acc[v][k]);
-            if (head_lead<G>(gl, v, LPH)) s_z[w][er_][hv[v]] = dz;
+            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
           }
         }
       };
@@ -821,7 +826,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
               make_float4(fmaf(derv[v], r4.x, acc[v][k]), fmaf(derv[v], r4.y, acc[v][k + 1]),
                           fmaf(derv[v], r4.z, acc[v][k + 2]), fmaf(derv[v], r4.w, acc[v][k + 3]));
         }
-        if (head_lead<G>(gl, v, LPH)) a.der[j * H + hv[v]] = derv[v];
+        if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
       const int64_t slot = item.w;
@@ -832,7 +837,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
         for (int k = 0; k < EPV; k += 4)
           *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
               make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
-        if (head_lead<G>(gl, v, LPH)) a.ws_bder[slot * H + hv[v]] = derv[v];
+        if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
       }
     }
   }
@@ -876,7 +881,7 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
 // del_i = sum_In dz; dWh_i += del_i a_l; da_l += del_i Wh_i; da_r += der_i Wh_i.
 template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_dst_kernel(const BwdArgs a) {
-  constexpr int EPV = Tr<T>::EPV, GPW = 32 / G;
+  constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G;
   __shared__ double s_red[1024];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
@@ -886,7 +891,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
   float dal[V][EPV], dar[V][EPV];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
-    hv[v] = ((v * G + gl) * EPV) / a.F;
+    hv[v] = ((v * G + gl) * EPV) / FF;
 #pragma unroll
     for (int k = 0; k < EPV; ++k) { dal[v][k] = 0.f; dar[v][k] = 0.f; }
   }
@@ -1083,7 +1088,8 @@ struct Shape {
 
 mega_status check_shape(int heads, int head_dim, mega_dtype dtype, Shape &s) {
   if (dtype != MEGA_F32 && dtype != MEGA_BF16) return fail(MEGA_ERR_INVALID_ARGUMENT, "dtype must be MEGA_F32 or MEGA_BF16");
-  if (heads < 1 || heads > MAXH) return fail(MEGA_ERR_UNSUPPORTED, "heads must be in [1, 8]");
+  if (heads < 1 || heads > MAXH || (heads & (heads - 1)))
+    return fail(MEGA_ERR_UNSUPPORTED, "heads must be 1, 2, 4 or 8");
   if (head_dim < 1) return fail(MEGA_ERR_INVALID_ARGUMENT, "head_dim must be >= 1");
   s.H = heads; s.F = head_dim; s.D = heads * head_dim;
   s.epv = dtype == MEGA_BF16 ? 8 : 4;
@@ -1153,10 +1159,12 @@ mega_status launch_eler(const void *feat, int64_t ldf, int64_t rows, int64_t row
   mega_status rc = MEGA_OK;
   dispatch_gv(s.nv, [&](auto g, auto v) {
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
-    auto k = eler_kernel<T, G, V>;
-    const int grid = grid_for(k, rows, 32 / G, dev);
-    k<<<grid, TPB, 0, st>>>(static_cast<const T *>(feat), ldf, rows, row0, al, ar, s.H, s.F, el, er);
-    rc = check_launch(st, "eler_kernel");
+    dispatch_h(s.H, [&](auto ht) {
+      auto k = eler_kernel<T, G, V, decltype(ht)::value>;
+      const int grid = grid_for(k, rows, 32 / G, dev);
+      k<<<grid, TPB, 0, st>>>(static_cast<const T *>(feat), ldf, rows, row0, al, ar, s.H, s.F, el, er);
+      rc = check_launch(st, "eler_kernel");
+    });
   });
   return rc;
 }
@@ -1230,7 +1238,7 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
       constexpr int HT = decltype(ht)::value;
       if (src_phase) {
         if (a.L.rows > 0) {
-          auto k = dlt_kernel<T, G, V>;
+          auto k = dlt_kernel<T, G, V, HT>;
           k<<<grid_for(k, a.L.rows, 32 / G, dev), TPB, 0, st>>>(a);
           if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
         }
