@@ -155,27 +155,31 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1):
 
 
 class Model:
-    """The config's GAT stack on one GPU, every step through libmega.so."""
+    """The config's GAT stack on this rank's part (k = world), every step through libmega.so."""
 
-    def __init__(self, wl, dtype, dev):
+    def __init__(self, wl, dtype, dev, rank=0, world=1):
         import torch
-        from paper_conf_icdcs_dengr24_b200.layer import GATLayer
+        from paper_conf_icdcs_dengr24_b200.dist import DistGATLayer
         self.torch = torch
         cfg = wl["cfg"]
         tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
-        self.x0 = torch.tensor(wl["x0"], device=dev).to(tdt).contiguous()
-        self.g = torch.tensor(wl["g_last"], device=dev).to(tdt).contiguous()
-        wl["layout"].bind(0)
+        lay = wl["layout"]
+        lay.bind(rank)
+        v = lay.view(rank, arrays=False)
+        self.b0, self.b1 = v["row_begin"], v["row_end"]
+        self.rows, self.part_edges = self.b1 - self.b0, v["part_edges"]
+        self.x0 = torch.tensor(wl["x0"][self.b0:self.b1], device=dev).to(tdt).contiguous()
+        self.g = torch.tensor(wl["g_last"][self.b0:self.b1], device=dev).to(tdt).contiguous()
         self.layers = []
         x = self.x0
         for li, inp in enumerate(wl["layers"]):
             w = torch.tensor(inp["w"], device=dev).to(tdt).contiguous()
-            L = GATLayer(wl["layout"], x, w, torch.tensor(inp["a_l"], device=dev),
-                         torch.tensor(inp["a_r"], device=dev), cfg.heads, cfg.head_dim, in_dim=inp["in_dim"],
-                         want_grad_x=li > 0)
-            self.layers.append(L)
-            x = L.out
-        self.launches = sum(L.launches_per_step() for L in self.layers)
+            Ld = DistGATLayer(lay, rank, x, w, torch.tensor(inp["a_l"], device=dev),
+                              torch.tensor(inp["a_r"], device=dev), cfg.heads, cfg.head_dim, in_dim=inp["in_dim"],
+                              want_grad_x=li > 0)
+            self.layers.append(Ld)
+            x = Ld.L.out
+        self.launches = sum(Ld.L.launches_per_step() for Ld in self.layers)
 
     def step(self, ev=None):
         """ev: optional dict name -> list of (start, end) event pairs to record into."""
@@ -191,16 +195,11 @@ class Model:
             e.record()
             ev.setdefault(name, []).append((s, e))
 
-        from paper_conf_icdcs_dengr24_b200 import mega as M
-        for L in self.layers:
-            timed("project_fwd", L.project)
-            timed("gat_fwd", lambda: L.attend(True))
+        for Ld in self.layers:
+            Ld.forward(timed)
         g = self.g
-        for L in reversed(self.layers):
-            timed("gat_bwd_src", lambda: L.attend_backward(g, M.MEGA_BWD_PHASE_SRC))
-            timed("gat_bwd_dst", lambda: L.attend_backward(g, M.MEGA_BWD_PHASE_DST))
-            timed("project_bwd", L.project_backward)
-            g = L.grad_x
+        for Ld in reversed(self.layers):
+            g = Ld.backward(g, timed)
 
 
 # ------------------------------------------------------------------ CPU oracle
@@ -273,107 +272,129 @@ def run_reference(args):
 
 def run_mega(args):
     import torch
+    import torch.distributed as dist
+    rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
-    if world > 1 or args.gpus > 1:
-        from paper_conf_icdcs_dengr24_b200 import dist as D
-        return D.bench_distributed(args, build_workload, METRIC, ClockSampler, peaks, algorithmic_bytes,
-                                   cpu_sample, cores)
+    local = int(os.environ.get("LOCAL_RANK", "0"))
     if not torch.cuda.is_available():
         raise SystemExit("bench.py needs a CUDA device (no CPU fallback)")
-    dev = torch.device("cuda:0")
-    torch.cuda.set_device(dev)
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    def sync_all():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
     t0 = time.time()
-    wl = build_workload(args.config, args.dtype, args.order)
+    wl = build_workload(args.config, args.dtype, args.order, rank, world)
     cfg = wl["cfg"]
-    log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s")
-    model = Model(wl, args.dtype, dev)
+    if rank == 0:
+        log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s, parts {world}")
+    model = Model(wl, args.dtype, dev, rank, world)
     for _ in range(max(3, args.warmup)):
         model.step()
-    torch.cuda.synchronize()
+    sync_all()
     # ---- device-timed region (inputs resident; inputs >> L2 so no flush) ----
     ev = {}
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    with ClockSampler(0) as clk:
-        torch.cuda.synchronize()
+    with ClockSampler(local) as clk:
+        sync_all()
         start.record()
         for _ in range(args.steps):
             model.step(ev)
         end.record()
-        torch.cuda.synchronize()
-    ms = start.elapsed_time(end) / args.steps
+        sync_all()
+    ms_t = torch.tensor([start.elapsed_time(end) / args.steps], device=dev)
+    if world > 1:
+        dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
+    ms = float(ms_t.item())
     calls = {k: float(np.mean([s.elapsed_time(e) for s, e in v])) for k, v in ev.items()}
     per_step_calls = {k: float(np.sum([s.elapsed_time(e) for s, e in v])) / args.steps for k, v in ev.items()}
     L = cfg.layers
     value = L * cfg.m / (ms * 1e-3)
-    # roofline of the dominant attention call
+    # roofline of the dominant attention call (this rank's part)
     pk = peaks()
     sb = 2 if args.dtype == "bf16" else 4
     att = {k: per_step_calls[k] for k in ("gat_fwd", "gat_bwd_src", "gat_bwd_dst")}
     dom = max(att, key=att.get)
-    bytes_per_launch = algorithmic_bytes(dom, cfg.n, cfg.m, cfg.heads, cfg.dim, sb)
+    bytes_per_launch = algorithmic_bytes(dom, cfg.n, model.part_edges, cfg.heads, cfg.dim, sb, rows=model.rows)
     achieved = bytes_per_launch / (calls[dom] * 1e-3) / 1e9
     traffic = None
     tp = os.path.join(ROOT, "profiles", f"traffic_{cfg.name}_{args.dtype}.json")
-    if os.path.exists(tp):
+    if os.path.exists(tp) and world == 1:
         traffic = json.load(open(tp)).get(dom)
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
                 "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "algorithmic_bytes": bytes_per_launch,
-                "launch_ms": calls[dom], "peak_source": pk["source"]}
-    # ---- e2e: pinned host inputs -> device each step, grads back ----
+                "launch_ms": calls[dom], "peak_source": pk["source"],
+                "note": "algorithmic bytes = compulsory floor (each gathered row once, DESIGN.md §5)"}
+    # ---- e2e: this step's inputs from pinned host memory, parameter grads back ----
     e2e = None
     if not args.no_e2e:
         hx = model.x0.cpu().pin_memory()
         hg = model.g.cpu().pin_memory()
-        outs = [L_.grad_w for L_ in model.layers] + [L_.grad_attn_l for L_ in model.layers] + \
-               [L_.grad_attn_r for L_ in model.layers]
+        outs = [Ld.L.grad_w for Ld in model.layers] + [Ld.L.grad_attn_l for Ld in model.layers] + \
+               [Ld.L.grad_attn_r for Ld in model.layers]
         hout = [torch.empty(o.shape, dtype=o.dtype).pin_memory() for o in outs]
         h2d = hx.numel() * hx.element_size() + hg.numel() * hg.element_size()
         d2h = sum(o.numel() * o.element_size() for o in outs)
-        for _ in range(2):
-            model.x0.copy_(hx, non_blocking=True); model.g.copy_(hg, non_blocking=True)
-            model.step()
-            for h, o in zip(hout, outs):
-                h.copy_(o, non_blocking=True)
-            torch.cuda.synchronize()
-        s2, e2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        s2.record()
-        for _ in range(args.steps):
+
+        def e2e_step():
             model.x0.copy_(hx, non_blocking=True)
             model.g.copy_(hg, non_blocking=True)
             model.step()
             for h, o in zip(hout, outs):
                 h.copy_(o, non_blocking=True)
+
+        for _ in range(2):
+            e2e_step()
+        sync_all()
+        s2, e2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s2.record()
+        for _ in range(args.steps):
+            e2e_step()
         e2.record()
-        torch.cuda.synchronize()
-        ms_e2e = s2.elapsed_time(e2) / args.steps
+        sync_all()
+        me = torch.tensor([s2.elapsed_time(e2) / args.steps], device=dev)
+        if world > 1:
+            dist.all_reduce(me, op=dist.ReduceOp.MAX)
+        ms_e2e = float(me.item())
         e2e = {"value": L * cfg.m / (ms_e2e * 1e-3), "unit": "edges/s", "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": int(d2h), "ms_per_step": ms_e2e}
-    # ---- CPU oracle baseline (bounded sample) ----
+    # ---- CPU oracle baseline (bounded sample; rank 0 at N = 1 only) ----
     cpu = None
-    if not args.no_cpu_baseline:
+    if not args.no_cpu_baseline and world == 1:
         run, R = cpu_sample(wl, args.cpu_seconds, cfg.heads, cfg.head_dim)
         t, e = run(R)
         cpu = {"value": e / t, "unit": "edges/s", "cores": cores(), "kind": "oracle",
                "sample": f"oracle/c fp64 one-layer GAT fwd+bwd over the first {R} destination rows of the MEGA "
                          f"order ({e} edges, all sources, n={cfg.n}); {t:.1f} s"}
-    st = wl["layout"].stats()
-    line = {
-        "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": 1, "steps": args.steps,
-        "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
-        "vs_baseline": None, "dtype": args.dtype,
-        "data": "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)",
-        "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
-                   "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
-                   "order": args.order, "parallelism": "single GPU",
-                   "value_definition": "layers * E / step time (each layer's edges fwd+bwd)",
-                   "l2": "no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)},
-        "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
-        "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
-        "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",
-                                      "tile_unique_sources", "max_in_degree", "preprocess_seconds")},
-        "setup_s": time.time() - t0,
-    }
-    print(json.dumps(line), flush=True)
+    if rank == 0:
+        st = wl["layout"].stats()
+        line = {
+            "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
+            "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
+            "vs_baseline": None, "dtype": args.dtype,
+            "data": "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)",
+            "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
+                       "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
+                       "order": args.order,
+                       "parallelism": "single GPU" if world == 1 else
+                       f"dst-partitioned x{world} (NCCL all-gather-v of [Wh|er], reduce-to-owner of [dWh|der])",
+                       "value_definition": "layers * E / step time (each layer's edges fwd+bwd; max over ranks)",
+                       "l2": "no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)},
+            "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
+            "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
+            "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",
+                                          "tile_unique_sources", "max_in_degree", "preprocess_seconds")},
+            "setup_s": time.time() - t0,
+        }
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier()
+        dist.destroy_process_group()
 
 
 def main():
