@@ -176,7 +176,7 @@ class Model:
             w = torch.tensor(inp["w"], device=dev).to(tdt).contiguous()
             Ld = DistGATLayer(lay, rank, x, w, torch.tensor(inp["a_l"], device=dev),
                               torch.tensor(inp["a_r"], device=dev), cfg.heads, cfg.head_dim, in_dim=inp["in_dim"],
-                              want_grad_x=li > 0)
+                              want_grad_x=li > 0, lp_only=dtype == "bf16")
             self.layers.append(Ld)
             x = Ld.L.out
         self.launches = sum(Ld.L.launches_per_step() for Ld in self.layers)

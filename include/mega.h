@@ -158,6 +158,9 @@ typedef struct {
 #define MEGA_BWD_PHASE_DST 4u    /* mega_gat_bwd: destination pass over this part's rows -> adds
                                     del_i a_l to grad_feat, writes grad_feat_lp, grad_attn_l and
                                     grad_attn_r (partials of this part for k > 1).  Neither flag = both. */
+#define MEGA_BWD_LP_ONLY 8u      /* mega_gat_bwd with grad_feat_lp != NULL: the final rows are written
+                                    only to grad_feat_lp (grad_feat keeps the source-phase partial);
+                                    saves a D*4-byte write per row when only the GEMM operand is needed */
 
 int mega_abi_version(void);
 const char *mega_status_string(mega_status s);

@@ -645,6 +645,7 @@ struct BwdArgs {
   double *ws_dal, *ws_dar;
   float *gal, *gar;
   int nb_dst;
+  int lp_only;  // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
 };
 
@@ -888,16 +889,31 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
   const int H = a.H;
   const uint64_t pol_cold = policy_first();
   int hv[V];
-  float dal[V][EPV], dar[V][EPV];
+  float dal[V][EPV], dar[V][EPV], alv[V][EPV];
 #pragma unroll
   for (int v = 0; v < V; ++v) {
     hv[v] = ((v * G + gl) * EPV) / FF;
 #pragma unroll
-    for (int k = 0; k < EPV; ++k) { dal[v][k] = 0.f; dar[v][k] = 0.f; }
+    for (int k = 0; k < EPV; ++k) { dal[v][k] = 0.f; dar[v][k] = 0.f; alv[v][k] = a.al[(v * G + gl) * EPV + k]; }
   }
   const T *feat = static_cast<const T *>(a.feat);
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
+    const int64_t grow = a.L.row_begin + r;
+    // row-local operands first: they do not depend on del, so their latency
+    // overlaps the dz gather below
+    float *gr = a.gfeat + grow * a.ldgf + gl * EPV;
+    const T *wr = feat + grow * a.ldf + gl * EPV;
+    float4 part[V][EPV / 4];
+    uint4 whp[V];
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      whp[v] = ldg16(wr + v * G * EPV);
+#pragma unroll
+      for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
+    }
+    float derr[HT];
+    load_h<HT>(a.der + grow * H, H, derr);
     const int e0 = a.L.indptr[r], e1 = a.L.indptr[r + 1];
     float dp[HT];
 #pragma unroll
@@ -912,24 +928,20 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     float del[HT];
 #pragma unroll
     for (int h = 0; h < HT; ++h) del[h] = h < H ? gsum<G>(dp[h], gmask) : 0.f;
-    const int64_t grow = a.L.row_begin + r;
-    float derr[HT];
-    load_h<HT>(a.der + grow * H, H, derr);
-    float *gr = a.gfeat + grow * a.ldgf + gl * EPV;
-    const T *wr = feat + grow * a.ldf + gl * EPV;
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       const float d = sel<HT>(del, hv[v]), dr = sel<HT>(derr, hv[v]);
-      const float *alp = a.al + (v * G + gl) * EPV;
       float y[EPV], wh[EPV];
-      unpack(ldg16(wr + v * G * EPV), wh, T());
+      unpack(whp[v], wh, T());
 #pragma unroll
-      for (int k = 0; k < EPV; k += 4) {
-        const float4 t = *reinterpret_cast<const float4 *>(gr + v * G * EPV + k);
-        const float4 l4 = __ldg(reinterpret_cast<const float4 *>(alp + k));
-        y[k] = fmaf(d, l4.x, t.x); y[k + 1] = fmaf(d, l4.y, t.y);
-        y[k + 2] = fmaf(d, l4.z, t.z); y[k + 3] = fmaf(d, l4.w, t.w);
-        *reinterpret_cast<float4 *>(gr + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+      for (int k = 0; k < EPV / 4; ++k) {
+        y[4 * k] = fmaf(d, alv[v][4 * k], part[v][k].x);
+        y[4 * k + 1] = fmaf(d, alv[v][4 * k + 1], part[v][k].y);
+        y[4 * k + 2] = fmaf(d, alv[v][4 * k + 2], part[v][k].z);
+        y[4 * k + 3] = fmaf(d, alv[v][4 * k + 3], part[v][k].w);
+        if (!a.lp_only)
+          *reinterpret_cast<float4 *>(gr + v * G * EPV + 4 * k) =
+              make_float4(y[4 * k], y[4 * k + 1], y[4 * k + 2], y[4 * k + 3]);
       }
       if (a.gfeat_lp) st16(static_cast<T *>(a.gfeat_lp) + grow * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
 #pragma unroll
@@ -1371,6 +1383,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
+  a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);

@@ -68,11 +68,11 @@ class DistGATLayer:
     """One GAT layer on part `rank` of a k-part layout."""
 
     def __init__(self, layout: M.Layout, rank, x_local, w, attn_l, attn_r, heads, head_dim, in_dim=None,
-                 want_grad_x=False, group=None):
+                 want_grad_x=False, group=None, lp_only=False):
         self.group = group
         self.bounds = layout.view(rank)["bounds"]
         self.L = GATLayer(layout, x_local, w, attn_l, attn_r, heads, head_dim, part=rank, in_dim=in_dim,
-                          want_grad_x=want_grad_x)
+                          want_grad_x=want_grad_x, lp_only=lp_only)
 
     def forward(self, timed=None):
         """timed(name, fn): optional wrapper used by bench.py to time each call."""

@@ -15,8 +15,9 @@ class GATLayer:
     """Buffers and calls for one layer on one layout part (k = 1: the whole graph)."""
 
     def __init__(self, layout: M.Layout, x, w, attn_l, attn_r, heads, head_dim, part=0, in_dim=None,
-                 negative_slope=M.SLOPE, want_grad_x=False):
+                 negative_slope=M.SLOPE, want_grad_x=False, lp_only=False):
         self.layout, self.part = layout, part
+        self.lp_only = lp_only  # training path: only the bf16 operand of the projection backward is needed
         view_counts = layout.view(part, arrays=False)
         self.n = view_counts["num_nodes"]
         self.row_begin, self.row_end = view_counts["row_begin"], view_counts["row_end"]
@@ -58,6 +59,8 @@ class GATLayer:
 
     # a6-a8
     def attend_backward(self, grad_out, flags=0, stream=None):
+        if self.lp_only and self.grad_feat_lp is not None:
+            flags |= M.MEGA_BWD_LP_ONLY
         M.mega_gat_bwd(self.layout, self.part, self.feat, self.attn_l, self.attn_r, self.H, self.F, self.out,
                        grad_out, self.ctx, self.grad_feat, self.grad_attn_l, self.grad_attn_r, self.ws_b,
                        self.grad_feat_lp, self.slope, flags, stream)

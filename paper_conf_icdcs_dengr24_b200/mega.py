@@ -21,6 +21,7 @@ MEGA_FLAG_ELER_IN_CTX = 1
 MEGA_CTX_PLANES = 5  # el, er, lse, Dlt, der
 MEGA_BWD_PHASE_SRC = 2
 MEGA_BWD_PHASE_DST = 4
+MEGA_BWD_LP_ONLY = 8
 SLOPE = float(np.float32(0.2))
 
 _c = ctypes

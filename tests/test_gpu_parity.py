@@ -156,3 +156,25 @@ def test_whole_layer(cuda_device, dtype, name):
            "grad_attn_r": b["grad_attn_r"].reshape(-1), "grad_w": pb["grad_w"], "grad_x": pb["grad_x"],
            "grad_feat": b["grad_feat"].reshape(n, D)}
     hz.check(got, ref, dtype, keys=tuple(ref))
+
+
+def test_lp_only_flag_matches(cuda_device):
+    """MEGA_BWD_LP_ONLY writes the same bf16 projection operand as the full path."""
+    cfg = synth.scaled(synth.CONFIGS["products"], 3000, 60000)
+    ip, ix, _ = synth.make_graph(cfg)
+    inp = synth.make_layer_inputs(cfg)
+    x, w = synth.bf16_round(inp["x"]), synth.bf16_round(inp["w"])
+    g = synth.bf16_round(inp["grad_out"])
+    lay = M.mega_preprocess(ip, ix)
+    lay.bind(0)
+    perm = lay.view(0)["perm"].astype(np.int64)
+    gt = torch.tensor(g[perm], device="cuda").bfloat16()
+    res = []
+    for lp_only in (False, True):
+        L = hz.layer(lay, x[perm], w, inp["a_l"], inp["a_r"], cfg.heads, cfg.head_dim, "bf16")
+        L.lp_only = lp_only
+        L.step(gt)
+        torch.cuda.synchronize()
+        res.append((L.grad_feat_lp.clone(), L.grad_w.clone(), L.grad_attn_l.clone(), L.grad_attn_r.clone()))
+    for a, b in zip(*res):
+        assert torch.equal(a, b)
