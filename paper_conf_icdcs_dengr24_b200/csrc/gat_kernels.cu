@@ -689,6 +689,12 @@ template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G, SP = HT + 1;
   constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U0 < G ? U0 : G;
+  // transpose-butterfly reduction of the U*V per-lane dot products over the
+  // LPH lanes of a head: log2(LPH) shuffles per batch instead of U*V*log2(LPH),
+  // and each lane then owns one (edge, vector) value (index `bidx`)
+  constexpr int NB = U * V;
+  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
+  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
   __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
   __shared__ float s_d[WPB][32][SP];  // Dlt_i
   __shared__ float s_z[WPB][32][SP];  // dz out
@@ -702,6 +708,12 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
+  int bidx = 0;  // butterfly: the (u, v) value this lane ends up holding, i = u * V + v
+#pragma unroll
+  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
+  const int bu = bidx / V, bv = bidx % V;
+  const int bhead = ((bv * G + gl) * EPV) / FF;
+  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
   const T *feat = static_cast<const T *>(a.feat);
   const T *goutl = static_cast<const T *>(a.gout) + gl * EPV;
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
@@ -714,7 +726,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
-    float whf[V][EPV], acc[V][EPV], derv[V];
+    float whf[V][EPV], acc[V][EPV], derv[V], dacc = 0.f;
     {
       const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
@@ -773,16 +785,42 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
             }
             p[u][v] = s;
           }
-        head_reduce<G, U, V, LPH>(p, gmask);
+        if constexpr (BFLY) {
+          float q[NB];
 #pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int er_ = rb + k0 + u;
+          for (int i = 0; i < NB; ++i) q[i] = p[i / V][i % V];
 #pragma unroll
-          for (int v = 0; v < V; ++v) {
-            const float sa = s_a[w][er_][hv[v]];
-            const float dz = fabsf(sa) * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
-            derv[v] += dz;
-            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
+          for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
+            if (n > 1) {
+              const bool up = (gl & o) != 0;
+#pragma unroll
+              for (int i = 0; i < n / 2; ++i) {
+                const float send = up ? q[i] : q[i + n / 2];
+                const float keep = up ? q[i + n / 2] : q[i];
+                q[i] = keep + __shfl_xor_sync(gmask, send, o, G);
+              }
+              n /= 2;
+            } else {
+              q[0] += __shfl_xor_sync(gmask, q[0], o, G);
+            }
+          }
+          const int er_ = rb + k0 + bu;
+          const float sa = s_a[w][er_][bhead];
+          const float dz = fabsf(sa) * (q[0] - s_d[w][er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
+          dacc += dz;
+          if (bwriter) s_z[w][er_][bhead] = dz;
+        } else {
+          head_reduce<G, U, V, LPH>(p, gmask);
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int er_ = rb + k0 + u;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const float sa = s_a[w][er_][hv[v]];
+              const float dz = fabsf(sa) * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+              derv[v] += dz;
+              if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
+            }
           }
         }
       };
@@ -814,6 +852,21 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
         }
       }
       __syncwarp(gmask);
+    }
+    if constexpr (BFLY) {  // sum over the edge slots u, then fetch each vector's head total
+      float dsum = dacc;
+#pragma unroll
+      for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o, G);
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        int src = gl;
+#pragma unroll
+        for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
+          const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
+          src = bit ? (src | o) : (src & ~o);
+        }
+        derv[v] = __shfl_sync(gmask, dsum, src, G);
+      }
     }
     if (item.w < 0) {
       float *orow = a.gfeat + j * a.ldgf + gl * EPV;
