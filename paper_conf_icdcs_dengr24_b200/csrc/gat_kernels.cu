@@ -254,10 +254,19 @@ struct FwdArgs {
 // register batches of U rows (batch b+1 is requested before batch b is
 // accumulated).  Batches are branch-free: the tail of a chunk re-reads its
 // last row (an L1 hit) with weight p = 0.
-template <typename T, int G, int V, int HT>
-__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const FwdArgs a) {
+// VAR selects the batch pipeline: 0 = two register batches of U (2U rows in
+// flight per lane, 2 CTAs/SM), 1 = one batch of U (3 CTAs/SM), 2 = one batch of 2U.
+template <int V, int VAR> struct FwdCfg {
+  static constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 4 : 8);
+  static constexpr int U = VAR == 2 ? 2 * U0 : U0;
+  static constexpr bool DB = VAR == 0;
+  static constexpr int MINB = V >= 4 ? 1 : (VAR == 1 ? 3 : 2);
+};
+template <typename T, int G, int V, int HT, int VAR = 0>
+__global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(const FwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 4 : 8), U = U0 < G ? U0 : G;  // U divides G
+  constexpr int U = FwdCfg<V, VAR>::U < G ? FwdCfg<V, VAR>::U : G;  // U divides G
+  constexpr bool DB = FwdCfg<V, VAR>::DB;
   __shared__ float s_p[WPB][32][SP];
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
@@ -297,12 +306,12 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
       const int jr = ld_stream(a.L.src + min(e, item.z - 1), pol_cold);
       float erj[HT];
       load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
-      uint4 ra[U][V], rz[U][V];
+      uint4 ra[U][V], rz[DB ? U : 1][V];
 #pragma unroll
       for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)__shfl_sync(gmask, jr, min(u, cnt - 1), G));
       s_j[w][lane] = jr;
       __syncwarp(gmask);
-      if (nb > 1) {
+      if (DB && nb > 1) {
 #pragma unroll
         for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_j[w][rb + min(U + u, cnt - 1)]);
       }
@@ -339,18 +348,28 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_fwd_kernel(const Fw
             for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
           }
       };
-      for (int b = 0; b < nb; b += 2) {
-        consume(ra, b * U);
-        if (b + 2 < nb) {
+      if constexpr (DB) {
+        for (int b = 0; b < nb; b += 2) {
+          consume(ra, b * U);
+          if (b + 2 < nb) {
 #pragma unroll
-          for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_j[w][rb + min((b + 2) * U + u, cnt - 1)]);
-        }
-        if (b + 1 < nb) {
-          consume(rz, (b + 1) * U);
-          if (b + 3 < nb) {
-#pragma unroll
-            for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_j[w][rb + min((b + 3) * U + u, cnt - 1)]);
+            for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_j[w][rb + min((b + 2) * U + u, cnt - 1)]);
           }
+          if (b + 1 < nb) {
+            consume(rz, (b + 1) * U);
+            if (b + 3 < nb) {
+#pragma unroll
+              for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_j[w][rb + min((b + 3) * U + u, cnt - 1)]);
+            }
+          }
+        }
+      } else {
+        for (int b = 0; b < nb; ++b) {
+          if (b > 0) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_j[w][rb + min(b * U + u, cnt - 1)]);
+          }
+          consume(ra, b * U);
         }
       }
       __syncwarp(gmask);
@@ -1130,6 +1149,14 @@ bool use_ring() {
   }
   return v == 1;
 }
+int fwd_variant() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_FWD_VAR");
+    v = e ? std::atoi(e) : 0;
+  }
+  return v;
+}
 int ring_blocks(size_t smem) {
   const size_t per_sm = 227 * 1024;
   return (int)std::max<size_t>(1, per_sm / (smem + 12 * 1024));
@@ -1276,9 +1303,15 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
             return;
           }
         }
-        auto k = gat_fwd_kernel<T, G, V, HT>;
-        k<<<grid_for(k, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
-        rc = check_launch(st, "gat_fwd_kernel");
+        auto launch = [&](auto kern_fn) {
+          kern_fn<<<grid_for(kern_fn, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+          rc = check_launch(st, "gat_fwd_kernel");
+        };
+        switch (fwd_variant()) {
+          case 1: launch(gat_fwd_kernel<T, G, V, HT, 1>); break;
+          case 2: launch(gat_fwd_kernel<T, G, V, HT, 2>); break;
+          default: launch(gat_fwd_kernel<T, G, V, HT, 0>); break;
+        }
       });
       if (rc != MEGA_OK) return;
     }
