@@ -153,6 +153,24 @@ template <int HT> __device__ __forceinline__ void load_h_v(const float *p, int H
       if (h < H) asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v[h]) : "l"(p + h));
   }
 }
+// Packed fp32x2 FMA (sm_100 FFMA2): d{0,1} += a{0,1} * b, and the two-lane dot
+// s{0,1} += a{0,1} * c{0,1}; halves the FMA issue count of the row loops.
+__device__ __forceinline__ void ffma2s(float &d0, float &d1, float a0, float a1, float b) {
+  unsigned long long D, A, B;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(A) : "f"(a0), "f"(a1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(D) : "f"(d0), "f"(d1));
+  asm("mov.b64 %0, {%1, %1};" : "=l"(B) : "f"(b));
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(D) : "l"(A), "l"(B));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(d0), "=f"(d1) : "l"(D));
+}
+__device__ __forceinline__ void ffma2v(float &d0, float &d1, float a0, float a1, float c0, float c1) {
+  unsigned long long D, A, C;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(A) : "f"(a0), "f"(a1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(C) : "f"(c0), "f"(c1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(D) : "f"(d0), "f"(d1));
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(D) : "l"(A), "l"(C));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(d0), "=f"(d1) : "l"(D));
+}
 // exp / log on the SFU: ex2.approx / lg2.approx (max rel. error ~2^-22; the
 // x*log2(e) rounding adds ~1e-7 |x| relative, within the fp32 parity bar)
 __device__ __forceinline__ float fexp(float x) {
@@ -345,7 +363,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
             float x[EPV];
             unpack(raw[u][v], x, T());
 #pragma unroll
-            for (int k = 0; k < EPV; ++k) acc[v][k] = fmaf(pw, x[k], acc[v][k]);
+            for (int k = 0; k < EPV; k += 2) ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], pw);
           }
       };
       if constexpr (DB) {
@@ -796,13 +814,13 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
             const float al = fabsf(s_a[w][rb + k0 + u][hv[v]]);
             float x[EPV];
             unpack(raw[u][v], x, T());
-            float s = 0.f;
+            float s0 = 0.f, s1 = 0.f;
 #pragma unroll
-            for (int k = 0; k < EPV; ++k) {
-              s = fmaf(x[k], whf[v][k], s);
-              acc[v][k] = fmaf(al, x[k], acc[v][k]);
+            for (int k = 0; k < EPV; k += 2) {
+              ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
+              ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
             }
-            p[u][v] = s;
+            p[u][v] = s0 + s1;
           }
         if constexpr (BFLY) {
           float q[NB];
