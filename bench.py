@@ -46,6 +46,7 @@ def parse():
     ap.add_argument("--config", default="products")
     ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
     ap.add_argument("--order", default="traversal")
+    ap.add_argument("--window", type=int, default=0, help="traversal window omega (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -126,7 +127,7 @@ def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
 
 
 # ------------------------------------------------------------------ workload
-def build_workload(cfg_name, dtype, order, rank=0, world=1):
+def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0):
     import synth
     cfg = synth.CONFIGS[cfg_name]
     t0 = time.time()
@@ -134,7 +135,7 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1):
     t_gen = time.time() - t0
     from paper_conf_icdcs_dengr24_b200 import mega as M
     t0 = time.time()
-    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world)
+    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
     layers = []
@@ -289,7 +290,7 @@ def run_mega(args):
             dist.barrier()
 
     t0 = time.time()
-    wl = build_workload(args.config, args.dtype, args.order, rank, world)
+    wl = build_workload(args.config, args.dtype, args.order, rank, world, args.window)
     cfg = wl["cfg"]
     if rank == 0:
         log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s, parts {world}")
