@@ -47,6 +47,7 @@ def parse():
     ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
     ap.add_argument("--order", default="traversal")
     ap.add_argument("--window", type=int, default=0, help="traversal window omega (0 = auto)")
+    ap.add_argument("--seg-edges", type=int, default=0, help="work-item segment size S (0 = auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -127,7 +128,7 @@ def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
 
 
 # ------------------------------------------------------------------ workload
-def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0):
+def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0):
     import synth
     cfg = synth.CONFIGS[cfg_name]
     t0 = time.time()
@@ -135,7 +136,7 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0):
     t_gen = time.time() - t0
     from paper_conf_icdcs_dengr24_b200 import mega as M
     t0 = time.time()
-    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window)
+    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window, seg_edges=seg_edges)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
     layers = []
@@ -290,7 +291,7 @@ def run_mega(args):
             dist.barrier()
 
     t0 = time.time()
-    wl = build_workload(args.config, args.dtype, args.order, rank, world, args.window)
+    wl = build_workload(args.config, args.dtype, args.order, rank, world, args.window, args.seg_edges)
     cfg = wl["cfg"]
     if rank == 0:
         log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s, parts {world}")
