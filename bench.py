@@ -124,6 +124,11 @@ def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
                                                     + 3 * rows * H * 4 + 4 * m * H + n * D * 4)
     if call == "gat_bwd_dst":  # KB5: indptr, csr2csc, dz, dWh RMW, Wh, bf16 copy
         return 4 * (rows + 1) + 4 * m + 4 * m * H + 2 * rows * D * 4 + rows * D * sb + (rows * D * sb if sb == 2 else 0)
+    if call == "gat_bwd":      # one call, LP_ONLY (bf16): KB3 + KB4 + KB5 with the partial kept in bf16
+        pb = sb if sb == 2 else 4
+        return ((2 * rows * D * sb + rows * H * 4)
+                + (4 * m + 16 * n + n * D * sb + n * H * 4 + rows * D * sb + 3 * rows * H * 4 + 4 * m * H + n * D * pb)
+                + (4 * (rows + 1) + 4 * m + 4 * m * H + 2 * rows * D * pb + rows * D * sb + rows * H * 4))
     raise KeyError(call)
 
 
@@ -320,7 +325,7 @@ def run_mega(args):
     # roofline of the dominant attention call (this rank's part)
     pk = peaks()
     sb = 2 if args.dtype == "bf16" else 4
-    att = {k: per_step_calls[k] for k in ("gat_fwd", "gat_bwd_src", "gat_bwd_dst")}
+    att = {k: per_step_calls[k] for k in ("gat_fwd", "gat_bwd", "gat_bwd_src", "gat_bwd_dst") if k in per_step_calls}
     dom = max(att, key=att.get)
     bytes_per_launch = algorithmic_bytes(dom, cfg.n, model.part_edges, cfg.heads, cfg.dim, sb, rows=model.rows)
     achieved = bytes_per_launch / (calls[dom] * 1e-3) / 1e9

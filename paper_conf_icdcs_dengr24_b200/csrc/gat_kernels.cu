@@ -682,7 +682,8 @@ struct BwdArgs {
   double *ws_dal, *ws_dar;
   float *gal, *gar;
   int nb_dst;
-  int lp_only;  // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
+  int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
+  int lp_partial;  // ... and (both phases in one call) the source-phase partial lives in gfeat_lp too
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
 };
 
@@ -722,10 +723,12 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // der_j into the der plane of ctx.  g rows stream through two register
 // batches; batches are branch-free (the chunk tail re-reads its last row with
 // alpha = 0).
-template <typename T, int G, int V, int HT>
+// VAR: 0 = two register batches of U rows, 1 = one batch of 2U rows.
+template <typename T, int G, int V, int HT, int VAR = 0>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G, SP = HT + 1;
-  constexpr int U0 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U0 < G ? U0 : G;
+  constexpr int U1 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U0 = VAR == 1 ? 2 * U1 : U1, U = U0 < G ? U0 : G;
+  constexpr bool DB = VAR == 0;
   // transpose-butterfly reduction of the U*V per-lane dot products over the
   // LPH lanes of a head: log2(LPH) shuffles per batch instead of U*V*log2(LPH),
   // and each lane then owns one (edge, vector) value (index `bidx`)
@@ -786,12 +789,12 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
       load_h<HT>(a.el + gi * H, H, eli);
       load_h<HT>(a.lse + gi * H, H, lsei);
       load_h<HT>(a.dlt + gi * H, H, dli);
-      uint4 ra[U][V], rz[U][V];
+      uint4 ra[U][V], rz[DB ? U : 1][V];
 #pragma unroll
       for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)__shfl_sync(gmask, ir, min(u, cnt - 1), G));
       s_i[w][lane] = ir;
       __syncwarp(gmask);
-      if (nb > 1) {
+      if (DB && nb > 1) {
 #pragma unroll
         for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_i[w][rb + min(U + u, cnt - 1)]);
       }
@@ -861,18 +864,28 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
           }
         }
       };
-      for (int b = 0; b < nb; b += 2) {
-        consume(ra, b * U);
-        if (b + 2 < nb) {
+      if constexpr (DB) {
+        for (int b = 0; b < nb; b += 2) {
+          consume(ra, b * U);
+          if (b + 2 < nb) {
 #pragma unroll
-          for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_i[w][rb + min((b + 2) * U + u, cnt - 1)]);
-        }
-        if (b + 1 < nb) {
-          consume(rz, (b + 1) * U);
-          if (b + 3 < nb) {
-#pragma unroll
-            for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_i[w][rb + min((b + 3) * U + u, cnt - 1)]);
+            for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_i[w][rb + min((b + 2) * U + u, cnt - 1)]);
           }
+          if (b + 1 < nb) {
+            consume(rz, (b + 1) * U);
+            if (b + 3 < nb) {
+#pragma unroll
+              for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)s_i[w][rb + min((b + 3) * U + u, cnt - 1)]);
+            }
+          }
+        }
+      } else {
+        for (int b = 0; b < nb; ++b) {
+          if (b > 0) {
+#pragma unroll
+            for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)s_i[w][rb + min(b * U + u, cnt - 1)]);
+          }
+          consume(ra, b * U);
         }
       }
       __syncwarp(gmask);
@@ -910,13 +923,16 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
 #pragma unroll
       for (int v = 0; v < V; ++v) {
         const float *arp = a.ar + (v * G + gl) * EPV;
+        float y[EPV];
 #pragma unroll
         for (int k = 0; k < EPV; k += 4) {
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
-          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) =
-              make_float4(fmaf(derv[v], r4.x, acc[v][k]), fmaf(derv[v], r4.y, acc[v][k + 1]),
-                          fmaf(derv[v], r4.z, acc[v][k + 2]), fmaf(derv[v], r4.w, acc[v][k + 3]));
+          y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
+          y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
+          if (!a.lp_partial)
+            *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
         }
+        if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
@@ -963,7 +979,13 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
       }
       float *orow = a.gfeat + j * a.ldgf + col;
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) orow[k] = fmaf(der, a.ar[col + k], y[k]);
+      for (int k = 0; k < EPV; ++k) y[k] = fmaf(der, a.ar[col + k], y[k]);
+      if (a.lp_partial) {
+        st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + col, pack(y, T()));
+      } else {
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) orow[k] = y[k];
+      }
     }
   }
 }
@@ -999,8 +1021,16 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       whp[v] = ldg16(wr + v * G * EPV);
+      if (a.lp_partial) {  // bf16 partial (one-call training path, k = 1)
+        float t[EPV];
+        unpack(*reinterpret_cast<const uint4 *>(static_cast<const T *>(a.gfeat_lp) + grow * a.ldlp +
+                                                 (v * G + gl) * EPV), t, T());
 #pragma unroll
-      for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
+        for (int k = 0; k < EPV / 4; ++k) part[v][k] = make_float4(t[4 * k], t[4 * k + 1], t[4 * k + 2], t[4 * k + 3]);
+      } else {
+#pragma unroll
+        for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
+      }
     }
     float derr[HT];
     load_h<HT>(a.der + grow * H, H, derr);
@@ -1171,6 +1201,14 @@ int fwd_variant() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_FWD_VAR");
+    v = e ? std::atoi(e) : 0;
+  }
+  return v;
+}
+int bwd_variant() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_BWD_VAR");
     v = e ? std::atoi(e) : 0;
   }
   return v;
@@ -1359,8 +1397,9 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
           if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
         }
         if (a.L.n_bwd_items > 0) {
-          auto ks = gat_bwd_src_kernel<T, G, V, HT>;
-          ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+          auto launch = [&](auto ks) { ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a); };
+          if (bwd_variant() == 1) launch(gat_bwd_src_kernel<T, G, V, HT, 1>);
+          else launch(gat_bwd_src_kernel<T, G, V, HT, 0>);
           if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
         }
         if (a.L.n_bwd_splits > 0) {
@@ -1488,6 +1527,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
+  a.lp_partial = a.lp_only && !(flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);

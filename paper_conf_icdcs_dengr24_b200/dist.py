@@ -87,10 +87,13 @@ class DistGATLayer:
     def backward(self, grad_out_local, timed=None):
         L = self.L
         t = timed or (lambda name, fn: fn())
-        t("gat_bwd_src", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_SRC))
-        t("comm_bwd", lambda: (reduce_to_owners(L.grad_feat, self.bounds, self.group),
-                               reduce_to_owners(L.ctx[4], self.bounds, self.group)))  # [dWh | der]
-        t("gat_bwd_dst", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_DST))
+        if _world(self.group) == 1:  # one call: lets LP_ONLY keep the partial in the bf16 operand
+            t("gat_bwd", lambda: L.attend_backward(grad_out_local, 0))
+        else:
+            t("gat_bwd_src", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_SRC))
+            t("comm_bwd", lambda: (reduce_to_owners(L.grad_feat, self.bounds, self.group),
+                                   reduce_to_owners(L.ctx[4], self.bounds, self.group)))  # [dWh | der]
+            t("gat_bwd_dst", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_DST))
         t("project_bwd", L.project_backward)
         if _world(self.group) > 1:
             for x in (L.grad_w, L.grad_attn_l, L.grad_attn_r):
