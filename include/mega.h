@@ -159,10 +159,9 @@ typedef struct {
                                     del_i a_l to grad_feat, writes grad_feat_lp, grad_attn_l and
                                     grad_attn_r (partials of this part for k > 1).  Neither flag = both. */
 #define MEGA_BWD_LP_ONLY 8u      /* mega_gat_bwd with grad_feat_lp != NULL: the final rows are written
-                                    only to grad_feat_lp (the GEMM operand of mega_project_bwd); with
-                                    both phases in one call the source-phase partial is also kept in
-                                    grad_feat_lp (dtype) and grad_feat is not touched; with a phase
-                                    flag grad_feat keeps the fp32 partial.  Training-path traffic saver */
+                                    only to grad_feat_lp (the GEMM operand of mega_project_bwd);
+                                    grad_feat keeps the fp32 source-phase partial.  Saves a D*4-byte
+                                    write per row on the training path */
 
 int mega_abi_version(void);
 const char *mega_status_string(mega_status s);

@@ -1527,7 +1527,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
-  a.lp_partial = a.lp_only && !(flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) ? 1 : 0;
+  a.lp_partial = 0;  // bf16 partial measured no faster than the fp32 partial (latency-bound); kept off
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
