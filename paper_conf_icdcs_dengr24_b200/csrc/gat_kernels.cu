@@ -443,7 +443,7 @@ template <int N> __device__ __forceinline__ void cp_async_wait() {
 }
 
 template <typename T, int V, int HT, int P>
-__global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
+__global__ void __launch_bounds__(TPB, 2) gat_fwd_ring_kernel(const FwdArgs a) {
   constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, SP = HT + 1, RSLOT = 4 * P;
   extern __shared__ uint4 ring_all[];   // [WPB][RSLOT][V][32]
   __shared__ float s_p[WPB][32][SP];
@@ -456,20 +456,19 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / FF;
-  const T *feat = static_cast<const T *>(a.feat);
+  const T *featl = static_cast<const T *>(a.feat) + lane * EPV;
+  const uint32_t ldf = (uint32_t)a.ldf;
   const int64_t stride = (int64_t)gridDim.x * WPB;
   auto issue_quad = [&](int q, int cnt) {
 #pragma unroll
     for (int r = 0; r < 4; ++r) {
-      const int k = 4 * q + r;
-      if (k < cnt) {
-        const uint32_t jj = (uint32_t)s_j[w][k];
-        const T *rp = feat + (int64_t)(jj & idm) * a.ldf + lane * EPV;
-        const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
-        uint4 *dst = ring + ((q % P) * 4 + r) * V * 32 + lane;
+      const int k = min(4 * q + r, cnt - 1);  // the tail re-reads the last row (weight p = 0)
+      const uint32_t jj = (uint32_t)s_j[w][k];
+      const T *rp = featl + (jj & idm) * ldf;
+      const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
+      uint4 *dst = ring + ((q % P) * 4 + r) * V * 32 + lane;
 #pragma unroll
-        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
-      }
+      for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
     }
     cp_async_commit();
   };
@@ -488,7 +487,7 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
     for (int base = item.y; base < item.z; base += G) {
       const int e = base + lane;
       const bool valid = e < item.z;
-      const int jr = valid ? ld_stream(a.L.src + e, pol_cold) : 0;
+      const int jr = ld_stream(a.L.src + min(e, item.z - 1), pol_cold);
       const int cnt = min(G, item.z - base), nq = (cnt + 3) >> 2;
       float erj[HT];
       load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
@@ -525,16 +524,14 @@ __global__ void __launch_bounds__(TPB, 1) gat_fwd_ring_kernel(const FwdArgs a) {
 #pragma unroll
         for (int r = 0; r < 4; ++r) {
           const int k = 4 * q + r;
-          if (k < cnt) {
-            const uint4 *src = ring + ((q % P) * 4 + r) * V * 32 + lane;
+          const uint4 *src = ring + ((q % P) * 4 + r) * V * 32 + lane;
 #pragma unroll
-            for (int v = 0; v < V; ++v) {
-              const float pw = s_p[w][k][hv[v]];
-              float x[EPV];
-              unpack(src[v * 32], x, T());
+          for (int v = 0; v < V; ++v) {
+            const float pw = s_p[w][k][hv[v]];
+            float x[EPV];
+            unpack(src[v * 32], x, T());
 #pragma unroll
-              for (int kk = 0; kk < EPV; ++kk) acc[v][kk] = fmaf(pw, x[kk], acc[v][kk]);
-            }
+            for (int kk = 0; kk < EPV; kk += 2) ffma2s(acc[v][kk], acc[v][kk + 1], x[kk], x[kk + 1], pw);
           }
         }
         if (q + P < nq) issue_quad(q + P, cnt);
@@ -1344,7 +1341,7 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
         if constexpr (G == 32) {
           if (use_ring()) {
             constexpr int RB = 32 * V * 16;                       // bytes per row
-            constexpr int P = RB >= 4096 ? 1 : (RB >= 2048 ? 3 : (RB >= 1024 ? 6 : 8));  // <= 192 KB ring
+            constexpr int P = RB >= 4096 ? 1 : (RB >= 2048 ? 1 : (RB >= 1024 ? 3 : 6));  // <= 96 KB ring per CTA, 2 CTAs/SM
             auto k = gat_fwd_ring_kernel<T, V, HT, P>;
             const size_t smem = (size_t)WPB * 4 * P * RB;
             static bool attr = false;
