@@ -48,6 +48,8 @@ def parse():
     ap.add_argument("--order", default="traversal")
     ap.add_argument("--window", type=int, default=0, help="traversal window omega (0 = auto)")
     ap.add_argument("--seg-edges", type=int, default=0, help="work-item segment size S (0 = auto)")
+    ap.add_argument("--block-rows", type=int, default=-1,
+                    help="L2 blocking B (DESIGN.md R24): -1 = auto (0.4 L2 / row bytes), 0 = off")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -133,15 +135,31 @@ def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
 
 
 # ------------------------------------------------------------------ workload
-def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0):
+def block_rows_for(cfg, dtype, block_rows=-1, l2_bytes=None):
+    """-1 -> auto: 0.4 of the device L2 in gathered rows (D * bytes per element)."""
+    if block_rows >= 0:
+        return block_rows
+    from paper_conf_icdcs_dengr24_b200 import mega as M
+    if l2_bytes is None:
+        try:
+            import torch
+            l2_bytes = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+        except Exception:  # noqa: BLE001 - no device: the B200 figure
+            l2_bytes = 126 * 1024 * 1024
+    return M.auto_block_rows(cfg.dim * (2 if dtype == "bf16" else 4), l2_bytes)
+
+
+def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1):
     import synth
     cfg = synth.CONFIGS[cfg_name]
+    block_rows = block_rows_for(cfg, dtype, block_rows)
     t0 = time.time()
     indptr, indices, gstats = synth.make_graph(cfg)
     t_gen = time.time() - t0
     from paper_conf_icdcs_dengr24_b200 import mega as M
     t0 = time.time()
-    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window, seg_edges=seg_edges)
+    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window, seg_edges=seg_edges,
+                               block_rows=block_rows)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
     layers = []
@@ -253,7 +271,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    wl = build_workload(args.config, args.dtype, args.order)
+    wl = build_workload(args.config, args.dtype, args.order, block_rows=args.block_rows)
     cfg = wl["cfg"]
     per_step = max(2.0, min(10.0, 150.0 / max(1, args.steps + args.warmup)))
     run, R = cpu_sample(wl, per_step, cfg.heads, cfg.head_dim)
@@ -296,7 +314,8 @@ def run_mega(args):
             dist.barrier()
 
     t0 = time.time()
-    wl = build_workload(args.config, args.dtype, args.order, rank, world, args.window, args.seg_edges)
+    wl = build_workload(args.config, args.dtype, args.order, rank, world, args.window, args.seg_edges,
+                        args.block_rows)
     cfg = wl["cfg"]
     if rank == 0:
         log(f"[bench] {cfg.name}: gen {wl['gen_s']:.1f}s, mega_preprocess {wl['pre_s']:.1f}s, parts {world}")
@@ -387,7 +406,7 @@ def run_mega(args):
             "data": "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)",
             "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
                        "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
-                       "order": args.order,
+                       "order": args.order, "block_rows": st["block_rows"],
                        "parallelism": "single GPU" if world == 1 else
                        f"dst-partitioned x{world} (NCCL all-gather-v of [Wh|er], reduce-to-owner of [dWh|der])",
                        "value_definition": "layers * E / step time (each layer's edges fwd+bwd; max over ranks)",
@@ -395,7 +414,8 @@ def run_mega(args):
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
             "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
             "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",
-                                          "tile_unique_sources", "max_in_degree", "preprocess_seconds")},
+                                          "tile_unique_sources", "max_in_degree", "preprocess_seconds",
+                                          "block_rows", "num_blocks", "block_sweeps")},
             "setup_s": time.time() - t0,
         }
         print(json.dumps(line), flush=True)

@@ -106,6 +106,14 @@ typedef struct {
   int32_t seg_edges;     /* S: rows/sources with more edges are split into segments; 0 = auto */
   int32_t num_parts;     /* k >= 1 destination partitions (one per GPU) */
   uint64_t seed;         /* MEGA_ORDER_RANDOM only */
+  /* L2 blocking (ours, not the paper's; R24): 0 = off.  B > 0 groups
+   * the nodes into blocks of at most B nodes by size-constrained label
+   * propagation on G_u, then stably sorts the order above by block (blocks
+   * ranked by their first position in it), so the source rows one block of
+   * destinations gathers fit the 126 MB L2.  Choose B ~ 0.4 * L2 bytes / row
+   * bytes.  Each block keeps the traversal's order inside it. */
+  int32_t block_rows;
+  int32_t block_sweeps;  /* maximum label-propagation sweeps; 0 = 10 */
 } mega_schedule_opts;
 
 typedef struct mega_layout mega_layout;
@@ -120,6 +128,9 @@ typedef struct {
   int64_t tile_unique_sources; /* sum over 64-row tiles of distinct sources (reuse = m / this) */
   int64_t max_in_degree, max_out_degree;
   double preprocess_seconds;
+  int64_t block_rows;   /* B (0 = no L2 blocking) */
+  int64_t num_blocks;   /* blocks after label propagation (1 per node with B = 1) */
+  int64_t block_sweeps; /* sweeps run (stops early once a sweep changes < n/1000 labels) */
 } mega_layout_stats;
 
 /* Read-only host view of one part (for parity tests and for moving data into

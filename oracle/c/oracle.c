@@ -385,3 +385,70 @@ int ora_traverse(int64_t n, const int64_t *indptr, const int32_t *indices, int w
   free(t.aptr); free(t.adj); free(t.deg); free(t.visited); free(t.score); free(t.cursor); free(stk);
   return 0;
 }
+
+/* ---------------------------------------------------------------------------
+ * L2 blocking (R24; oracle/blocks.py states the definition).  Plain:
+ * G_u built as in ora_traverse; per visited node a full scan of the labels
+ * present among its neighbours, counted with a scratch array.
+ * label[n] out; stats[0] = sweeps run.  Returns 0.
+ * ------------------------------------------------------------------------- */
+static const int64_t *g_sort_deg;
+static int cmp_deg_id(const void *a, const void *b) {
+  int32_t x = *(const int32_t *)a, y = *(const int32_t *)b;
+  if (g_sort_deg[x] != g_sort_deg[y]) return g_sort_deg[x] < g_sort_deg[y] ? -1 : 1;
+  return (x > y) - (x < y);
+}
+
+int ora_l2_blocks(int64_t n, const int64_t *indptr, const int32_t *indices, int32_t B, int sweeps,
+                  int32_t *label, int64_t *stats) {
+  int64_t *aptr = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t k = indptr[i]; k < indptr[i + 1]; ++k)
+      if (indices[k] != i) { aptr[i + 1]++; aptr[indices[k] + 1]++; }
+  for (int64_t v = 0; v < n; ++v) aptr[v + 1] += aptr[v];
+  int32_t *adj = (int32_t *)malloc(sizeof(int32_t) * (size_t)(aptr[n] + 1));
+  int64_t *fill = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n + 1));
+  memcpy(fill, aptr, sizeof(int64_t) * (size_t)n);
+  for (int64_t i = 0; i < n; ++i)
+    for (int64_t k = indptr[i]; k < indptr[i + 1]; ++k)
+      if (indices[k] != i) { adj[fill[i]++] = indices[k]; adj[fill[indices[k]]++] = (int32_t)i; }
+  int64_t *deg = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n + 1));
+  for (int64_t v = 0; v < n; ++v) {
+    int64_t b = aptr[v], e = aptr[v + 1], w = b;
+    qsort(adj + b, (size_t)(e - b), sizeof(int32_t), cmp_i32);
+    for (int64_t k = b; k < e; ++k)
+      if (k == b || adj[k] != adj[k - 1]) adj[w++] = adj[k];
+    deg[v] = w - b;
+  }
+  int32_t *visit = (int32_t *)malloc(sizeof(int32_t) * (size_t)(n + 1));
+  int64_t *size = (int64_t *)malloc(sizeof(int64_t) * (size_t)(n + 1));
+  int64_t *cnt = (int64_t *)calloc((size_t)n + 1, sizeof(int64_t));
+  for (int64_t v = 0; v < n; ++v) { visit[v] = (int32_t)v; label[v] = (int32_t)v; size[v] = 1; }
+  g_sort_deg = deg;
+  qsort(visit, (size_t)n, sizeof(int32_t), cmp_deg_id);
+  const int T = sweeps > 0 ? sweeps : 10;
+  int run = 0;
+  for (int it = 0; it < T; ++it) {
+    run++;
+    int64_t changed = 0;
+    for (int64_t q = 0; q < n; ++q) {
+      int32_t v = visit[q];
+      if (deg[v] == 0) continue;
+      for (int64_t k = aptr[v]; k < aptr[v] + deg[v]; ++k) cnt[label[adj[k]]]++;
+      int32_t cur = label[v], best = cur;
+      /* key (cnt, l == cur, -l), maximised; cur is always a candidate */
+      for (int64_t k = aptr[v]; k < aptr[v] + deg[v]; ++k) {
+        int32_t l = label[adj[k]];
+        if (l == cur || size[l] >= B) continue;
+        int better = cnt[l] > cnt[best] || (cnt[l] == cnt[best] && best != cur && l < best);
+        if (better) best = l;
+      }
+      for (int64_t k = aptr[v]; k < aptr[v] + deg[v]; ++k) cnt[label[adj[k]]] = 0;
+      if (best != cur) { size[cur]--; size[best]++; label[v] = best; changed++; }
+    }
+    if (changed * 1000 < n) break;
+  }
+  if (stats) stats[0] = run;
+  free(aptr); free(adj); free(fill); free(deg); free(visit); free(size); free(cnt);
+  return 0;
+}

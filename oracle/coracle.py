@@ -42,6 +42,8 @@ def lib():
                                        P, P]
         L.ora_traverse.argtypes = [I64, P, P, ctypes.c_int, ctypes.c_int, P, P, P]
         L.ora_traverse.restype = ctypes.c_int
+        L.ora_l2_blocks.argtypes = [I64, P, P, ctypes.c_int32, ctypes.c_int, P, P]
+        L.ora_l2_blocks.restype = ctypes.c_int
         _lib = L
     return _lib
 
@@ -121,3 +123,13 @@ def traverse(n, indptr, indices, window=0, cap=0, with_path=True):
     if with_path:
         res["P"] = Pbuf[:st[0]].copy()
     return res
+
+
+def l2_blocks(indptr, indices, B, sweeps=0):
+    """-> (label int32 [n], sweeps run); same definition as oracle/blocks.propagate."""
+    ip, ix = _graph(indptr, indices)
+    n = len(ip) - 1
+    label = np.empty(n, np.int32)
+    st = np.zeros(1, np.int64)
+    lib().ora_l2_blocks(n, ip.ctypes.data, ix.ctypes.data, int(B), int(sweeps), label.ctypes.data, st.ctypes.data)
+    return label, int(st[0])

@@ -22,12 +22,16 @@ static const size_t kAlign = 256;
 static size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
 // Device image of one part: 9 int32 arrays at 256-byte aligned offsets.
-size_t part_image_bytes(const mega_layout *L, int part, size_t offs[9]) {
+// Device image: the view arrays, plus two derived per-edge arrays the
+// edge-streaming kernels read (erow: CSR edge -> local row; csrc: CSC edge ->
+// source), 4 bytes per edge each.
+size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]) {
   const Part &P = L->parts[part];
-  const size_t sizes[9] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(), P.csr2csc.size(),
-                           P.fwd_items.size(), P.fwd_splits.size(), P.bwd_items.size(), P.bwd_splits.size()};
+  const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
+                                      P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
+                                      P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size()};
   size_t off = 0;
-  for (int i = 0; i < 9; ++i) {
+  for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
     off = align_up(off + sizes[i] * sizeof(int32_t));
   }
@@ -79,6 +83,8 @@ mega_status mega_preprocess(const mega_csr *csr, const mega_schedule_opts *opts,
   if (opts->candidate_cap < 0 || opts->candidate_cap > 64)
     return fail(MEGA_ERR_INVALID_ARGUMENT, "candidate_cap must be in [0, 64]");
   if (opts->window < 0 || opts->seg_edges < 0) return fail(MEGA_ERR_INVALID_ARGUMENT, "negative window/seg_edges");
+  if (opts->block_rows < 0 || opts->block_sweeps < 0 || opts->block_sweeps > 1000)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "block_rows must be >= 0 and block_sweeps in [0, 1000]");
   if (opts->order < 0 || opts->order > MEGA_ORDER_RANDOM) return fail(MEGA_ERR_INVALID_ARGUMENT, "unknown order");
   if (csr->indptr[0] != 0 || csr->indptr[n] != m) return fail(MEGA_ERR_INVALID_GRAPH, "indptr[0] != 0 or indptr[n] != m");
   for (int64_t i = 0; i < n; ++i)
@@ -146,7 +152,7 @@ mega_status mega_layout_device_bytes(const mega_layout *L, int32_t part, size_t 
   clear_error();
   if (!L || !bytes) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
   if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
-  size_t offs[9];
+  size_t offs[kImageArrays];
   *bytes = part_image_bytes(L, part, offs);
   return MEGA_OK;
 }
@@ -157,7 +163,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   if (!L || !dev_buf) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
   if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
   if (reinterpret_cast<uintptr_t>(dev_buf) % 256) return fail(MEGA_ERR_INVALID_ARGUMENT, "dev_buf must be 256-byte aligned");
-  size_t offs[9];
+  size_t offs[kImageArrays];
   const size_t need = part_image_bytes(L, part, offs);
   if (bytes < need) return fail(MEGA_ERR_OUT_OF_MEMORY, "device buffer smaller than mega_layout_device_bytes");
   Part &P = L->parts[part];
@@ -180,10 +186,16 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
       pcdst[q] = (int32_t)(((uint32_t)degree_class(P.indptr[r + 1] - P.indptr[r]) << 26) | (uint32_t)r);
     }
   }
-  const std::vector<int32_t> *arrs[9] = {&P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst,
-                                         &P.csr2csc, &P.fwd_items, &P.fwd_splits, &P.bwd_items, &P.bwd_splits};
+  std::vector<int32_t> erow(P.src.size()), csrc(P.cdst.size());
+  for (size_t r = 0; r + 1 < P.indptr.size(); ++r)
+    for (int32_t q = P.indptr[r]; q < P.indptr[r + 1]; ++q) erow[q] = (int32_t)r;
+  for (int64_t v = 0; v < L->n; ++v)
+    for (int32_t q = P.cindptr[v]; q < P.cindptr[v + 1]; ++q) csrc[q] = (int32_t)v;
+  const std::vector<int32_t> *arrs[kImageArrays] = {
+      &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
+      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc};
   char *base = static_cast<char *>(dev_buf);
-  for (int i = 0; i < 9; ++i) {
+  for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
     ce = cudaMemcpyAsync(base + offs[i], arrs[i]->data(), arrs[i]->size() * sizeof(int32_t), cudaMemcpyHostToDevice,
                          (cudaStream_t)stream);
@@ -201,6 +213,8 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.fwd_splits = reinterpret_cast<const int32_t *>(base + offs[6]);
   D.bwd_items = reinterpret_cast<const int4 *>(base + offs[7]);
   D.bwd_splits = reinterpret_cast<const int32_t *>(base + offs[8]);
+  D.erow = reinterpret_cast<const int32_t *>(base + offs[9]);
+  D.csrc = reinterpret_cast<const int32_t *>(base + offs[10]);
   D.n = L->n;
   D.rows = P.row_end - P.row_begin;
   D.row_begin = P.row_begin;

@@ -30,241 +30,11 @@
 #include <unordered_map>
 
 #include "mega_internal.h"
+#include "kern_common.cuh"
 
 namespace mega {
 namespace kern {
 
-constexpr int MAXH = 8;
-constexpr int WPB = 8;
-constexpr int TPB = WPB * 32;
-constexpr int MAX_GRID = 4096;  // upper bound for per-block partial buffers
-
-template <typename T> struct Tr;
-template <> struct Tr<float> { static constexpr int EPV = 4; };
-template <> struct Tr<__nv_bfloat16> { static constexpr int EPV = 8; };
-
-// ---------------------------------------------------------------- loads
-__device__ __forceinline__ uint64_t policy_last() {
-  uint64_t p;
-  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ uint64_t policy_first() {
-  uint64_t p;
-  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
-  return p;
-}
-__device__ __forceinline__ uint4 ldg16(const void *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
-__device__ __forceinline__ uint4 ldg16_pol(const void *p, uint64_t pol) {
-  uint4 r;
-  asm("ld.global.nc.L2::cache_hint.v4.u32 {%0, %1, %2, %3}, [%4], %5;"
-      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
-      : "l"(p), "l"(pol));
-  return r;
-}
-// streamed index arrays: no L1 allocation, L2 evict_first
-__device__ __forceinline__ int ld_stream(const int32_t *p, uint64_t pol) {
-  int v;
-  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ void st16(void *p, uint4 v) { *reinterpret_cast<uint4 *>(p) = v; }
-
-__device__ __forceinline__ void unpack(const uint4 &r, float (&x)[4], float) {
-  x[0] = __uint_as_float(r.x); x[1] = __uint_as_float(r.y);
-  x[2] = __uint_as_float(r.z); x[3] = __uint_as_float(r.w);
-}
-__device__ __forceinline__ void unpack(const uint4 &r, float (&x)[8], __nv_bfloat16) {
-  x[0] = __uint_as_float(r.x << 16); x[1] = __uint_as_float(r.x & 0xffff0000u);
-  x[2] = __uint_as_float(r.y << 16); x[3] = __uint_as_float(r.y & 0xffff0000u);
-  x[4] = __uint_as_float(r.z << 16); x[5] = __uint_as_float(r.z & 0xffff0000u);
-  x[6] = __uint_as_float(r.w << 16); x[7] = __uint_as_float(r.w & 0xffff0000u);
-}
-__device__ __forceinline__ uint32_t pk2(float a, float b) {
-  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
-  return *reinterpret_cast<uint32_t *>(&t);
-}
-__device__ __forceinline__ uint4 pack(const float (&x)[4], float) {
-  return make_uint4(__float_as_uint(x[0]), __float_as_uint(x[1]), __float_as_uint(x[2]), __float_as_uint(x[3]));
-}
-__device__ __forceinline__ uint4 pack(const float (&x)[8], __nv_bfloat16) {
-  return make_uint4(pk2(x[0], x[1]), pk2(x[2], x[3]), pk2(x[4], x[5]), pk2(x[6], x[7]));
-}
-
-template <int G> __device__ __forceinline__ float gmax(float v, unsigned mask) {
-#pragma unroll
-  for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(mask, v, o, G));
-  return v;
-}
-template <int G> __device__ __forceinline__ float gsum(float v, unsigned mask) {
-#pragma unroll
-  for (int o = G / 2; o > 0; o >>= 1) v += __shfl_xor_sync(mask, v, o, G);
-  return v;
-}
-template <int HT> __device__ __forceinline__ float sel(const float (&a)[HT], int i) {
-  float r = a[0];
-#pragma unroll
-  for (int h = 1; h < HT; ++h)
-    if (i == h) r = a[h];
-  return r;
-}
-// H (<= HT) consecutive fp32 values; 16-byte vectors when H % 4 == 0
-template <int HT> __device__ __forceinline__ void load_h(const float *p, int H, float (&v)[HT]) {
-  if (HT >= 4 && (H & 3) == 0) {
-#pragma unroll
-    for (int q = 0; q < HT / 4; ++q)
-      if (4 * q < H) {
-        float4 t = __ldg(reinterpret_cast<const float4 *>(p) + q);
-        v[4 * q] = t.x; v[4 * q + 1] = t.y; v[4 * q + 2] = t.z; v[4 * q + 3] = t.w;
-      }
-  } else {
-#pragma unroll
-    for (int h = 0; h < HT; ++h)
-      if (h < H) v[h] = __ldg(p + h);
-  }
-}
-// volatile loads: issued exactly where written (software-pipelined prefetches)
-__device__ __forceinline__ int ldv_i32(const int32_t *p, uint64_t pol) {
-  int v;
-  asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
-  return v;
-}
-__device__ __forceinline__ int4 ldv_i4(const int4 *p) {
-  int4 r;
-  asm volatile("ld.global.nc.v4.s32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
-  return r;
-}
-__device__ __forceinline__ uint4 ldv16(const void *p) {
-  uint4 r;
-  asm volatile("ld.global.nc.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w) : "l"(p));
-  return r;
-}
-template <int HT> __device__ __forceinline__ void load_h_v(const float *p, int H, float (&v)[HT]) {
-  if (HT >= 4 && (H & 3) == 0) {
-#pragma unroll
-    for (int q = 0; q < HT / 4; ++q)
-      if (4 * q < H)
-        asm volatile("ld.global.nc.v4.f32 {%0, %1, %2, %3}, [%4];"
-                     : "=f"(v[4 * q]), "=f"(v[4 * q + 1]), "=f"(v[4 * q + 2]), "=f"(v[4 * q + 3])
-                     : "l"(p + 4 * q));
-  } else {
-#pragma unroll
-    for (int h = 0; h < HT; ++h)
-      if (h < H) asm volatile("ld.global.nc.f32 %0, [%1];" : "=f"(v[h]) : "l"(p + h));
-  }
-}
-// Packed fp32x2 FMA (sm_100 FFMA2): d{0,1} += a{0,1} * b, and the two-lane dot
-// s{0,1} += a{0,1} * c{0,1}; halves the FMA issue count of the row loops.
-__device__ __forceinline__ void ffma2s(float &d0, float &d1, float a0, float a1, float b) {
-  unsigned long long D, A, B;
-  asm("mov.b64 %0, {%1, %2};" : "=l"(A) : "f"(a0), "f"(a1));
-  asm("mov.b64 %0, {%1, %2};" : "=l"(D) : "f"(d0), "f"(d1));
-  asm("mov.b64 %0, {%1, %1};" : "=l"(B) : "f"(b));
-  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(D) : "l"(A), "l"(B));
-  asm("mov.b64 {%0, %1}, %2;" : "=f"(d0), "=f"(d1) : "l"(D));
-}
-__device__ __forceinline__ void ffma2v(float &d0, float &d1, float a0, float a1, float c0, float c1) {
-  unsigned long long D, A, C;
-  asm("mov.b64 %0, {%1, %2};" : "=l"(A) : "f"(a0), "f"(a1));
-  asm("mov.b64 %0, {%1, %2};" : "=l"(C) : "f"(c0), "f"(c1));
-  asm("mov.b64 %0, {%1, %2};" : "=l"(D) : "f"(d0), "f"(d1));
-  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(D) : "l"(A), "l"(C));
-  asm("mov.b64 {%0, %1}, %2;" : "=f"(d0), "=f"(d1) : "l"(D));
-}
-// exp / log on the SFU: ex2.approx / lg2.approx (max rel. error ~2^-22; the
-// x*log2(e) rounding adds ~1e-7 |x| relative, within the fp32 parity bar)
-__device__ __forceinline__ float fexp(float x) {
-  float y;
-  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x * 1.4426950408889634f));
-  return y;
-}
-__device__ __forceinline__ float flog(float x) {
-  float y;
-  asm("lg2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
-  return y * 0.6931471805599453f;
-}
-__device__ __forceinline__ float leaky(float z, float slope) { return z > 0.f ? z : slope * z; }
-
-// Sum per-vector partial dot products over the lanes (and vectors) of a head.
-// LPH = lanes per head within one vector (head_dim / EPV), a compile-time
-// power of two (heads is a power of two for every supported row width).
-template <int G, int U, int V, int LPH>
-__device__ __forceinline__ void head_reduce(float (&p)[U][V], unsigned mask) {
-  if constexpr (LPH <= G) {
-#pragma unroll
-    for (int o = LPH >> 1; o > 0; o >>= 1) {
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-#pragma unroll
-        for (int v = 0; v < V; ++v) p[u][v] += __shfl_xor_sync(mask, p[u][v], o, G);
-    }
-  } else {
-    constexpr int VPH = LPH / G;
-#pragma unroll
-    for (int u = 0; u < U; ++u) {
-      float q[V];
-#pragma unroll
-      for (int v = 0; v < V; ++v) {
-        float t = 0.f;
-#pragma unroll
-        for (int v2 = 0; v2 < V; ++v2)
-          if (v2 / VPH == v / VPH) t += p[u][v2];
-        q[v] = t;
-      }
-#pragma unroll
-      for (int v = 0; v < V; ++v) p[u][v] = gsum<G>(q[v], mask);
-    }
-  }
-}
-// Does this lane write the (reduced) value of vector v's head?
-template <int G, int LPH>
-__device__ __forceinline__ bool head_lead(int gl, int v) {
-  if constexpr (LPH <= G) return (gl & (LPH - 1)) == 0;
-  else return gl == 0 && (v % (LPH / G)) == 0;
-}
-
-// Reduce per-lane [V][EPV] accumulators over all groups of the block and store
-// the block's [D] partial (fixed order -> deterministic; the cross-warp sum is
-// carried in fp64 because these are long reductions with cancellation).
-template <int G, int V, int EPV>
-__device__ void block_partial(float (&acc)[V][EPV], double *s_red, double *dst, int D) {
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G;
-#pragma unroll
-  for (int o = G; o < 32; o <<= 1)
-#pragma unroll
-    for (int v = 0; v < V; ++v)
-#pragma unroll
-      for (int k = 0; k < EPV; ++k) acc[v][k] += __shfl_xor_sync(0xffffffffu, acc[v][k], o);
-  __syncthreads();
-  for (int ww = 0; ww < WPB; ++ww) {
-    if (w == ww && lane < G) {
-#pragma unroll
-      for (int v = 0; v < V; ++v)
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) {
-          const int col = (v * G + gl) * EPV + k;
-          s_red[col] = (ww == 0 ? 0.0 : s_red[col]) + (double)acc[v][k];
-        }
-    }
-    __syncthreads();
-  }
-  for (int d = threadIdx.x; d < D; d += TPB) dst[d] = s_red[d];
-  __syncthreads();
-}
-
-struct FwdArgs {
-  DevPart L;
-  const void *feat;
-  int64_t ldf;
-  const float *el, *er;
-  float *lse;
-  int H, F, D;
-  float slope;
-  void *out;
-  int64_t ldo;
-  float *ws_m, *ws_l, *ws_acc;
-  int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
-};
 
 // ---- a3+a4+a5: fused score / online edge softmax / aggregation ----
 // Per chunk of G edges: lane l scores edge base+l for all heads (online
@@ -658,31 +428,6 @@ __global__ void __launch_bounds__(TPB) eler_kernel(const T *feat, int64_t ldf, i
   }
 }
 
-struct BwdArgs {
-  DevPart L;
-  const void *feat;
-  int64_t ldf;
-  const float *al, *ar;
-  int H, F, D;
-  float slope;
-  const void *out;
-  int64_t ldo;
-  const void *gout;
-  int64_t ldg;
-  const float *el, *er, *lse;
-  float *dlt, *der;
-  float *gfeat;
-  int64_t ldgf;
-  void *gfeat_lp;
-  int64_t ldlp;
-  float *dz, *ws_bacc, *ws_bder;
-  double *ws_dal, *ws_dar;
-  float *gal, *gar;
-  int nb_dst;
-  int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
-  int lp_partial;  // ... and (both phases in one call) the source-phase partial lives in gfeat_lp too
-  int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
-};
 
 // ---- a6: Dlt_i = g_i . out_i ----
 template <typename T, int G, int V, int HT>
@@ -1202,6 +947,15 @@ int fwd_variant() {
   }
   return v;
 }
+// edge-streaming TMA forward for wide rows (gat_stream.cu); MEGA_FWD_STREAM=0 selects the fused kernel
+bool use_stream_fwd() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_FWD_STREAM");
+    v = (e && e[0] == '0') ? 0 : 1;
+  }
+  return v == 1;
+}
 int bwd_variant() {
   static int v = -1;
   if (v < 0) {
@@ -1266,14 +1020,15 @@ mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
   return MEGA_OK;
 }
 
-struct WsFwd { size_t m, l, acc, total; };
+struct WsFwd { size_t m, l, acc, part, total; };
 WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   WsFwd w;
   size_t slots = (size_t)std::max(1, D.n_fwd_slots);
   w.m = 0;
   w.l = align256(w.m + slots * s.H * 4);
   w.acc = align256(w.l + slots * s.H * 4);
-  w.total = align256(w.acc + slots * s.D * 4);
+  w.part = align256(w.acc + slots * s.D * 4);
+  w.total = align256(w.part + (s.G == 32 ? (size_t)2 * kStreamMaxWarps * s.D * 4 : 0));
   return w;
 }
 struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
@@ -1335,6 +1090,12 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
   mega_status rc = MEGA_OK;
   dispatch_gv(s.nv, [&](auto g, auto v) {
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
+    if constexpr (G == 32) {
+      if (use_stream_fwd() && !use_ring()) {
+        rc = run_fwd_stream(a, s.nv, s.H, std::is_same<T, __nv_bfloat16>::value, st, dev_info(dev).sms);
+        return;
+      }
+    }
     if (a.L.n_fwd_items > 0) {
       dispatch_h(s.H, [&](auto ht) {
         constexpr int HT = decltype(ht)::value;
@@ -1476,6 +1237,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
+  a.ws_part = reinterpret_cast<float *>(wb + w.part);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }

@@ -25,6 +25,8 @@ struct DevPart {
   const int32_t *fwd_splits = nullptr;
   const int4 *bwd_items = nullptr;
   const int32_t *bwd_splits = nullptr;
+  const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
+  const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
   int64_t n = 0, rows = 0, row_begin = 0, edges = 0;
   // src (CSR) and cdst (CSC) entries carry a degree class in bits [31:26] when
   // n < 2^26: class = floor(2 log2(deg)) of the row they name (out-degree of the
@@ -63,7 +65,8 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-size_t part_image_bytes(const mega_layout *L, int part, size_t offs[9]);
+constexpr int kImageArrays = 11;
+size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]);
 // degree class: floor(2 log2 d) for d >= 1, clamped to 63; 0 for d = 0
 inline int degree_class(int64_t d) {
   if (d <= 0) return 0;

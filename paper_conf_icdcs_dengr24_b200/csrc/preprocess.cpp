@@ -172,6 +172,43 @@ struct Traversal {
   }
 };
 
+// L2 blocking (R24; ours, not the paper's).  Size-constrained label
+// propagation on G_u: nodes visited in ascending (deg_u, id); a node takes the
+// label most frequent among its neighbours, preferring its own label on a tie,
+// then the smallest label; a foreign label is eligible only while its block
+// holds fewer than B nodes.  Sweeps stop at `max_sweeps` or once a sweep
+// changes fewer than n/1000 labels.  Returns the label of every node.
+std::vector<int32_t> l2_blocks(int64_t n, const Adj &A, int32_t B, int max_sweeps, int64_t &sweeps) {
+  std::vector<int32_t> label(n), size(n, 1), visit(n), cnt(n, 0), seen;
+  seen.reserve(1024);
+  for (int64_t v = 0; v < n; ++v) label[v] = visit[v] = (int32_t)v;
+  auto dg = [&](int32_t v) { return A.end[v] - A.begin[v]; };
+  std::stable_sort(visit.begin(), visit.end(), [&](int32_t a, int32_t b) { return dg(a) < dg(b); });
+  sweeps = 0;
+  for (int it = 0; it < max_sweeps; ++it) {
+    ++sweeps;
+    int64_t changed = 0;
+    for (int32_t v : visit) {
+      if (dg(v) == 0) continue;
+      seen.clear();
+      for (int64_t k = A.begin[v]; k < A.end[v]; ++k) {
+        int32_t l = label[A.nbr[k]];
+        if (cnt[l]++ == 0) seen.push_back(l);
+      }
+      const int32_t cur = label[v];
+      int32_t best = cur, bc = cnt[cur];
+      for (int32_t l : seen) {
+        if (l == cur || size[l] >= B) continue;
+        if (cnt[l] > bc || (cnt[l] == bc && best != cur && l < best)) { best = l; bc = cnt[l]; }
+      }
+      for (int32_t l : seen) cnt[l] = 0;
+      if (best != cur) { label[v] = best; --size[cur]; ++size[best]; ++changed; }
+    }
+    if (changed * 1000 < n) break;
+  }
+  return label;
+}
+
 void items_for(const std::vector<int32_t> &ptr, int32_t S, std::vector<int32_t> &items,
                std::vector<int32_t> &splits, int32_t &nslots) {
   const int64_t rows = (int64_t)ptr.size() - 1;
@@ -221,12 +258,15 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
   }
 
   // ---- node order ----
-  int64_t path_len = n, jumps = 0;
+  int64_t path_len = n, jumps = 0, sweeps = 0, nblocks = n;
   L->perm.resize(n);
+  Adj A;
+  std::vector<int32_t> label;
+  if (opts->block_rows > 0 || opts->order == MEGA_ORDER_TRAVERSAL) build_adj(n, indptr, indices, A);
+  if (opts->block_rows > 0)  // before the traversal compacts the adjacency lists
+    label = l2_blocks(n, A, opts->block_rows, opts->block_sweeps > 0 ? opts->block_sweeps : 10, sweeps);
   switch (opts->order) {
     case MEGA_ORDER_TRAVERSAL: {
-      Adj A;
-      build_adj(n, indptr, indices, A);
       Traversal T(n, omega, K, A);
       T.run(path_len, jumps);
       L->perm = std::move(T.order);
@@ -254,6 +294,21 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
     default:
       return fail(MEGA_ERR_INVALID_ARGUMENT, "unknown order");
   }
+  if (opts->block_rows > 0) {  // stable regroup by block, blocks ranked by first position
+    std::vector<int32_t> rank(n, -1), start;
+    nblocks = 0;
+    for (int64_t r = 0; r < n; ++r) {
+      int32_t &k = rank[label[L->perm[r]]];
+      if (k < 0) { k = (int32_t)nblocks++; start.push_back(0); }
+      start[k]++;
+    }
+    int32_t acc = 0;
+    for (auto &c : start) { int32_t t = c; c = acc; acc += t; }
+    std::vector<int32_t> grouped(n);
+    for (int64_t r = 0; r < n; ++r) grouped[start[rank[label[L->perm[r]]]]++] = L->perm[r];
+    L->perm.swap(grouped);
+  }
+  { std::vector<int32_t>().swap(A.nbr); std::vector<int64_t>().swap(A.begin); }
   L->new_of_old.resize(n);
   for (int64_t r = 0; r < n; ++r) L->new_of_old[L->perm[r]] = (int32_t)r;
 
@@ -357,6 +412,9 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
     }
     st.tile_unique_sources = tot;
   }
+  st.block_rows = opts->block_rows;
+  st.num_blocks = opts->block_rows > 0 ? nblocks : 0;
+  st.block_sweeps = sweeps;
   st.preprocess_seconds = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
   return MEGA_OK;
 }

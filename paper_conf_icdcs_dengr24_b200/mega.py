@@ -42,14 +42,15 @@ class mega_csr(_c.Structure):
 class mega_schedule_opts(_c.Structure):
     _fields_ = [("struct_size", _c.c_uint32), ("window", _c.c_int32), ("candidate_cap", _c.c_int32),
                 ("order", _c.c_int32), ("seg_edges", _c.c_int32), ("num_parts", _c.c_int32),
-                ("seed", _c.c_uint64)]
+                ("seed", _c.c_uint64), ("block_rows", _c.c_int32), ("block_sweeps", _c.c_int32)]
 
 
 class mega_layout_stats(_c.Structure):
     _fields_ = [("struct_size", _c.c_uint32)] + [(k, _c.c_int64) for k in (
         "num_nodes", "num_edges", "num_parts", "window", "candidate_cap", "seg_edges", "order", "path_length",
         "revisits", "jumps", "tile_unique_sources", "max_in_degree", "max_out_degree")] + [
-        ("preprocess_seconds", _c.c_double)]
+        ("preprocess_seconds", _c.c_double)] + [(k, _c.c_int64) for k in ("block_rows", "num_blocks",
+                                                                          "block_sweeps")]
 
 
 _VIEW_INTS = ("num_nodes", "num_edges", "row_begin", "row_end", "part_edges", "num_fwd_items", "num_fwd_splits",
@@ -144,17 +145,23 @@ class Layout:
 
 
 def mega_preprocess(indptr, indices, window=0, candidate_cap=0, order="traversal", seg_edges=0, num_parts=1,
-                    seed=0) -> Layout:
+                    seed=0, block_rows=0, block_sweeps=0) -> Layout:
     indptr = np.ascontiguousarray(indptr, dtype=np.int64)
     indices = np.ascontiguousarray(indices, dtype=np.int32)
     csr = mega_csr(len(indptr) - 1, len(indices), indptr.ctypes.data, indices.ctypes.data)
     o = mega_schedule_opts()
     lib().mega_schedule_opts_init(_c.byref(o))
     o.window, o.candidate_cap, o.seg_edges, o.num_parts, o.seed = window, candidate_cap, seg_edges, num_parts, seed
+    o.block_rows, o.block_sweeps = block_rows, block_sweeps
     o.order = ORDERS[order] if isinstance(order, str) else int(order)
     h = _c.c_void_p()
     _check(lib().mega_preprocess(_c.byref(csr), _c.byref(o), _c.byref(h)))
     return Layout(h.value)
+
+
+def auto_block_rows(row_bytes: int, l2_bytes: int = 126 * 1024 * 1024) -> int:
+    """B for L2 blocking: 0.4 of the L2 in gathered rows (R24)."""
+    return max(1, int(0.4 * l2_bytes) // max(1, int(row_bytes)))
 
 
 def mega_layout_stats_get(layout: Layout) -> dict:

@@ -55,6 +55,10 @@ def main():
         for order in ("traversal", "identity"):
             lay = M.mega_preprocess(ip, ix, order=order)
             pats[f"csr_src_{order}"] = lay.view(0)["src"]
+        lay = M.mega_preprocess(ip, ix, block_rows=M.auto_block_rows(rb))
+        pats["csr_src_traversal_l2blocked"] = lay.view(0)["src"]
+        # L2-resident table: random rows of the first 24 MB (the L2 gather ceiling)
+        pats["random_l2_resident"] = rng.integers(0, (24 << 20) // rb, n, dtype=np.int32)
         pats["sequential"] = (np.arange(n, dtype=np.int64) % cfg.n).astype(np.int32)
         for k, v in pats.items():
             idx = torch.tensor(v, device="cuda")

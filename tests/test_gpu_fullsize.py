@@ -50,7 +50,8 @@ def test_fullsize_sampled(cuda_device, name):
     x, w = synth.bf16_round(inp["x"]), synth.bf16_round(inp["w"])
     g = synth.bf16_round(inp["grad_out"])
     H, F, D, n = cfg.heads, cfg.head_dim, cfg.dim, cfg.n
-    lay = M.mega_preprocess(ip, ix)
+    import bench
+    lay = M.mega_preprocess(ip, ix, block_rows=bench.block_rows_for(cfg, "bf16"))  # bench's layout options
     lay.bind(0)
     perm = lay.view(0)["perm"].astype(np.int64)
     L = hz.layer(lay, x[perm], w, inp["a_l"], inp["a_r"], H, F, "bf16", want_grad_x=False)

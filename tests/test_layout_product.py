@@ -10,6 +10,7 @@ import pytest
 
 import synth
 from oracle import coracle
+from oracle import blocks as ob
 from oracle import layout as ol
 from oracle import traverse as ot
 from paper_conf_icdcs_dengr24_b200 import mega as M
@@ -39,7 +40,7 @@ def test_invalid_inputs_are_rejected():
     assert e.value.status == 1
 
 
-def _oracle_layout(ip, ix, order, window, cap, parts, seg, seed=0):
+def _oracle_layout(ip, ix, order, window, cap, parts, seg, seed=0, block_rows=0):
     n = len(ip) - 1
     if order == "traversal":
         r = ot.traverse(n, ip, ix, window=window, cap=cap) if n <= 3000 else coracle.traverse(n, ip, ix, window, cap)
@@ -50,6 +51,12 @@ def _oracle_layout(ip, ix, order, window, cap, parts, seg, seed=0):
         perm, r = ot.order_degree(n, ip), None
     else:
         perm, r = ot.order_random(n, seed), None
+    if block_rows > 0:
+        if n <= 3000:
+            perm = ob.blocked_order(n, ip, ix, perm, block_rows)["perm"]
+        else:
+            label, _ = coracle.l2_blocks(ip, ix, block_rows)
+            perm, _ = ob.regroup([int(v) for v in perm], label.tolist())
     return ol.build(ip, ix, perm, num_parts=parts, seg_edges=seg), r
 
 
@@ -103,6 +110,53 @@ def test_bit_exact_vs_oracle_arxiv():
     lay = M.mega_preprocess(ip, ix, num_parts=4, seg_edges=64)
     ref, r = _oracle_layout(ip, ix, "traversal", 0, 0, 4, 64)
     _compare(lay, ref, r)
+
+
+@pytest.mark.parametrize("seed", range(6))
+@pytest.mark.parametrize("order", ["traversal", "degree", "random"])
+def test_bit_exact_blocked_vs_oracle_tiny(seed, order):
+    rng = np.random.default_rng(100 + seed)
+    n = int(rng.integers(3, 200))
+    ip, ix = synth.random_multigraph(100 + seed, n, int(rng.integers(1, 8 * n)), undirected=bool(seed % 2),
+                                     isolated=seed % 3)
+    B = [1, 2, 5, 17, 64, 1000][seed]
+    lay = M.mega_preprocess(ip, ix, order=order, num_parts=1 + seed % 3, seg_edges=1 + seed, block_rows=B,
+                            seed=7 + seed)
+    ref, r = _oracle_layout(ip, ix, order, 0, 0, 1 + seed % 3, 1 + seed, seed=7 + seed, block_rows=B)
+    _compare(lay, ref, r if order == "traversal" else None)
+    st = lay.stats()
+    label, sweeps = coracle.l2_blocks(ip, ix, B)
+    assert st["block_sweeps"] == sweeps and st["num_blocks"] == len(set(label.tolist()))
+
+
+@pytest.mark.parametrize("name", ["cora", "pubmed"])
+def test_bit_exact_blocked_vs_oracle_configs(name):
+    cfg = synth.CONFIGS[name]
+    ip, ix, _ = synth.make_graph(cfg)
+    B = M.auto_block_rows(cfg.dim * 2, 2 * 1024 * 1024)  # a small L2 so that the configs split into blocks
+    lay = M.mega_preprocess(ip, ix, num_parts=2, block_rows=B)
+    ref, r = _oracle_layout(ip, ix, "traversal", 0, 0, 2, 0, block_rows=B)
+    _compare(lay, ref, r)
+    assert lay.stats()["num_blocks"] > 1
+
+
+def test_l2_blocking_improves_block_scale_reuse():
+    """On a products-shaped graph the blocked order should need far fewer
+    distinct sources per L2-sized run of destinations than the plain traversal."""
+    cfg = synth.scaled(synth.CONFIGS["products"], 40000, 600000)
+    ip, ix, _ = synth.make_graph(cfg)
+    B = 4000
+
+    def distinct_per_run(lay):
+        v = lay.view(0)
+        tot = 0
+        for r0 in range(0, cfg.n, B):
+            a, b = int(v["indptr"][r0]), int(v["indptr"][min(cfg.n, r0 + B)])
+            tot += np.unique(v["src"][a:b]).size
+        return tot
+    plain = distinct_per_run(M.mega_preprocess(ip, ix))
+    blocked = distinct_per_run(M.mega_preprocess(ip, ix, block_rows=B))
+    assert blocked < 0.7 * plain, (blocked, plain)
 
 
 def test_save_load_roundtrip(tmp_path):
