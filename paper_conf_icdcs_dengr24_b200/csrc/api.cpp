@@ -25,11 +25,40 @@ static size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 // Device image: the view arrays, plus two derived per-edge arrays the
 // edge-streaming kernels read (erow: CSR edge -> local row; csrc: CSC edge ->
 // source), 4 bytes per edge each.
+std::vector<int32_t> make_tiles(const std::vector<int32_t> &items) {
+  std::vector<int32_t> t;
+  int32_t b = 0, e = 0;
+  bool open = false;
+  auto close = [&] {
+    if (open) t.insert(t.end(), {b, e, -1, 0});
+    open = false;
+  };
+  for (size_t k = 0; k + 3 < items.size(); k += 4) {
+    const int32_t e0 = items[k + 1], e1 = items[k + 2], slot = items[k + 3];
+    if (e1 == e0) continue;
+    if (slot >= 0) {
+      t.insert(t.end(), {e0, e1, slot, 0});
+      continue;
+    }
+    if (open && e == e0 && (e1 - b) <= kTileEdges) {
+      e = e1;
+    } else {
+      close();
+      b = e0;
+      e = e1;
+      open = true;
+    }
+  }
+  close();
+  return t;
+}
+
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]) {
   const Part &P = L->parts[part];
   const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
-                                      P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size()};
+                                      P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
+                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size()};
   size_t off = 0;
   for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
@@ -191,9 +220,10 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
     for (int32_t q = P.indptr[r]; q < P.indptr[r + 1]; ++q) erow[q] = (int32_t)r;
   for (int64_t v = 0; v < L->n; ++v)
     for (int32_t q = P.cindptr[v]; q < P.cindptr[v + 1]; ++q) csrc[q] = (int32_t)v;
+  const std::vector<int32_t> ftiles = make_tiles(P.fwd_items), btiles = make_tiles(P.bwd_items);
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
-      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc};
+      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
@@ -215,6 +245,10 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.bwd_splits = reinterpret_cast<const int32_t *>(base + offs[8]);
   D.erow = reinterpret_cast<const int32_t *>(base + offs[9]);
   D.csrc = reinterpret_cast<const int32_t *>(base + offs[10]);
+  D.ftiles = reinterpret_cast<const int4 *>(base + offs[11]);
+  D.btiles = reinterpret_cast<const int4 *>(base + offs[12]);
+  D.n_ftiles = (int32_t)(ftiles.size() / 4);
+  D.n_btiles = (int32_t)(btiles.size() / 4);
   D.n = L->n;
   D.rows = P.row_end - P.row_begin;
   D.row_begin = P.row_begin;

@@ -62,7 +62,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
   const int H = a.H, rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
   const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
   const float *sp_v[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
@@ -71,7 +71,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
   // element offsets fit in 32 bits (checked on the host: n * ldf < 2^32)
   auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
     const T *rp = featl + (jj & idm) * ldf;
-    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_cold;
+    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
     for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
@@ -202,16 +202,6 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
 // quads (4 rows each) with cp.async (LDGSTS, L2 cache-policy hints): every lane
 // copies and later reads back exactly its own 16-byte pieces, so the ring
 // needs no barriers; P quads stay in flight without holding registers.
-__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, uint64_t pol) {
-  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
-  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N> __device__ __forceinline__ void cp_async_wait() {
-  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
-}
-
 template <typename T, int V, int HT, int P>
 __global__ void __launch_bounds__(TPB, 2) gat_fwd_ring_kernel(const FwdArgs a) {
   constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, SP = HT + 1, RSLOT = 4 * P;
@@ -222,7 +212,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_fwd_ring_kernel(const FwdArgs a) {
   uint4 *ring = ring_all + (size_t)w * RSLOT * V * 32;
   const int H = a.H;
   const uint32_t idm = a.L.id_mask;
-  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / FF;
@@ -235,7 +225,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_fwd_ring_kernel(const FwdArgs a) {
       const int k = min(4 * q + r, cnt - 1);  // the tail re-reads the last row (weight p = 0)
       const uint32_t jj = (uint32_t)s_j[w][k];
       const T *rp = featl + (jj & idm) * ldf;
-      const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_cold;
+      const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_row;
       uint4 *dst = ring + ((q % P) * 4 + r) * V * 32 + lane;
 #pragma unroll
       for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
@@ -486,7 +476,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   const int H = a.H, rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
   const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = policy_last(), pol_cold = policy_first();
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
@@ -501,7 +491,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   auto row_load = [&](uint4 (&r)[V], uint32_t ii) {
     const T *rp = goutl + (ii & idm) * ldg;
-    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_cold;
+    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
     for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
@@ -939,6 +929,14 @@ bool use_ring() {
   }
   return v == 1;
 }
+int l2_policy_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_L2_POLICY");
+    v = e ? std::atoi(e) : 0;
+  }
+  return v;
+}
 int fwd_variant() {
   static int v = -1;
   if (v < 0) {
@@ -1020,15 +1018,15 @@ mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
   return MEGA_OK;
 }
 
-struct WsFwd { size_t m, l, acc, part, total; };
+struct WsFwd { size_t m, l, acc, alpha, total; };
 WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   WsFwd w;
   size_t slots = (size_t)std::max(1, D.n_fwd_slots);
   w.m = 0;
   w.l = align256(w.m + slots * s.H * 4);
   w.acc = align256(w.l + slots * s.H * 4);
-  w.part = align256(w.acc + slots * s.D * 4);
-  w.total = align256(w.part + (s.G == 32 ? (size_t)2 * kStreamMaxWarps * s.D * 4 : 0));
+  w.alpha = align256(w.acc + slots * s.D * 4);
+  w.total = align256(w.alpha + (s.G == 32 ? (size_t)std::max<int64_t>(1, D.edges) * s.H * 4 : 0));
   return w;
 }
 struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
@@ -1237,8 +1235,9 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.ws_part = reinterpret_cast<float *>(wb + w.part);
+  a.alpha = reinterpret_cast<float *>(wb + w.alpha);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
+  a.pol_mode = l2_policy_mode();
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1288,6 +1287,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.lp_partial = 0;  // bf16 partial measured no faster than the fp32 partial (latency-bound); kept off
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
+  a.pol_mode = l2_policy_mode();
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }

@@ -16,7 +16,7 @@ constexpr int MAXH = 8;
 constexpr int WPB = 8;
 constexpr int TPB = WPB * 32;
 constexpr int MAX_GRID = 4096;
-constexpr int kStreamMaxWarps = 4096;  // warps of the edge-streaming kernels (sizes their partial buffers)  // upper bound for per-block partial buffers
+
 
 template <typename T> struct Tr;
 template <> struct Tr<float> { static constexpr int EPV = 4; };
@@ -33,6 +33,15 @@ __device__ __forceinline__ uint64_t policy_first() {
   asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
+__device__ __forceinline__ uint64_t policy_normal() {
+  uint64_t p;
+  asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// L2 policy of gathered feature rows (MEGA_L2_POLICY): 0 = hot rows evict_last,
+// the rest evict_first; 1 = all evict_normal; 2 = hot evict_last, rest evict_normal.
+__device__ __forceinline__ uint64_t row_policy_hot(int mode) { return mode == 1 ? policy_normal() : policy_last(); }
+__device__ __forceinline__ uint64_t row_policy_cold(int mode) { return mode == 0 ? policy_first() : policy_normal(); }
 __device__ __forceinline__ uint4 ldg16(const void *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
 __device__ __forceinline__ uint4 ldg16_pol(const void *p, uint64_t pol) {
   uint4 r;
@@ -231,6 +240,17 @@ __device__ void block_partial(float (&acc)[V][EPV], double *s_red, double *dst, 
   __syncthreads();
 }
 
+// cp.async (LDGSTS) 16-byte copies with an L2 policy; commit / wait groups
+__device__ __forceinline__ void cp_async16(void *smem, const void *gmem, uint64_t pol) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+template <int N> __device__ __forceinline__ void cp_async_wait() {
+  asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
+}
+
 struct FwdArgs {
   DevPart L;
   const void *feat;
@@ -242,8 +262,9 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
-  float *ws_part;  // edge-streaming forward: [2 * kStreamMaxWarps][D] fp32 partials of rows cut by warp ranges
+  float *alpha;    // edge-streaming forward: [E_p][H] fp32 attention weights in CSR order
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
+  int pol_mode; // MEGA_L2_POLICY
 };
 
 struct BwdArgs {
@@ -270,6 +291,7 @@ struct BwdArgs {
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
   int lp_partial;  // ... and (both phases in one call) the source-phase partial lives in gfeat_lp too
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
+  int pol_mode; // MEGA_L2_POLICY
 };
 
 }  // namespace kern

@@ -27,6 +27,9 @@ struct DevPart {
   const int32_t *bwd_splits = nullptr;
   const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
   const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
+  const int4 *ftiles = nullptr;      // (e_begin, e_end, slot, 0): runs of whole CSR rows / one split segment
+  const int4 *btiles = nullptr;      // the same over the CSC (sources)
+  int32_t n_ftiles = 0, n_btiles = 0;
   int64_t n = 0, rows = 0, row_begin = 0, edges = 0;
   // src (CSR) and cdst (CSC) entries carry a degree class in bits [31:26] when
   // n < 2^26: class = floor(2 log2(deg)) of the row they name (out-degree of the
@@ -65,7 +68,12 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-constexpr int kImageArrays = 11;
+constexpr int kImageArrays = 13;
+// Edge tiles of the streaming kernels: consecutive unsplit work items are
+// merged while their edges stay contiguous and total <= kTileEdges; a split
+// segment (slot >= 0) is a tile of its own; rows without edges are skipped.
+constexpr int kTileEdges = 512;
+std::vector<int32_t> make_tiles(const std::vector<int32_t> &items);
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]);
 // degree class: floor(2 log2 d) for d >= 1, clamped to 63; 0 for d = 0
 inline int degree_class(int64_t d) {

@@ -1,8 +1,9 @@
 """From an ncu launch list with gpu__time_duration / dram bytes per launch, derive
 per-kernel shares and per-call DRAM traffic (bench.py's `traffic` field).
 
-usage: launch_traffic.py launches.csv steps_profiled layers out_prefix
-The last `steps_profiled` steps of launches are used (warm-up launches dropped)."""
+usage: launch_traffic.py launches.csv steps_run layers out_prefix
+The launch list holds `steps_run` identical steps (warm-up + timed); the last
+one is used."""
 import collections
 import csv
 import io
@@ -27,13 +28,7 @@ def short(n):
 
 
 L = list(launch.values())
-# our kernels only: find the last `steps` occurrences per step by counting gat_fwd launches
-fwd_idx = [i for i, d in enumerate(L) if "gat_fwd_kernel" in d["name"]]
-first = fwd_idx[-steps * layers] if len(fwd_idx) >= steps * layers else 0
-# the step starts with the projection that precedes the first timed gat_fwd
-while first > 0 and "gat_fwd_kernel" not in L[first - 1]["name"] and "eler" not in L[first - 1]["name"]:
-    first -= 1
-sel = L[max(0, first - 3):]
+sel = L[len(L) * (steps - 1) // steps:]
 tot = collections.defaultdict(lambda: [0, 0.0, 0.0])
 for d in sel:
     k = short(d["name"])
@@ -55,7 +50,7 @@ def per_launch(pred):
 
 
 traffic = {
-    "gat_fwd": per_launch(lambda k: k.startswith("gat_fwd")),
+    "gat_fwd": per_launch(lambda k: k.startswith(("gat_fwd", "fwd_stats"))),
     "gat_bwd": per_launch(lambda k: k.startswith(("dlt_kernel", "gat_bwd_src", "gat_bwd_dst", "param_reduce"))),
     "gat_bwd_src": per_launch(lambda k: k.startswith(("dlt_kernel", "gat_bwd_src"))),
     "gat_bwd_dst": per_launch(lambda k: k.startswith(("gat_bwd_dst", "param_reduce"))),
