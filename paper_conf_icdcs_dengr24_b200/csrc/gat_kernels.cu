@@ -945,12 +945,13 @@ int fwd_variant() {
   }
   return v;
 }
-// edge-streaming TMA forward for wide rows (gat_stream.cu); MEGA_FWD_STREAM=0 selects the fused kernel
+// edge-streaming TMA forward for wide rows (gat_stream.cu), opt-in with MEGA_FWD_STREAM=1: measured
+// 46.7 vs 29.2 ms/step for the fused kernel on products (3 layers)
 bool use_stream_fwd() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_FWD_STREAM");
-    v = (e && e[0] == '0') ? 0 : 1;
+    v = (e && e[0] == '1') ? 1 : 0;
   }
   return v == 1;
 }
