@@ -197,6 +197,224 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
   }
 }
 
+// ---- a3+a4+a5, chunk-pipelined (the default) ----
+// The same per-chunk arithmetic as gat_fwd_kernel, but the dependency chain
+// item descriptor -> source ids -> er / source rows is taken off the critical
+// path: while chunk c is scored and aggregated, the NEXT chunk of the group's
+// stream (the next G edges of this item, else the first G of its next item)
+// has its source ids, el and er staged in shared memory with cp.async, and its
+// source rows prefetched into L2 by the TMA engine (cp.async.bulk.prefetch),
+// so chunk c+1 starts with everything but the row bytes on chip and the row
+// loads hit L2.  Item descriptors are staged G at a time, double-buffered.
+template <typename T, int G, int V, int HT>
+__global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(const FwdArgs a) {
+  constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, GPW = 32 / G, SP = HT + 1;
+  constexpr int U = FwdCfg<V, 0>::U < G ? FwdCfg<V, 0>::U : G;  // U divides G
+  __shared__ float s_p[WPB][32][SP];
+  __shared__ int4 s_desc[2][WPB][32];
+  __shared__ int s_src[2][WPB][32];  // packed source ids (class bits + id) of a chunk
+  __shared__ __align__(16) float s_er[2][WPB][32][HT];
+  __shared__ __align__(16) float s_el[2][WPB][GPW][HT];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
+  const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
+  const int H = a.H, rb = grp * G;
+  const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
+  const int hot_cls = a.hot_cls;
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
+  const uint32_t row_bytes = (uint32_t)(a.D * sizeof(T));
+  const float *sp_v[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *featl = feat + gl * EPV;
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  const int64_t it0 = ((int64_t)blockIdx.x * WPB + w) * GPW + grp, n_items = a.L.n_fwd_items;
+  if (it0 >= n_items) return;
+  auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
+    const T *rp = featl + (jj & idm) * ldf;
+    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
+#pragma unroll
+    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
+  };
+  // descriptor batch k: items it0 + (kG + l) stride, l < G, into s_desc[k & 1]
+  auto stage_desc = [&](int k) {
+    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
+    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][rb + gl], a.L.fwd_items + itq);
+    cp_async_commit();
+  };
+  // chunk (itm, bse): source ids (tail lanes repeat the last edge) and, for the first chunk of an item, el
+  auto stage_src = [&](int b, int4 itm, int bse) {
+    if (itm.z > itm.y) cp_async_small<4>(&s_src[b][w][rb + gl], a.L.src + min(bse + gl, itm.z - 1));
+    else s_src[b][w][rb + gl] = 0;
+    if (bse == itm.y && gl == 0) cp_async_h<HT>(&s_el[b][w][grp][0], a.el + (a.L.row_begin + itm.x) * H);
+    cp_async_commit();
+  };
+  // er of the staged chunk's sources, and their rows into L2
+  auto stage_er = [&](int b, int4 itm, int bse) {
+    const uint32_t jj = (uint32_t)s_src[b][w][rb + gl];
+    cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
+    if (bse + gl < itm.z && gl < a.pf_rows)
+      prefetch_l2_bulk(feat + (jj & idm) * ldf, row_bytes, (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row);
+    cp_async_commit();
+  };
+  // prologue: descriptor batches 0 and 1, chunk 0 staged
+  stage_desc(0);
+  stage_desc(1);
+  cp_async_wait<1>();
+  __syncwarp(gmask);
+  int q = 0;
+  int4 item = s_desc[0][w][rb];
+  int base = item.y, buf = 0;
+  stage_src(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp(gmask);
+  stage_er(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp(gmask);
+  float elr[HT], mrun[HT], lrun[HT], acc[V][EPV];
+  while (true) {
+    // ---- the next chunk of this group's stream; stage its ids (and el) ----
+    int4 nitem = item;
+    int nbase = base + G;
+    int nq = q;
+    bool has_next = true;
+    if (nbase >= item.z) {
+      nq = q + 1;
+      if (it0 + (int64_t)nq * stride >= n_items) {
+        has_next = false;
+      } else {
+        if (nq % G == 0) {  // entering descriptor batch nq/G: make sure it landed, refill the other buffer
+          cp_async_wait<0>();
+          __syncwarp(gmask);
+          nitem = s_desc[(nq / G) & 1][w][rb];
+          __syncwarp(gmask);
+          stage_desc(nq / G + 1);
+        } else {
+          nitem = s_desc[(nq / G) & 1][w][rb + (int)(nq % G)];
+        }
+        nbase = nitem.y;
+      }
+    }
+    const int nb_ = buf ^ 1;
+    if (has_next) stage_src(nb_, nitem, nbase);
+    // ---- the current chunk ----
+    if (base == item.y) {
+#pragma unroll
+      for (int h = 0; h < HT; ++h) { elr[h] = s_el[buf][w][grp][h]; mrun[h] = -INFINITY; lrun[h] = 0.f; }
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+    }
+    const int *sj = &s_src[buf][w][rb];
+    const bool valid = base + gl < item.z;
+    const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
+    uint4 ra[U][V], rz[U][V];
+    if (cnt > 0) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)sj[min(u, cnt - 1)]);
+      if (nbt > 1) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)sj[min(U + u, cnt - 1)]);
+      }
+    }
+    float sc[HT];
+#pragma unroll
+    for (int h = 0; h < HT; ++h) {
+      sc[h] = 1.f;
+      if (h < H) {
+        const float s = valid ? leaky(elr[h] + s_er[buf][w][rb + gl][h], a.slope) : -INFINITY;
+        const float mn = fmaxf(mrun[h], gmax<G>(s, gmask));
+        sc[h] = mn == -INFINITY ? 1.f : fexp(mrun[h] - mn);
+        const float p = valid ? fexp(s - mn) : 0.f;
+        lrun[h] = fmaf(lrun[h], sc[h], p);
+        mrun[h] = mn;
+        s_p[w][lane][h] = p;
+      }
+    }
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const float f = sel<HT>(sc, ((v * G + gl) * EPV) / FF);
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
+    }
+    // next chunk's ids have had the score phase to land: stage its er, prefetch its rows
+    cp_async_wait<0>();
+    __syncwarp(gmask);
+    if (has_next) stage_er(nb_, nitem, nbase);
+    auto consume = [&](const uint4 (&raw)[U][V], int k0) {
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float pw = sp_v[v][(k0 + u) * SP];
+          float x[EPV];
+          unpack(raw[u][v], x, T());
+#pragma unroll
+          for (int k = 0; k < EPV; k += 2) ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], pw);
+        }
+    };
+    for (int b = 0; b < nbt; b += 2) {
+      consume(ra, b * U);
+      if (b + 2 < nbt) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)sj[min((b + 2) * U + u, cnt - 1)]);
+      }
+      if (b + 1 < nbt) {
+        consume(rz, (b + 1) * U);
+        if (b + 3 < nbt) {
+#pragma unroll
+          for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)sj[min((b + 3) * U + u, cnt - 1)]);
+        }
+      }
+    }
+    // ---- end of the item: finalise ----
+    if (base + G >= item.z) {
+      const int64_t grow = a.L.row_begin + item.x;
+      float lt[HT];
+#pragma unroll
+      for (int h = 0; h < HT; ++h) lt[h] = h < H ? gsum<G>(lrun[h], gmask) : 0.f;
+      if (item.w < 0) {
+        T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float Lh = sel<HT>(lt, ((v * G + gl) * EPV) / FF);
+          const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
+          float y[EPV];
+#pragma unroll
+          for (int k = 0; k < EPV; ++k) y[k] = acc[v][k] * inv;
+          st16(orow + v * G * EPV, pack(y, T()));
+        }
+        for (int h = gl; h < H; h += G) {
+          const float Lh = sel<HT>(lt, h);
+          a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + flog(Lh) : -INFINITY;
+        }
+      } else {
+        const int64_t slot = item.w;
+        for (int h = gl; h < H; h += G) {
+          a.ws_m[slot * H + h] = sel<HT>(mrun, h);
+          a.ws_l[slot * H + h] = sel<HT>(lt, h);
+        }
+        float *pr = a.ws_acc + slot * a.D + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+#pragma unroll
+          for (int k = 0; k < EPV; k += 4)
+            *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+                make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+      }
+    }
+    if (!has_next) break;
+    cp_async_wait<0>();
+    __syncwarp(gmask);
+    item = nitem;
+    base = nbase;
+    q = nq;
+    buf = nb_;
+  }
+  cp_async_wait<0>();
+}
+
 // ---- a3+a4+a5 for wide rows (G = 32 lanes per row): cp.async ring pipeline ----
 // Each warp streams its source rows through a private shared-memory ring of P
 // quads (4 rows each) with cp.async (LDGSTS, L2 cache-policy hints): every lane
@@ -682,6 +900,298 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   }
 }
 
+// ---- a7, chunk-pipelined (G = 32, H <= 4) ----
+// gat_bwd_src_kernel's arithmetic with the fwd pipe kernel's staging: while
+// chunk c runs, the next chunk's destination ids, their (el, lse, Dlt) and
+// (for a new source) er_j are staged in shared memory with cp.async, and the
+// next chunk's g rows and the next source's Wh row are prefetched into L2.
+template <typename T, int V, int HT>
+__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_pipe_kernel(const BwdArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
+  constexpr int U1 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U1 < G ? U1 : G;
+  constexpr int NB = U * V;
+  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
+  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
+  __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
+  __shared__ float s_z[WPB][32][SP];  // dz out
+  __shared__ int4 s_desc[2][WPB][32];
+  __shared__ int s_i[2][WPB][32];     // packed destination rows of a chunk
+  __shared__ __align__(16) float s_el[2][WPB][32][HT];
+  __shared__ __align__(16) float s_ls[2][WPB][32][HT];
+  __shared__ __align__(16) float s_dl[2][WPB][32][HT];
+  __shared__ __align__(16) float s_er[2][WPB][HT];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
+  const unsigned gmask = 0xffffffffu;
+  const int H = a.H;
+  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
+  const int hot_cls = a.hot_cls;
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
+  const uint32_t grow_bytes = (uint32_t)(a.D * sizeof(T));
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
+  int bidx = 0;
+#pragma unroll
+  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
+  const int bu = bidx / V, bv = bidx % V;
+  const int bhead = ((bv * G + gl) * EPV) / FF;
+  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *gout = static_cast<const T *>(a.gout);
+  const T *goutl = gout + gl * EPV;
+  const int64_t stride = (int64_t)gridDim.x * WPB;
+  const int64_t it0 = (int64_t)blockIdx.x * WPB + w, n_items = a.L.n_bwd_items;
+  if (it0 >= n_items) return;
+  auto row_load = [&](uint4 (&r)[V], uint32_t ii) {
+    const T *rp = goutl + (ii & idm) * ldg;
+    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
+#pragma unroll
+    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
+  };
+  auto stage_desc = [&](int k) {
+    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
+    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][gl], a.L.bwd_items + itq);
+    cp_async_commit();
+  };
+  // chunk (itm, bse): destination ids; for the first chunk of a source its er, and its Wh row into L2
+  auto stage_ids = [&](int b, int4 itm, int bse) {
+    if (itm.z > itm.y) cp_async_small<4>(&s_i[b][w][gl], a.L.cdst + min(bse + gl, itm.z - 1));
+    else s_i[b][w][gl] = 0;
+    if (bse == itm.y && gl == 0) {
+      cp_async_h<HT>(&s_er[b][w][0], a.er + (int64_t)itm.x * H);
+      prefetch_l2_bulk(feat + (int64_t)itm.x * a.ldf, grow_bytes, pol_row);
+    }
+    cp_async_commit();
+  };
+  // the staged chunk's destination values, and its g rows into L2
+  auto stage_dst = [&](int b, int4 itm, int bse) {
+    const uint32_t ii = (uint32_t)s_i[b][w][gl];
+    const int64_t gi = a.L.row_begin + (int)(ii & idm);
+    cp_async_h<HT>(&s_el[b][w][gl][0], a.el + gi * H);
+    cp_async_h<HT>(&s_ls[b][w][gl][0], a.lse + gi * H);
+    cp_async_h<HT>(&s_dl[b][w][gl][0], a.dlt + gi * H);
+    cp_async_commit();
+    // the chunk's first pf_rows g rows into L2, one 128-byte line per lane per step
+    constexpr int LPR = (32 * V * 16) / 128, RPS = 32 / LPR;
+    const int cnt_n = min(a.pf_rows, itm.z - bse);
+    for (int r0 = 0; r0 < cnt_n; r0 += RPS) {
+      const int r = r0 + gl / LPR;
+      if (r < cnt_n)
+        prefetch_l2_line(reinterpret_cast<const char *>(gout + ((uint32_t)s_i[b][w][r] & idm) * ldg) + (gl % LPR) * 128);
+    }
+  };
+  stage_desc(0);
+  stage_desc(1);
+  cp_async_wait<1>();
+  __syncwarp();
+  int q = 0;
+  int4 item = s_desc[0][w][0];
+  int base = item.y, buf = 0;
+  stage_ids(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp();
+  stage_dst(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp();
+  float whf[V][EPV], acc[V][EPV], derv[V], erj[HT], dacc = 0.f;
+  while (true) {
+    int4 nitem = item;
+    int nbase = base + G;
+    int nq = q;
+    bool has_next = true;
+    if (nbase >= item.z) {
+      nq = q + 1;
+      if (it0 + (int64_t)nq * stride >= n_items) {
+        has_next = false;
+      } else {
+        if (nq % G == 0) {
+          cp_async_wait<0>();
+          __syncwarp();
+          nitem = s_desc[(nq / G) & 1][w][0];
+          __syncwarp();
+          stage_desc(nq / G + 1);
+        } else {
+          nitem = s_desc[(nq / G) & 1][w][nq % G];
+        }
+        nbase = nitem.y;
+      }
+    }
+    const int nb_ = buf ^ 1;
+    if (has_next) stage_ids(nb_, nitem, nbase);
+    const int64_t j = item.x;
+    if (base == item.y) {
+      const T *rp = feat + j * a.ldf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        unpack(ldg16(rp + v * G * EPV), whf[v], T());
+        derv[v] = 0.f;
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+      }
+#pragma unroll
+      for (int h = 0; h < HT; ++h) erj[h] = s_er[buf][w][h];
+      dacc = 0.f;
+    }
+    const int *si = &s_i[buf][w][0];
+    const int c = base + gl;
+    const bool valid = c < item.z;
+    const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
+    uint4 ra[U][V], rz[U][V];
+    if (cnt > 0) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)si[min(u, cnt - 1)]);
+      if (nbt > 1) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)si[min(U + u, cnt - 1)]);
+      }
+    }
+#pragma unroll
+    for (int h = 0; h < HT; ++h)
+      if (h < H) {
+        const float z = s_el[buf][w][gl][h] + erj[h];
+        const float al = valid ? fexp(leaky(z, a.slope) - s_ls[buf][w][gl][h]) : 0.f;
+        s_a[w][lane][h] = z > 0.f ? al : -al;
+      }
+    cp_async_wait<0>();
+    __syncwarp();
+    if (has_next) stage_dst(nb_, nitem, nbase);
+    const float(*sd)[HT] = s_dl[buf][w];
+    auto consume = [&](const uint4 (&raw)[U][V], int k0) {
+      float p[U][V];
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float al = fabsf(s_a[w][k0 + u][hv[v]]);
+          float x[EPV];
+          unpack(raw[u][v], x, T());
+          float s0 = 0.f, s1 = 0.f;
+#pragma unroll
+          for (int k = 0; k < EPV; k += 2) {
+            ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
+            ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
+          }
+          p[u][v] = s0 + s1;
+        }
+      if constexpr (BFLY) {
+        float qv[NB];
+#pragma unroll
+        for (int i = 0; i < NB; ++i) qv[i] = p[i / V][i % V];
+#pragma unroll
+        for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
+          if (n > 1) {
+            const bool up = (gl & o) != 0;
+#pragma unroll
+            for (int i = 0; i < n / 2; ++i) {
+              const float send = up ? qv[i] : qv[i + n / 2];
+              const float keep = up ? qv[i + n / 2] : qv[i];
+              qv[i] = keep + __shfl_xor_sync(gmask, send, o);
+            }
+            n /= 2;
+          } else {
+            qv[0] += __shfl_xor_sync(gmask, qv[0], o);
+          }
+        }
+        const int er_ = k0 + bu;
+        const float sa = s_a[w][er_][bhead];
+        const float dz = fabsf(sa) * (qv[0] - sd[er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
+        dacc += dz;
+        if (bwriter) s_z[w][er_][bhead] = dz;
+      } else {
+        head_reduce<G, U, V, LPH>(p, gmask);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int er_ = k0 + u;
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float sa = s_a[w][er_][hv[v]];
+            const float dz = fabsf(sa) * (p[u][v] - sd[er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+            derv[v] += dz;
+            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
+          }
+        }
+      }
+    };
+    for (int b = 0; b < nbt; b += 2) {
+      consume(ra, b * U);
+      if (b + 2 < nbt) {
+#pragma unroll
+        for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)si[min((b + 2) * U + u, cnt - 1)]);
+      }
+      if (b + 1 < nbt) {
+        consume(rz, (b + 1) * U);
+        if (b + 3 < nbt) {
+#pragma unroll
+          for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)si[min((b + 3) * U + u, cnt - 1)]);
+        }
+      }
+    }
+    __syncwarp();
+    if (valid) {
+      float *dzp = a.dz + (int64_t)c * H;
+      if constexpr (HT == 4) {
+        reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
+      } else {
+        for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
+      }
+    }
+    if (base + G >= item.z) {  // last chunk of this source: finalise
+      if constexpr (BFLY) {
+        float dsum = dacc;
+#pragma unroll
+        for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o);
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          int src = gl;
+#pragma unroll
+          for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
+            const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
+            src = bit ? (src | o) : (src & ~o);
+          }
+          derv[v] = __shfl_sync(gmask, dsum, src);
+        }
+      }
+      if (item.w < 0) {
+        float *orow = a.gfeat + j * a.ldgf + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float *arp = a.ar + (v * G + gl) * EPV;
+          float y[EPV];
+#pragma unroll
+          for (int k = 0; k < EPV; k += 4) {
+            const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
+            y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
+            y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
+            if (!a.lp_partial)
+              *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          }
+          if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
+          if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
+        }
+      } else {
+        const int64_t slot = item.w;
+        float *pr = a.ws_bacc + slot * a.D + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+#pragma unroll
+          for (int k = 0; k < EPV; k += 4)
+            *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+                make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+          if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
+        }
+      }
+    }
+    if (!has_next) break;
+    cp_async_wait<0>();
+    __syncwarp();
+    item = nitem;
+    base = nbase;
+    q = nq;
+    buf = nb_;
+  }
+  cp_async_wait<0>();
+}
+
 // Split sources: dWh_j = sum_k acc_k + der_j a_r, der_j = sum_k der_k.
 template <typename T, int G, int V>
 __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a) {
@@ -937,11 +1447,13 @@ int l2_policy_mode() {
   }
   return v;
 }
+// forward kernel: 3 = chunk-pipelined gat_fwd_pipe_kernel (default; products 3 layers: 25.5 vs 29.3 ms/step),
+// 0/1/2 = gat_fwd_kernel batch variants
 int fwd_variant() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_FWD_VAR");
-    v = e ? std::atoi(e) : 0;
+    v = e ? std::atoi(e) : 3;
   }
   return v;
 }
@@ -955,6 +1467,15 @@ bool use_stream_fwd() {
   }
   return v == 1;
 }
+int pf_rows() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_PF_ROWS");
+    v = e ? std::atoi(e) : 0;  // 0..32 rows measured within 1% (the staging of ids/el/er is what pays)
+  }
+  return v;
+}
+// source pass: 0 = gat_bwd_src_kernel (default), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel
 int bwd_variant() {
   static int v = -1;
   if (v < 0) {
@@ -1121,6 +1642,10 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
           rc = check_launch(st, "gat_fwd_kernel");
         };
         switch (fwd_variant()) {
+          case 3:
+            if constexpr (G >= 8) launch(gat_fwd_pipe_kernel<T, G, V, HT>);  // (narrow rows: static smem)
+            else launch(gat_fwd_kernel<T, G, V, HT, 0>);
+            break;
           case 1: launch(gat_fwd_kernel<T, G, V, HT, 1>); break;
           case 2: launch(gat_fwd_kernel<T, G, V, HT, 2>); break;
           default: launch(gat_fwd_kernel<T, G, V, HT, 0>); break;
@@ -1155,7 +1680,12 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
         }
         if (a.L.n_bwd_items > 0) {
           auto launch = [&](auto ks) { ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a); };
-          if (bwd_variant() == 1) launch(gat_bwd_src_kernel<T, G, V, HT, 1>);
+          bool piped = false;
+          if constexpr (G == 32 && HT <= 4) {
+            if (bwd_variant() == 3) { launch(gat_bwd_src_pipe_kernel<T, V, HT>); piped = true; }
+          }
+          if (piped) {
+          } else if (bwd_variant() == 1) launch(gat_bwd_src_kernel<T, G, V, HT, 1>);
           else launch(gat_bwd_src_kernel<T, G, V, HT, 0>);
           if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
         }
@@ -1239,6 +1769,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.alpha = reinterpret_cast<float *>(wb + w.alpha);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.pf_rows = pf_rows();
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1289,6 +1820,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.lp_partial = 0;  // bf16 partial measured no faster than the fp32 partial (latency-bound); kept off
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.pf_rows = pf_rows();
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }

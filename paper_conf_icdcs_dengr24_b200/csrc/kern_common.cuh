@@ -250,6 +250,32 @@ __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commi
 template <int N> __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
 }
+// small cp.async staging copies (4 / 8 / 16 bytes, default L2 policy)
+template <int B> __device__ __forceinline__ void cp_async_small(void *smem, const void *gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  if constexpr (B == 16)
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(gmem) : "memory");
+  else
+    asm volatile("cp.async.ca.shared.global [%0], [%1], %2;" ::"r"(s), "l"(gmem), "n"(B) : "memory");
+}
+// H consecutive fp32 values (H a power of two <= 8, 4H-byte aligned) -> shared memory
+template <int HT> __device__ __forceinline__ void cp_async_h(float *smem, const float *gmem) {
+  if constexpr (HT == 8) {
+    cp_async_small<16>(smem, gmem);
+    cp_async_small<16>(smem + 4, gmem + 4);
+  } else {
+    cp_async_small<4 * HT>(smem, gmem);
+  }
+}
+// per-thread prefetch of the 128-byte line holding p into L2
+__device__ __forceinline__ void prefetch_l2_line(const void *p) {
+  asm volatile("prefetch.global.L2 [%0];" ::"l"(p));
+}
+// TMA-engine prefetch of a contiguous range into L2 (no registers, no completion tracking)
+__device__ __forceinline__ void prefetch_l2_bulk(const void *g, uint32_t bytes, uint64_t pol) {
+  asm volatile("cp.async.bulk.prefetch.L2.global.L2::cache_hint [%0], %1, %2;" ::"l"(g), "r"(bytes), "l"(pol)
+               : "memory");
+}
 
 struct FwdArgs {
   DevPart L;
@@ -265,6 +291,7 @@ struct FwdArgs {
   float *alpha;    // edge-streaming forward: [E_p][H] fp32 attention weights in CSR order
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
   int pol_mode; // MEGA_L2_POLICY
+  int pf_rows;  // gat_fwd_pipe_kernel: rows of the next chunk prefetched into L2 (MEGA_PF_ROWS)
 };
 
 struct BwdArgs {
@@ -290,6 +317,7 @@ struct BwdArgs {
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
   int lp_partial;  // ... and (both phases in one call) the source-phase partial lives in gfeat_lp too
+  int pf_rows;     // gat_bwd_src_pipe_kernel: g rows of the next chunk prefetched into L2 (MEGA_PF_ROWS)
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int pol_mode; // MEGA_L2_POLICY
 };
