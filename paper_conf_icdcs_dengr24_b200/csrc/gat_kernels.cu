@@ -900,6 +900,216 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   }
 }
 
+// ---- a7 with a shared-memory ring (G = 32) ----
+// gat_bwd_src_kernel's arithmetic, but the g rows of a chunk stream through a
+// per-warp ring of NBF batches of U rows filled with cp.async (LDGSTS): every
+// lane copies and later reads back exactly its own 16-byte pieces, so the ring
+// needs no barriers, and NBF*U rows per warp are in flight without holding
+// registers (the register-batch kernel keeps 2U = 4 in 125 registers).
+template <typename T, int V, int HT, int NBF>
+__global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
+  constexpr int U = V >= 4 ? 1 : (V == 2 ? 2 : 4), RS = NBF * U;  // rows per batch, ring slots
+  constexpr int NB = U * V;
+  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
+  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
+  extern __shared__ uint4 ring_all[];  // [WPB][RS][V][32]
+  __shared__ float s_a[WPB][32][SP];
+  __shared__ float s_d[WPB][32][SP];
+  __shared__ float s_z[WPB][32][SP];
+  __shared__ int s_i[WPB][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
+  const unsigned gmask = 0xffffffffu;
+  const int H = a.H;
+  uint4 *ring = ring_all + (size_t)w * RS * V * 32;
+  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
+  const int hot_cls = a.hot_cls;
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
+  int bidx = 0;
+#pragma unroll
+  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
+  const int bu = bidx / V, bv = bidx % V;
+  const int bhead = ((bv * G + gl) * EPV) / FF;
+  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *goutl = static_cast<const T *>(a.gout) + gl * EPV;
+  const int64_t stride = (int64_t)gridDim.x * WPB;
+  // batch b of the chunk (rows bU .. bU+U-1, clamped to the last) -> ring slots (b % NBF) U ..; one group per batch
+  auto issue = [&](int b, int cnt) {
+    if (b * U < cnt) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint32_t ii = (uint32_t)s_i[w][min(b * U + u, cnt - 1)];
+        const T *rp = goutl + (ii & idm) * ldg;
+        const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
+        uint4 *dst = ring + (((b % NBF) * U + u) * V) * 32 + lane;
+#pragma unroll
+        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
+      }
+    }
+    cp_async_commit();
+  };
+  for (int64_t it = (int64_t)blockIdx.x * WPB + w; it < a.L.n_bwd_items; it += stride) {
+    const int4 item = a.L.bwd_items[it];
+    const int64_t j = item.x;
+    float whf[V][EPV], acc[V][EPV], derv[V], dacc = 0.f;
+    {
+      const T *rp = feat + j * a.ldf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        unpack(ldg16(rp + v * G * EPV), whf[v], T());
+        derv[v] = 0.f;
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+      }
+    }
+    float erj[HT];
+    load_h<HT>(a.er + j * H, H, erj);
+    for (int base = item.y; base < item.z; base += G) {
+      const int c = base + gl;
+      const bool valid = c < item.z;
+      const int cnt = min(G, item.z - base), nb = (cnt + U - 1) / U;
+      const int ir = ld_stream(a.L.cdst + min(c, item.z - 1), pol_cold);
+      const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
+      float eli[HT], lsei[HT], dli[HT];
+      load_h<HT>(a.el + gi * H, H, eli);
+      load_h<HT>(a.lse + gi * H, H, lsei);
+      load_h<HT>(a.dlt + gi * H, H, dli);
+      s_i[w][lane] = ir;
+      __syncwarp();
+#pragma unroll
+      for (int b = 0; b < NBF; ++b) issue(b, cnt);
+#pragma unroll
+      for (int h = 0; h < HT; ++h)
+        if (h < H) {
+          const float z = eli[h] + erj[h];
+          const float al = valid ? fexp(leaky(z, a.slope) - lsei[h]) : 0.f;
+          s_a[w][lane][h] = z > 0.f ? al : -al;
+          s_d[w][lane][h] = dli[h];
+        }
+      __syncwarp();
+      for (int b = 0; b < nb; ++b) {
+        cp_async_wait<NBF - 1>();
+        const uint4 *slot = ring + ((b % NBF) * U * V) * 32 + lane;
+        const int k0 = b * U;
+        float p[U][V];
+#pragma unroll
+        for (int u = 0; u < U; ++u)
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float al = fabsf(s_a[w][k0 + u][hv[v]]);
+            float x[EPV];
+            unpack(slot[(u * V + v) * 32], x, T());
+            float s0 = 0.f, s1 = 0.f;
+#pragma unroll
+            for (int k = 0; k < EPV; k += 2) {
+              ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
+              ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
+            }
+            p[u][v] = s0 + s1;
+          }
+        issue(b + NBF, cnt);  // refill the slot just read (this lane's own pieces)
+        if constexpr (BFLY) {
+          float q[NB];
+#pragma unroll
+          for (int i = 0; i < NB; ++i) q[i] = p[i / V][i % V];
+#pragma unroll
+          for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
+            if (n > 1) {
+              const bool up = (gl & o) != 0;
+#pragma unroll
+              for (int i = 0; i < n / 2; ++i) {
+                const float send = up ? q[i] : q[i + n / 2];
+                const float keep = up ? q[i + n / 2] : q[i];
+                q[i] = keep + __shfl_xor_sync(gmask, send, o);
+              }
+              n /= 2;
+            } else {
+              q[0] += __shfl_xor_sync(gmask, q[0], o);
+            }
+          }
+          const int er_ = k0 + bu;
+          const float sa = s_a[w][er_][bhead];
+          const float dz = fabsf(sa) * (q[0] - s_d[w][er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
+          dacc += dz;
+          if (bwriter) s_z[w][er_][bhead] = dz;
+        } else {
+          head_reduce<G, U, V, LPH>(p, gmask);
+#pragma unroll
+          for (int u = 0; u < U; ++u) {
+            const int er_ = k0 + u;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const float sa = s_a[w][er_][hv[v]];
+              const float dz = fabsf(sa) * (p[u][v] - s_d[w][er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+              derv[v] += dz;
+              if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
+            }
+          }
+        }
+      }
+      cp_async_wait<0>();  // the ring is empty between chunks (issue() past the chunk commits empty groups)
+      __syncwarp();
+      if (valid) {
+        float *dzp = a.dz + (int64_t)c * H;
+        if constexpr (HT == 4) {
+          reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
+        } else {
+          for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
+        }
+      }
+      __syncwarp();
+    }
+    if constexpr (BFLY) {
+      float dsum = dacc;
+#pragma unroll
+      for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o);
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        int src = gl;
+#pragma unroll
+        for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
+          const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
+          src = bit ? (src | o) : (src & ~o);
+        }
+        derv[v] = __shfl_sync(gmask, dsum, src);
+      }
+    }
+    if (item.w < 0) {
+      float *orow = a.gfeat + j * a.ldgf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const float *arp = a.ar + (v * G + gl) * EPV;
+        float y[EPV];
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4) {
+          const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
+          y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
+          y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
+          if (!a.lp_partial)
+            *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+        }
+        if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
+        if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
+      }
+    } else {
+      const int64_t slot = item.w;
+      float *pr = a.ws_bacc + slot * a.D + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+              make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+        if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
+      }
+    }
+  }
+}
+
 // ---- a7, chunk-pipelined (G = 32, H <= 4) ----
 // gat_bwd_src_kernel's arithmetic with the fwd pipe kernel's staging: while
 // chunk c runs, the next chunk's destination ids, their (el, lse, Dlt) and
@@ -1475,12 +1685,14 @@ int pf_rows() {
   }
   return v;
 }
-// source pass: 0 = gat_bwd_src_kernel (default), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel
+// source pass: 4 = gat_bwd_src_ring_kernel with 4 batches in flight (default where G = 32 and V <= 2;
+// products 3 layers: gat_bwd 60.5 -> 52.9 ms/step), 5 = the ring with 6 batches (56.6), 0 = register-batch
+// gat_bwd_src_kernel (the default elsewhere), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel (60.3)
 int bwd_variant() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_BWD_VAR");
-    v = e ? std::atoi(e) : 0;
+    v = e ? std::atoi(e) : 4;
   }
   return v;
 }
@@ -1683,6 +1895,24 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
           bool piped = false;
           if constexpr (G == 32 && HT <= 4) {
             if (bwd_variant() == 3) { launch(gat_bwd_src_pipe_kernel<T, V, HT>); piped = true; }
+          }
+          if constexpr (G == 32 && V <= 2) {
+            const int bv = bwd_variant();
+            if (bv == 4 || bv == 5) {  // shared-memory ring: 4 = 4 batches in flight, 5 = 6 batches
+              auto ring_launch = [&](auto kr, int nbf) {
+                constexpr int U = V == 2 ? 2 : 4;
+                const size_t smem = (size_t)WPB * nbf * U * V * 32 * 16;
+                cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                int nblk = 0;
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
+                const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
+                                                        (int64_t)dev_info(dev).sms * std::max(nblk, 1));
+                kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
+              };
+              if (bv == 4) ring_launch(gat_bwd_src_ring_kernel<T, V, HT, 4>, 4);
+              else ring_launch(gat_bwd_src_ring_kernel<T, V, HT, 6>, 6);
+              piped = true;
+            }
           }
           if (piped) {
           } else if (bwd_variant() == 1) launch(gat_bwd_src_kernel<T, G, V, HT, 1>);
