@@ -58,7 +58,7 @@ size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays
   const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
                                       P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
-                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size()};
+                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size()};
   size_t off = 0;
   for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
@@ -223,7 +223,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   const std::vector<int32_t> ftiles = make_tiles(P.fwd_items), btiles = make_tiles(P.bwd_items);
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
-      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles};
+      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
@@ -247,6 +247,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.csrc = reinterpret_cast<const int32_t *>(base + offs[10]);
   D.ftiles = reinterpret_cast<const int4 *>(base + offs[11]);
   D.btiles = reinterpret_cast<const int4 *>(base + offs[12]);
+  D.cpos = reinterpret_cast<const int32_t *>(base + offs[13]);
   D.n_ftiles = (int32_t)(ftiles.size() / 4);
   D.n_btiles = (int32_t)(btiles.size() / 4);
   D.n = L->n;

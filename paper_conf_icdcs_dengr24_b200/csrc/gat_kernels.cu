@@ -669,7 +669,7 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
 // ---- a7: source-major pass over the CSC ----
 // For source j and out-edge (j -> i): alpha = exp(LeakyReLU(el_i + er_j) - lse_i),
 // dalpha = g_i . Wh_j, dz = alpha (dalpha - Dlt_i) (z > 0 ? 1 : slope);
-// dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored per CSC edge,
+// dWh_j = sum alpha g_i + der_j a_r with der_j = sum dz; dz stored at the edge's CSR position,
 // der_j into the der plane of ctx.  g rows stream through two register
 // batches; batches are branch-free (the chunk tail re-reads its last row with
 // alpha = 0).
@@ -732,6 +732,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
+      const int cp_c = ld_stream(a.L.cpos + min(c, item.z - 1), policy_first());  // dz's CSR position
       const int cnt = min(G, item.z - base), nb = (cnt + U - 1) / U;
       const int ir = ld_stream(a.L.cdst + min(c, item.z - 1), pol_cold);
       const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
@@ -840,7 +841,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
       }
       __syncwarp(gmask);
       if (valid) {
-        float *dzp = a.dz + (int64_t)c * H;
+        float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
         if (HT >= 4 && (H & 3) == 0) {
 #pragma unroll
           for (int q = 0; q < HT / 4; ++q)
@@ -971,6 +972,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
     for (int base = item.y; base < item.z; base += G) {
       const int c = base + gl;
       const bool valid = c < item.z;
+      const int cp_c = ld_stream(a.L.cpos + min(c, item.z - 1), policy_first());  // dz's CSR position
       const int cnt = min(G, item.z - base), nb = (cnt + U - 1) / U;
       const int ir = ld_stream(a.L.cdst + min(c, item.z - 1), pol_cold);
       const int64_t gi = a.L.row_begin + (int)((uint32_t)ir & idm);
@@ -1054,7 +1056,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       cp_async_wait<0>();  // the ring is empty between chunks (issue() past the chunk commits empty groups)
       __syncwarp();
       if (valid) {
-        float *dzp = a.dz + (int64_t)c * H;
+        float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
         if constexpr (HT == 4) {
           reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
         } else {
@@ -1245,6 +1247,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_pipe_kernel
     const int *si = &s_i[buf][w][0];
     const int c = base + gl;
     const bool valid = c < item.z;
+    const int cp_c = item.z > item.y ? ld_stream(a.L.cpos + min(c, item.z - 1), policy_first()) : 0;
     const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
     uint4 ra[U][V], rz[U][V];
     if (cnt > 0) {
@@ -1338,7 +1341,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_pipe_kernel
     }
     __syncwarp();
     if (valid) {
-      float *dzp = a.dz + (int64_t)c * H;
+      float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
       if constexpr (HT == 4) {
         reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
       } else {
@@ -1492,7 +1495,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     for (int h = 0; h < HT; ++h) dp[h] = 0.f;
     for (int e = e0 + gl; e < e1; e += G) {
       float t[HT];
-      load_h<HT>(a.dz + (int64_t)ld_stream(a.L.csr2csc + e, pol_cold) * H, H, t);
+      load_h<HT>(a.dz + (int64_t)e * H, H, t);  // dz is stored in CSR order by the source pass
 #pragma unroll
       for (int h = 0; h < HT; ++h)
         if (h < H) dp[h] += t[h];

@@ -27,6 +27,7 @@ struct DevPart {
   const int32_t *bwd_splits = nullptr;
   const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
   const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
+  const int32_t *cpos = nullptr;      // [E_p] CSR position of each CSC edge (dz is stored in CSR order)
   const int4 *ftiles = nullptr;      // (e_begin, e_end, slot, 0): runs of whole CSR rows / one split segment
   const int4 *btiles = nullptr;      // the same over the CSC (sources)
   int32_t n_ftiles = 0, n_btiles = 0;
@@ -68,7 +69,7 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-constexpr int kImageArrays = 13;
+constexpr int kImageArrays = 14;
 // Edge tiles of the streaming kernels: consecutive unsplit work items are
 // merged while their edges stay contiguous and total <= kTileEdges; a split
 // segment (slot >= 0) is a tile of its own; rows without edges are skipped.
