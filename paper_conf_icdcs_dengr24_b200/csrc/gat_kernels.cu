@@ -1451,10 +1451,10 @@ template <typename T, int G, int V, int HT>
 __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_dst_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, GPW = 32 / G;
   __shared__ double s_red[1024];
+  __shared__ __align__(16) float s_dz[2][WPB][32][HT];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H;
-  const uint64_t pol_cold = policy_first();
+  const int H = a.H, rb = grp * G;
   int hv[V];
   float dal[V][EPV], dar[V][EPV], alv[V][EPV];
 #pragma unroll
@@ -1465,7 +1465,19 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
   }
   const T *feat = static_cast<const T *>(a.feat);
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
+  // software pipeline over this group's rows: row k+1's first G dz values are
+  // staged in shared memory with cp.async (each lane copies and reads back its
+  // own slot: no barriers) and row k+2's indptr pair is loaded, while row k runs
+  auto stage_dz = [&](int b, int e0, int e1) {
+    if (e0 + gl < e1) cp_async_h<HT>(&s_dz[b][w][rb + gl][0], a.dz + (int64_t)(e0 + gl) * H);
+    cp_async_commit();
+  };
+  int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  int ce0 = 0, ce1 = 0, ne0 = 0, ne1 = 0, buf = 0;
+  if (r < a.L.rows) { ce0 = a.L.indptr[r]; ce1 = a.L.indptr[r + 1]; }
+  stage_dz(0, ce0, ce1);
+  if (r + stride < a.L.rows) { ne0 = a.L.indptr[r + stride]; ne1 = a.L.indptr[r + stride + 1]; }
+  for (; r < a.L.rows; r += stride) {
     const int64_t grow = a.L.row_begin + r;
     // row-local operands first: they do not depend on del, so their latency
     // overlaps the dz gather below
@@ -1489,11 +1501,17 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     }
     float derr[HT];
     load_h<HT>(a.der + grow * H, H, derr);
-    const int e0 = a.L.indptr[r], e1 = a.L.indptr[r + 1];
+    const int e0 = ce0, e1 = ce1;
+    if (r + stride < a.L.rows) stage_dz(buf ^ 1, ne0, ne1);
+    else cp_async_commit();
+    ce0 = ne0; ce1 = ne1;
+    if (r + 2 * stride < a.L.rows) { ne0 = a.L.indptr[r + 2 * stride]; ne1 = a.L.indptr[r + 2 * stride + 1]; }
+    cp_async_wait<1>();  // this row's staged dz
     float dp[HT];
 #pragma unroll
-    for (int h = 0; h < HT; ++h) dp[h] = 0.f;
-    for (int e = e0 + gl; e < e1; e += G) {
+    for (int h = 0; h < HT; ++h) dp[h] = e0 + gl < e1 ? s_dz[buf][w][rb + gl][h] : 0.f;
+    buf ^= 1;
+    for (int e = e0 + G + gl; e < e1; e += G) {
       float t[HT];
       load_h<HT>(a.dz + (int64_t)e * H, H, t);  // dz is stored in CSR order by the source pass
 #pragma unroll
@@ -1526,6 +1544,7 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
       }
     }
   }
+  cp_async_wait<0>();
   block_partial<G, V, EPV>(dal, s_red, a.ws_dal + (int64_t)blockIdx.x * a.D, a.D);
   block_partial<G, V, EPV>(dar, s_red, a.ws_dar + (int64_t)blockIdx.x * a.D, a.D);
 }
