@@ -206,8 +206,9 @@ class Model:
             x = Ld.L.out
         self.launches = sum(Ld.L.launches_per_step() for Ld in self.layers)
 
-    def step(self, ev=None):
-        """ev: optional dict name -> list of (start, end) event pairs to record into."""
+    def step(self, ev=None, before_bwd=None):
+        """ev: optional dict name -> list of (start, end) event pairs to record into;
+        before_bwd: called between the forward and the backward (e2e: wait for grad_out's copy)."""
         torch = self.torch
 
         def timed(name, fn):
@@ -222,6 +223,8 @@ class Model:
 
         for Ld in self.layers:
             Ld.forward(timed)
+        if before_bwd is not None:
+            before_bwd()
         g = self.g
         for Ld in reversed(self.layers):
             g = Ld.backward(g, timed)
@@ -366,6 +369,9 @@ def run_mega(args):
                 "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "algorithmic_bytes": bytes_per_launch,
                 "launch_ms": calls[dom], "peak_source": pk["source"],
                 "note": "algorithmic bytes = compulsory floor (each gathered row once, DESIGN.md §5)"}
+    if traffic:  # measured DRAM bytes of the same kernels (ncu, committed) over this run's live launch time
+        roofline["traffic_gbs"] = traffic / (calls[dom] * 1e-3) / 1e9
+        roofline["traffic_frac"] = roofline["traffic_gbs"] / pk["hbm_gbs"]
     # ---- e2e: this step's inputs from pinned host memory, parameter grads back ----
     e2e = None
     if not args.no_e2e:
@@ -377,10 +383,17 @@ def run_mega(args):
         h2d = hx.numel() * hx.element_size() + hg.numel() * hg.element_size()
         d2h = sum(o.numel() * o.element_size() for o in outs)
 
+        cs = torch.cuda.Stream(device=dev)
+
         def e2e_step():
+            # grad_out's host->device copy runs on a side stream, overlapped with the forward
+            cs.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(cs):
+                model.g.copy_(hg, non_blocking=True)
+                g_ready = torch.cuda.Event()
+                g_ready.record(cs)
             model.x0.copy_(hx, non_blocking=True)
-            model.g.copy_(hg, non_blocking=True)
-            model.step()
+            model.step(before_bwd=lambda: torch.cuda.current_stream().wait_event(g_ready))
             for h, o in zip(hout, outs):
                 h.copy_(o, non_blocking=True)
 
