@@ -149,7 +149,7 @@ def block_rows_for(cfg, dtype, block_rows=-1, l2_bytes=None):
     return M.auto_block_rows(cfg.dim * (2 if dtype == "bf16" else 4), l2_bytes)
 
 
-def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1):
+def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1, graph_only=False):
     import synth
     cfg = synth.CONFIGS[cfg_name]
     block_rows = block_rows_for(cfg, dtype, block_rows)
@@ -162,6 +162,9 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=
                                block_rows=block_rows)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
+    if graph_only:  # the CPU reference arm needs the graph and its layout only
+        return {"cfg": cfg, "indptr": indptr, "indices": indices, "layout": layout, "perm": perm,
+                "gen_s": t_gen, "pre_s": t_pre, "graph_stats": gstats}
     layers = []
     in_dim = cfg.f_in
     for li in range(cfg.layers):
@@ -261,13 +264,29 @@ def cpu_sample(wl, seconds_target, H, F):
         coracle.gat_backward(ptr, idx, Wh, a_l, a_r, g, fwd=f)
         return time.perf_counter() - t0, e
 
+    # host-memory bound: the oracle holds ~6 fp64 [k, H, F] arrays for the k touched nodes
+    try:
+        import psutil
+        cap = 0.4 * psutil.virtual_memory().available
+    except Exception:  # pragma: no cover
+        cap = 16e9
+
+    def fits(R):
+        k = len(np.unique(np.concatenate([np.arange(R, dtype=np.int64), src_new[:indptr_new[R]]])))
+        return k * H * F * 8 * 6 + 32 * int(indptr_new[R]) <= cap
+
     R = max(1, min(n, int(np.searchsorted(indptr_new, 200000))))
     t, e = run(R)
     for _ in range(3):
         if t >= seconds_target / 2 or R >= n:
             break
         e_want = int(e * seconds_target / max(t, 1e-3))
-        R = max(R + 1, min(n, int(np.searchsorted(indptr_new, min(wl["cfg"].m, e_want)))))
+        R2 = max(R + 1, min(n, int(np.searchsorted(indptr_new, min(wl["cfg"].m, e_want)))))
+        while R2 > R + 1 and not fits(R2):
+            R2 = R + (R2 - R) // 2
+        if R2 <= R + 1 and not fits(R2):
+            break
+        R = R2
         t, e = run(R)
     return run, R
 
@@ -284,7 +303,7 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    wl = build_workload(args.config, args.dtype, args.order, block_rows=args.block_rows)
+    wl = build_workload(args.config, args.dtype, args.order, block_rows=args.block_rows, graph_only=True)
     cfg = wl["cfg"]
     per_step = max(2.0, min(10.0, 150.0 / max(1, args.steps + args.warmup)))
     run, R = cpu_sample(wl, per_step, cfg.heads, cfg.head_dim)

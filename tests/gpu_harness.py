@@ -114,7 +114,9 @@ def assert_bf16_close(got, ref, name):
     assert np.array_equal(fin, np.isfinite(got)), f"{name}: finiteness differs"
     scale = np.max(np.abs(ref[fin])) if fin.any() else 0.0
     err = np.max(np.abs(got[fin] - ref[fin])) if fin.any() else 0.0
-    assert err <= 2e-2 * scale + 1e-30, f"{name}: max err {err:.3e} > 2e-2 * {scale:.3e}"
+    # + the fp32 absolute term (DESIGN.md R-tol): the bf16 path accumulates in fp32, and a tensor whose
+    # reference is exactly 0 by cancellation (e.g. all in-edges of a row from one source) keeps fp32 noise
+    assert err <= 2e-2 * scale + 1e-4, f"{name}: max err {err:.3e} > 2e-2 * {scale:.3e} + 1e-4"
 
 
 def assert_fp32_close_reduction(got, ref, name):

@@ -74,17 +74,23 @@ def test_attention_multipart_loopback(cuda_device, dtype, k):
     hz.check(got, _oracle(ip, ix, Wh, a_l, a_r, g), dtype)
 
 
-def test_edge_cases(cuda_device):
-    # single node without edges; graph where only one row has in-edges; a self-loop-only row
+# (H, F, dtype): narrow rows (register-batch source pass) and the G = 32 row widths of the
+# chunk-pipelined forward and the shared-memory-ring source pass (V = 1 and 2)
+@pytest.mark.parametrize("H,F,dtype", [(4, 8, "fp32"), (4, 128, "bf16"), (4, 64, "fp32"), (1, 256, "bf16")])
+def test_edge_cases(cuda_device, H, F, dtype):
+    # single node without edges; graph where only one row has in-edges; a self-loop-only row;
+    # a 70-edge hub row next to empty rows (split into segments, several chunks per segment)
+    hub = synth.from_edge_list(9, list(np.arange(70) % 9), [4] * 70)
     for ip, ix in [(np.array([0, 0]), np.zeros(0, np.int32)),
                    synth.from_edge_list(6, [1, 2, 3, 4, 5], [0, 0, 0, 0, 0]),
-                   synth.from_edge_list(4, [2, 2, 2, 0], [2, 2, 2, 1])]:
+                   synth.from_edge_list(4, [2, 2, 2, 0], [2, 2, 2, 1]), hub]:
         n = len(ip) - 1
-        Wh, a_l, a_r, g = hz.inputs(1, n, 4, 8, False)
-        lay = M.mega_preprocess(ip, ix, seg_edges=2)
-        got = hz.run_attention(lay, Wh, a_l, a_r, g, "fp32")
-        ref = _oracle(ip, ix, Wh, a_l, a_r, g)
-        hz.check(got, ref, "fp32")
+        Wh, a_l, a_r, g = hz.inputs(1, n, H, F, dtype == "bf16")
+        for seg in (2, 64):
+            lay = M.mega_preprocess(ip, ix, seg_edges=seg)
+            got = hz.run_attention(lay, Wh, a_l, a_r, g, dtype)
+            ref = _oracle(ip, ix, Wh, a_l, a_r, g)
+            hz.check(got, ref, dtype)
         deg = np.diff(ip)
         assert np.all(got["out"][deg == 0] == 0) and np.all(got["lse"][deg == 0] == -np.inf)
 
