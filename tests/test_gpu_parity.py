@@ -76,7 +76,8 @@ def test_attention_multipart_loopback(cuda_device, dtype, k):
 
 # (H, F, dtype): narrow rows (register-batch source pass) and the G = 32 row widths of the
 # chunk-pipelined forward and the shared-memory-ring source pass (V = 1 and 2)
-@pytest.mark.parametrize("H,F,dtype", [(4, 8, "fp32"), (4, 128, "bf16"), (4, 64, "fp32"), (1, 256, "bf16")])
+@pytest.mark.parametrize("H,F,dtype", [(4, 8, "fp32"), (4, 128, "bf16"), (4, 64, "fp32"), (1, 256, "bf16"),
+                                       (1, 128, "fp32")])
 def test_edge_cases(cuda_device, H, F, dtype):
     # single node without edges; graph where only one row has in-edges; a self-loop-only row;
     # a 70-edge hub row next to empty rows (split into segments, several chunks per segment)
@@ -90,7 +91,13 @@ def test_edge_cases(cuda_device, H, F, dtype):
             lay = M.mega_preprocess(ip, ix, seg_edges=seg)
             got = hz.run_attention(lay, Wh, a_l, a_r, g, dtype)
             ref = _oracle(ip, ix, Wh, a_l, a_r, g)
-            hz.check(got, ref, dtype)
+            keys = ["out", "lse", "grad_feat", "grad_attn_l", "grad_attn_r"]
+            if dtype == "bf16":
+                # these graphs make the parameter gradients 0 by exact cancellation (every row's in-edges
+                # come from one source, so ds = 0); in bf16 mode Dlt = g . out reads the stored bf16 out
+                # (DESIGN R-prec), which leaves a rounding residue there -- the fp32 cases check them exactly
+                keys = [k for k in keys if not (k.startswith("grad_attn") and np.max(np.abs(ref[k])) < 1e-9)]
+            hz.check(got, ref, dtype, keys=keys)
         deg = np.diff(ip)
         assert np.all(got["out"][deg == 0] == 0) and np.all(got["lse"][deg == 0] == -np.inf)
 
