@@ -1405,6 +1405,297 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_pipe_kernel
   cp_async_wait<0>();
 }
 
+// ---- a7, chunk-pipelined with a shared-memory ring (G = 32, H <= 4) ----
+// gat_bwd_src_pipe_kernel's staging of the next chunk (ids, el / lse / Dlt, er)
+// combined with gat_bwd_src_ring_kernel's cp.async ring for the g rows.
+// gat_bwd_src_kernel's arithmetic with the fwd pipe kernel's staging: while
+// chunk c runs, the next chunk's destination ids, their (el, lse, Dlt) and
+// (for a new source) er_j are staged in shared memory with cp.async, and the
+// next chunk's g rows and the next source's Wh row are prefetched into L2.
+template <typename T, int V, int HT, int NBF>
+__global__ void __launch_bounds__(TPB, 2) gat_bwd_src_pipering_kernel(const BwdArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
+  constexpr int U1 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U1 < G ? U1 : G;
+  constexpr int NB = U * V;
+  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
+  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
+  extern __shared__ uint4 ring_all[];  // [WPB][NBF * U][V][32]
+  __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
+  __shared__ float s_z[WPB][32][SP];  // dz out
+  __shared__ int4 s_desc[2][WPB][32];
+  __shared__ int s_i[2][WPB][32];     // packed destination rows of a chunk
+  __shared__ __align__(16) float s_el[2][WPB][32][HT];
+  __shared__ __align__(16) float s_ls[2][WPB][32][HT];
+  __shared__ __align__(16) float s_dl[2][WPB][32][HT];
+  __shared__ __align__(16) float s_er[2][WPB][HT];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
+  const unsigned gmask = 0xffffffffu;
+  const int H = a.H;
+  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
+  const int hot_cls = a.hot_cls;
+  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
+  const uint32_t grow_bytes = (uint32_t)(a.D * sizeof(T));
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
+  int bidx = 0;
+#pragma unroll
+  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
+  const int bu = bidx / V, bv = bidx % V;
+  const int bhead = ((bv * G + gl) * EPV) / FF;
+  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *gout = static_cast<const T *>(a.gout);
+  const T *goutl = gout + gl * EPV;
+  const int64_t stride = (int64_t)gridDim.x * WPB;
+  const int64_t it0 = (int64_t)blockIdx.x * WPB + w, n_items = a.L.n_bwd_items;
+  if (it0 >= n_items) return;
+  uint4 *ring = ring_all + (size_t)w * NBF * U * V * 32;
+  // batch b of the current chunk -> ring slots (b % NBF) U ..; one cp.async group per batch (empty past the chunk)
+  auto issue = [&](const int *ids, int b, int cnt) {
+    if (b * U < cnt) {
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const uint32_t ii = (uint32_t)ids[min(b * U + u, cnt - 1)];
+        const T *rp = goutl + (ii & idm) * ldg;
+        const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
+        uint4 *dst = ring + (((b % NBF) * U + u) * V) * 32 + lane;
+#pragma unroll
+        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
+      }
+    }
+    cp_async_commit();
+  };
+  auto stage_desc = [&](int k) {
+    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
+    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][gl], a.L.bwd_items + itq);
+    cp_async_commit();
+  };
+  // chunk (itm, bse): destination ids; for the first chunk of a source its er, and its Wh row into L2
+  auto stage_ids = [&](int b, int4 itm, int bse) {
+    if (itm.z > itm.y) cp_async_small<4>(&s_i[b][w][gl], a.L.cdst + min(bse + gl, itm.z - 1));
+    else s_i[b][w][gl] = 0;
+    if (bse == itm.y && gl == 0) {
+      cp_async_h<HT>(&s_er[b][w][0], a.er + (int64_t)itm.x * H);
+      prefetch_l2_bulk(feat + (int64_t)itm.x * a.ldf, grow_bytes, pol_row);
+    }
+    cp_async_commit();
+  };
+  // the staged chunk's destination values, and its g rows into L2
+  auto stage_dst = [&](int b, int4 itm, int bse) {
+    const uint32_t ii = (uint32_t)s_i[b][w][gl];
+    const int64_t gi = a.L.row_begin + (int)(ii & idm);
+    cp_async_h<HT>(&s_el[b][w][gl][0], a.el + gi * H);
+    cp_async_h<HT>(&s_ls[b][w][gl][0], a.lse + gi * H);
+    cp_async_h<HT>(&s_dl[b][w][gl][0], a.dlt + gi * H);
+    cp_async_commit();
+    // the chunk's first pf_rows g rows into L2, one 128-byte line per lane per step
+    constexpr int LPR = (32 * V * 16) / 128, RPS = 32 / LPR;
+    const int cnt_n = min(a.pf_rows, itm.z - bse);
+    for (int r0 = 0; r0 < cnt_n; r0 += RPS) {
+      const int r = r0 + gl / LPR;
+      if (r < cnt_n)
+        prefetch_l2_line(reinterpret_cast<const char *>(gout + ((uint32_t)s_i[b][w][r] & idm) * ldg) + (gl % LPR) * 128);
+    }
+  };
+  stage_desc(0);
+  stage_desc(1);
+  cp_async_wait<1>();
+  __syncwarp();
+  int q = 0;
+  int4 item = s_desc[0][w][0];
+  int base = item.y, buf = 0;
+  stage_ids(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp();
+  stage_dst(0, item, base);
+  cp_async_wait<0>();
+  __syncwarp();
+  float whf[V][EPV], acc[V][EPV], derv[V], erj[HT], dacc = 0.f;
+  while (true) {
+    int4 nitem = item;
+    int nbase = base + G;
+    int nq = q;
+    bool has_next = true;
+    if (nbase >= item.z) {
+      nq = q + 1;
+      if (it0 + (int64_t)nq * stride >= n_items) {
+        has_next = false;
+      } else {
+        if (nq % G == 0) {
+          cp_async_wait<0>();
+          __syncwarp();
+          nitem = s_desc[(nq / G) & 1][w][0];
+          __syncwarp();
+          stage_desc(nq / G + 1);
+        } else {
+          nitem = s_desc[(nq / G) & 1][w][nq % G];
+        }
+        nbase = nitem.y;
+      }
+    }
+    const int nb_ = buf ^ 1;
+    if (has_next) stage_ids(nb_, nitem, nbase);
+    const int64_t j = item.x;
+    if (base == item.y) {
+      const T *rp = feat + j * a.ldf + gl * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        unpack(ldg16(rp + v * G * EPV), whf[v], T());
+        derv[v] = 0.f;
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+      }
+#pragma unroll
+      for (int h = 0; h < HT; ++h) erj[h] = s_er[buf][w][h];
+      dacc = 0.f;
+    }
+    const int *si = &s_i[buf][w][0];
+    const int c = base + gl;
+    const bool valid = c < item.z;
+    const int cp_c = item.z > item.y ? ld_stream(a.L.cpos + min(c, item.z - 1), policy_first()) : 0;
+    const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
+#pragma unroll
+    for (int b = 0; b < NBF; ++b) issue(si, b, cnt);
+#pragma unroll
+    for (int h = 0; h < HT; ++h)
+      if (h < H) {
+        const float z = s_el[buf][w][gl][h] + erj[h];
+        const float al = valid ? fexp(leaky(z, a.slope) - s_ls[buf][w][gl][h]) : 0.f;
+        s_a[w][lane][h] = z > 0.f ? al : -al;
+      }
+    cp_async_wait<NBF>();  // the next chunk's ids (older than the NBF ring groups) have landed
+    __syncwarp();
+    if (has_next) stage_dst(nb_, nitem, nbase);
+    else cp_async_commit();  // keep the group count uniform
+    const float(*sd)[HT] = s_dl[buf][w];
+    auto consume = [&](const uint4 *slot, int k0) {
+      float p[U][V];
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float al = fabsf(s_a[w][k0 + u][hv[v]]);
+          float x[EPV];
+          unpack(slot[(u * V + v) * 32], x, T());
+          float s0 = 0.f, s1 = 0.f;
+#pragma unroll
+          for (int k = 0; k < EPV; k += 2) {
+            ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
+            ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
+          }
+          p[u][v] = s0 + s1;
+        }
+      if constexpr (BFLY) {
+        float qv[NB];
+#pragma unroll
+        for (int i = 0; i < NB; ++i) qv[i] = p[i / V][i % V];
+#pragma unroll
+        for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
+          if (n > 1) {
+            const bool up = (gl & o) != 0;
+#pragma unroll
+            for (int i = 0; i < n / 2; ++i) {
+              const float send = up ? qv[i] : qv[i + n / 2];
+              const float keep = up ? qv[i + n / 2] : qv[i];
+              qv[i] = keep + __shfl_xor_sync(gmask, send, o);
+            }
+            n /= 2;
+          } else {
+            qv[0] += __shfl_xor_sync(gmask, qv[0], o);
+          }
+        }
+        const int er_ = k0 + bu;
+        const float sa = s_a[w][er_][bhead];
+        const float dz = fabsf(sa) * (qv[0] - sd[er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
+        dacc += dz;
+        if (bwriter) s_z[w][er_][bhead] = dz;
+      } else {
+        head_reduce<G, U, V, LPH>(p, gmask);
+#pragma unroll
+        for (int u = 0; u < U; ++u) {
+          const int er_ = k0 + u;
+#pragma unroll
+          for (int v = 0; v < V; ++v) {
+            const float sa = s_a[w][er_][hv[v]];
+            const float dz = fabsf(sa) * (p[u][v] - sd[er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
+            derv[v] += dz;
+            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
+          }
+        }
+      }
+    };
+    for (int b = 0; b < nbt; ++b) {
+      cp_async_wait<NBF>();  // groups after batch b: NBF - 1 - b ring batches, the dst staging, b refills
+      consume(ring + ((b % NBF) * U * V) * 32 + lane, b * U);
+      issue(si, b + NBF, cnt);
+    }
+    __syncwarp();
+    if (valid) {
+      float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
+      if constexpr (HT == 4) {
+        reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
+      } else {
+        for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
+      }
+    }
+    if (base + G >= item.z) {  // last chunk of this source: finalise
+      if constexpr (BFLY) {
+        float dsum = dacc;
+#pragma unroll
+        for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o);
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          int src = gl;
+#pragma unroll
+          for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
+            const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
+            src = bit ? (src | o) : (src & ~o);
+          }
+          derv[v] = __shfl_sync(gmask, dsum, src);
+        }
+      }
+      if (item.w < 0) {
+        float *orow = a.gfeat + j * a.ldgf + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const float *arp = a.ar + (v * G + gl) * EPV;
+          float y[EPV];
+#pragma unroll
+          for (int k = 0; k < EPV; k += 4) {
+            const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
+            y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
+            y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
+            if (!a.lp_partial)
+              *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          }
+          if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
+          if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
+        }
+      } else {
+        const int64_t slot = item.w;
+        float *pr = a.ws_bacc + slot * a.D + gl * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+#pragma unroll
+          for (int k = 0; k < EPV; k += 4)
+            *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
+                make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+          if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
+        }
+      }
+    }
+    if (!has_next) break;
+    cp_async_wait<0>();
+    __syncwarp();
+    item = nitem;
+    base = nbase;
+    q = nq;
+    buf = nb_;
+  }
+  cp_async_wait<0>();
+}
+
 // Split sources: dWh_j = sum_k acc_k + der_j a_r, der_j = sum_k der_k.
 template <typename T, int G, int V>
 __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a) {
@@ -1709,7 +2000,8 @@ int pf_rows() {
 }
 // source pass: 4 = gat_bwd_src_ring_kernel with 4 batches in flight (default where G = 32 and V <= 2;
 // products 3 layers: gat_bwd 60.5 -> 52.9 ms/step), 5 = the ring with 6 batches (56.6), 0 = register-batch
-// gat_bwd_src_kernel (the default elsewhere), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel (60.3)
+// gat_bwd_src_kernel (the default elsewhere), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel (60.3),
+// 6 = gat_bwd_src_pipering_kernel (staged chain + ring: 49.7-50.1 vs 48.1 for 4; the staging costs more than it hides)
 int bwd_variant() {
   static int v = -1;
   if (v < 0) {
@@ -1917,6 +2209,20 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
           bool piped = false;
           if constexpr (G == 32 && HT <= 4) {
             if (bwd_variant() == 3) { launch(gat_bwd_src_pipe_kernel<T, V, HT>); piped = true; }
+            if constexpr (V <= 2) {
+              if (bwd_variant() == 6) {  // staged chain + shared-memory ring (4 batches in flight)
+                constexpr int U = V == 2 ? 2 : 4, NBF = 4;
+                auto kr = gat_bwd_src_pipering_kernel<T, V, HT, NBF>;
+                const size_t smem = (size_t)WPB * NBF * U * V * 32 * 16;
+                cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+                int nblk = 0;
+                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
+                const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
+                                                        (int64_t)dev_info(dev).sms * std::max(nblk, 1));
+                kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
+                piped = true;
+              }
+            }
           }
           if constexpr (G == 32 && V <= 2) {
             const int bv = bwd_variant();
