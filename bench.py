@@ -151,7 +151,7 @@ def block_rows_for(cfg, dtype, block_rows=-1, l2_bytes=None):
 
 def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1, graph_only=False):
     import synth
-    cfg = synth.CONFIGS[cfg_name]
+    cfg = synth.get_config(cfg_name)
     block_rows = block_rows_for(cfg, dtype, block_rows)
     t0 = time.time()
     indptr, indices, gstats = synth.make_graph(cfg)

@@ -64,6 +64,9 @@ class GraphConfig:
     mu: float
     gamma: float
     d_cap: float
+    batch: str = ""       # Table II dataset shape of a block-diagonal batch (synth/batch.py), "" = one graph
+    num_graphs: int = 0
+    drop: float = 0.0     # edge-dropping fraction per graph
 
     @property
     def f_in_pad(self) -> int:    # 16-byte rows for bf16 (TMA/ld.128): multiple of 8
@@ -88,6 +91,36 @@ CONFIGS = {
 }
 
 
+# The paper's own workload: batches of small graphs, hidden 128 = 8 heads x 16
+# (batch 64 / hidden 128; batch 64, 128, 256; 20% edge drop).
+# n and m are filled in from the generated batch by get_config().
+_BATCHES = {
+    "zinc-b64": ("zinc", 64, 0.0), "zinc-b128": ("zinc", 128, 0.0), "zinc-b256": ("zinc", 256, 0.0),
+    "aqsol-b128": ("aqsol", 128, 0.0), "aqsol-b128-drop20": ("aqsol", 128, 0.2),
+    "csl-b128": ("csl", 128, 0.0), "cycles-b128": ("cycles", 128, 0.0),
+}
+
+
+def _batch_graph(name, num_graphs, drop, seed):
+    from synth.batch import drop_edges, make_batch
+    ip, ix, gptr = make_batch(name, num_graphs, seed)
+    if drop > 0:
+        ip, ix = drop_edges(ip, ix, gptr, drop, seed + 1)
+    return ip, ix, gptr
+
+
+def get_config(name: str) -> GraphConfig:
+    """BASELINE.json configs by name, or a batch config (exact n, m of its seeded batch)."""
+    if name in CONFIGS:
+        return CONFIGS[name]
+    ds, b, drop = _BATCHES[name]
+    index = 5 + sorted(_BATCHES).index(name)
+    seed = 0x4D454741 + 16 * index
+    ip, ix, _ = _batch_graph(ds, b, drop, seed)
+    return GraphConfig(name, index, len(ip) - 1, len(ix), False, 128, 8, 16, 4, 0, 0.0, 0.0, 0.0,
+                       batch=ds, num_graphs=b, drop=drop)
+
+
 def scaled(cfg: GraphConfig, n: int, m: int, name: str | None = None) -> GraphConfig:
     """Same shape recipe at a smaller size (for tests)."""
     if not cfg.directed and m % 2:
@@ -99,6 +132,9 @@ def scaled(cfg: GraphConfig, n: int, m: int, name: str | None = None) -> GraphCo
 
 def make_graph(cfg: GraphConfig):
     """-> (indptr int64[n+1], indices int32[m], stats dict).  Rows are destinations."""
+    if cfg.batch:
+        ip, ix, _ = _batch_graph(cfg.batch, cfg.num_graphs, cfg.drop, cfg.seed)
+        return ip, ix, {"duplicates": 0, "self_loops": 0}
     lib = _load()
     indptr = np.empty(cfg.n + 1, dtype=np.int64)
     indices = np.empty(cfg.m, dtype=np.int32)

@@ -131,11 +131,12 @@ def test_ablation_orders_same_result(cuda_device, order):
 
 
 @pytest.mark.parametrize("dtype", ["fp32", "bf16"])
-@pytest.mark.parametrize("name", ["cora", "products-small"])
+@pytest.mark.parametrize("name", ["cora", "products-small", "zinc-b64", "aqsol-b128-drop20"])
 def test_whole_layer(cuda_device, dtype, name):
     """a2-a9 through GATLayer: projection on tensor cores, attention, backward,
     projection backward; oracle computes Wh = X W in fp64 from the same X, W."""
-    cfg = synth.CONFIGS["cora"] if name == "cora" else synth.scaled(synth.CONFIGS["products"], 5000, 120000)
+    cfg = (synth.scaled(synth.CONFIGS["products"], 5000, 120000) if name == "products-small"
+           else synth.get_config(name))
     ip, ix, _ = synth.make_graph(cfg)
     inp = synth.make_layer_inputs(cfg)
     x, w = inp["x"], inp["w"]
