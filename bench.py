@@ -50,6 +50,8 @@ def parse():
     ap.add_argument("--seg-edges", type=int, default=0, help="work-item segment size S (0 = auto)")
     ap.add_argument("--block-rows", type=int, default=-1,
                     help="L2 blocking B (DESIGN.md R24): -1 = auto (0.4 L2 / row bytes), 0 = off")
+    ap.add_argument("--cuda-graph", action="store_true",
+                    help="capture one step in a CUDA graph and replay it (launch-bound batch workloads)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -356,16 +358,57 @@ def run_mega(args):
         model.step()
     sync_all()
     # ---- device-timed region (inputs resident; inputs >> L2 so no flush) ----
+    graph = None
+    if args.cuda_graph:   # one step captured once; every kernel in it is ours or cuBLAS's
+        side = torch.cuda.Stream(device=dev)
+        side.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(side):
+            model.step()
+        torch.cuda.current_stream().wait_stream(side)
+        graph = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(graph):
+            model.step()
+        for _ in range(max(3, args.warmup)):
+            graph.replay()
+        sync_all()
+    run_step = (lambda: graph.replay()) if graph is not None else (lambda: model.step())
+    # inputs smaller than L2 (the batch workloads): flush L2 between timed steps, outside the events
+    sb0 = 2 if args.dtype == "bf16" else 4
+    l2_bytes = torch.cuda.get_device_properties(dev).L2_cache_size
+    flush = None
+    if cfg.n * cfg.dim * sb0 * 4 < 2 * l2_bytes:
+        flush = torch.empty(2 * l2_bytes // 4, dtype=torch.float32, device=dev)
     ev = {}
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         sync_all()
-        start.record()
-        for _ in range(args.steps):
-            model.step(ev)
-        end.record()
+        if flush is None and graph is None:
+            start.record()
+            for _ in range(args.steps):
+                model.step(ev)
+            end.record()
+            sync_all()
+            ms_step = start.elapsed_time(end) / args.steps
+        else:
+            pairs = []
+            for _ in range(args.steps):
+                if flush is not None:
+                    flush.fill_(1.0)
+                s1, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                s1.record()
+                run_step()
+                e1.record()
+                pairs.append((s1, e1))
+            sync_all()
+            ms_step = float(np.sum([a.elapsed_time(b) for a, b in pairs])) / args.steps
+    if graph is not None or flush is not None:   # per-call breakdown from a separate eager pass
         sync_all()
-    ms_t = torch.tensor([start.elapsed_time(end) / args.steps], device=dev)
+        for _ in range(args.steps):
+            if flush is not None:
+                flush.fill_(1.0)
+            model.step(ev)
+        sync_all()
+    ms_t = torch.tensor([ms_step], device=dev)
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms = float(ms_t.item())
@@ -412,7 +455,11 @@ def run_mega(args):
                 g_ready = torch.cuda.Event()
                 g_ready.record(cs)
             model.x0.copy_(hx, non_blocking=True)
-            model.step(before_bwd=lambda: torch.cuda.current_stream().wait_event(g_ready))
+            if graph is not None:
+                torch.cuda.current_stream().wait_event(g_ready)
+                graph.replay()
+            else:
+                model.step(before_bwd=lambda: torch.cuda.current_stream().wait_event(g_ready))
             for h, o in zip(hout, outs):
                 h.copy_(o, non_blocking=True)
 
@@ -445,14 +492,20 @@ def run_mega(args):
             "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": world, "steps": args.steps,
             "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "strong",
             "vs_baseline": None, "dtype": args.dtype,
-            "data": "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)",
+            "data": ("synthetic (mega-synth v1: Table II-shaped block-diagonal batch, seeded; random-init weights)"
+                     if cfg.batch else "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)"),
             "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
                        "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
                        "order": args.order, "block_rows": st["block_rows"],
                        "parallelism": "single GPU" if world == 1 else
                        f"dst-partitioned x{world} (NCCL all-gather-v of [Wh|er], reduce-to-owner of [dWh|der])",
                        "value_definition": "layers * E / step time (each layer's edges fwd+bwd; max over ranks)",
-                       "l2": "no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)},
+                       "l2": ("no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)
+                              if flush is None else "L2 flushed between timed steps (%d MB write, outside the "
+                              "events)" % (flush.numel() * 4 >> 20)),
+                       "cuda_graph": graph is not None,
+                       **({"batch": cfg.batch, "num_graphs": cfg.num_graphs, "edge_drop": cfg.drop}
+                          if cfg.batch else {})},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
             "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
             "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",
