@@ -13,6 +13,8 @@ follows; PAPER.md:L = line L of /root/reference/PAPER.md):
                (readings R1-R12).
   layout.py    The exact relabelled layout built from the traversal's
                permutation (PAPER.md:34, 310; DESIGN.md "Layout").
+  gt.py        Graph Transformer attention (Q.K/sqrt(F) scores), fp64 — NEXT-3
+               row, oracle only so far (DESIGN.md R-gt).
   c/oracle.c   The same definitions as plain C loops (fp64, OpenMP over
                destinations) for sizes numpy cannot reach in seconds;
                loaded through coracle.py.
