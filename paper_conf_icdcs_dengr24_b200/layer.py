@@ -87,6 +87,6 @@ class GATLayer:
 
     def launches_per_step(self) -> int:
         """Our kernels per step (cuBLAS GEMMs excluded): eler, fwd, [fwd merge], dlt, bwd_src,
-        [bwd_src merge], reduce(a_r), bwd_dst, reduce(a_l)."""
+        [bwd_src merge], bwd_dst, reduce(a_l, a_r)."""
         v = self.layout.view(self.part, arrays=False)
-        return 7 + (1 if v["num_fwd_splits"] > 0 else 0) + (1 if v["num_bwd_splits"] > 0 else 0)
+        return 6 + (1 if v["num_fwd_splits"] > 0 else 0) + (1 if v["num_bwd_splits"] > 0 else 0)

@@ -96,6 +96,10 @@ def lib():
             "mega_gat_bwd": (S, [P, _c.c_int32, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64,
                                  P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P]),
             "mega_project_bwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, S, P, I64, P, I64, P, P]),
+            "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P]),
+            "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, P]),
+            "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P, I64, P, P, P, I64,
+                                P, _c.c_size_t, P]),
         }
         for name, (res, args) in sig.items():
             f = getattr(L, name)
@@ -276,3 +280,23 @@ def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_d
     _check(lib().mega_project_bwd(_ptr(x), x.stride(0), x.shape[0], in_dim or w.shape[0], _ptr(w), heads, head_dim,
                                   dt, _ptr(grad_feat), grad_feat.stride(0), _ptr(grad_x),
                                   grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _stream(stream)))
+
+
+# NEXT-3: Graph Transformer edge attention (include/mega.h mega_gt_*; fp32)
+def mega_gt_workspace_bytes(layout: Layout, part: int, heads: int):
+    b = _c.c_size_t()
+    _check(lib().mega_gt_workspace_bytes(layout.handle, part, heads, _c.byref(b)))
+    return b.value
+
+
+def mega_gt_fwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, stream=None):
+    _check(lib().mega_gt_fwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
+                             out.stride(0), _ptr(lse), _stream(stream)))
+
+
+def mega_gt_bwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, grad_out, grad_q, grad_k, grad_v, ws,
+                stream=None):
+    _check(lib().mega_gt_bwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
+                             out.stride(0), _ptr(lse), _ptr(grad_out), grad_out.stride(0), _ptr(grad_q), _ptr(grad_k),
+                             _ptr(grad_v), grad_k.stride(0), _ptr(ws), ws.numel() * ws.element_size(),
+                             _stream(stream)))
