@@ -57,7 +57,35 @@ __global__ void __launch_bounds__(kWarps * 32) gt_fwd_kernel(Args a) {
     }
     float m = -INFINITY, S = 0.f;
     const int e0 = a.L.indptr[r], e1 = a.L.indptr[r + 1];
-    for (int e = e0; e < e1; ++e) {
+    int e = e0;
+    for (; e + 1 < e1; e += 2) {    // two edges per iteration: both rows' loads in flight together
+      const int64_t j0 = (int64_t)((uint32_t)a.L.src[e] & a.L.id_mask);
+      const int64_t j1 = (int64_t)((uint32_t)a.L.src[e + 1] & a.L.id_mask);
+      const float *k0 = a.k + j0 * a.ld + h * a.F, *k1 = a.k + j1 * a.ld + h * a.F;
+      const float *v0 = a.v + j0 * a.ld + h * a.F, *v1 = a.v + j1 * a.ld + h * a.F;
+      float p0 = 0.f, p1 = 0.f, w0[KF], w1[KF];
+#pragma unroll
+      for (int t = 0; t < KF; ++t) {
+        const int f = lane + 32 * t;
+        const bool ok = f < a.F;
+        p0 += ok ? q[t] * k0[f] : 0.f;
+        p1 += ok ? q[t] * k1[f] : 0.f;
+        w0[t] = ok ? v0[f] : 0.f;
+        w1[t] = ok ? v1[f] : 0.f;
+      }
+#pragma unroll
+      for (int o = 16; o; o >>= 1) {
+        p0 += __shfl_xor_sync(0xffffffffu, p0, o);
+        p1 += __shfl_xor_sync(0xffffffffu, p1, o);
+      }
+      const float mn = fmaxf(m, fmaxf(p0, p1));
+      const float c = __expf(m - mn), x0 = __expf(p0 - mn), x1 = __expf(p1 - mn);
+      S = S * c + x0 + x1;
+#pragma unroll
+      for (int t = 0; t < KF; ++t) acc[t] = acc[t] * c + x0 * w0[t] + x1 * w1[t];
+      m = mn;
+    }
+    for (; e < e1; ++e) {
       const int64_t j = (int64_t)((uint32_t)a.L.src[e] & a.L.id_mask);
       const float *kj = a.k + j * a.ld + h * a.F;
       const float *vj = a.v + j * a.ld + h * a.F;
