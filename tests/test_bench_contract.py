@@ -40,3 +40,18 @@ def test_gpu_arm_line():
     assert d["cpu_baseline"]["kind"] == "oracle"
     assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
     assert {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
+
+
+def test_reference_arm_batch_config():
+    d = _run(["--impl", "reference", "--config", "aqsol-b128-drop20", "--steps", "2", "--warmup", "1"], 600)
+    assert KEYS <= set(d) and d["impl"] == "reference" and d["value"] > 0
+    assert "aqsol-b128-drop20" in d["config"]["workload"]
+
+
+@pytest.mark.gpu
+def test_gpu_arm_batch_cuda_graph():
+    d = _run(["--config", "zinc-b64", "--steps", "5", "--warmup", "3", "--cuda-graph", "--cpu-seconds", "1"], 900)
+    assert KEYS <= set(d) and d["value"] > 0 and d["gpu_launches"] > 0
+    c = d["config"]
+    assert c["cuda_graph"] is True and c["batch"] == "zinc" and c["num_graphs"] == 64
+    assert c["l2"].startswith("L2 flushed")
