@@ -138,20 +138,22 @@ def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
 
 # ------------------------------------------------------------------ workload
 def block_rows_for(cfg, dtype, block_rows=-1, l2_bytes=None):
-    """-1 -> auto: 0.4 of the device L2 in gathered rows (D * bytes per element)."""
+    """-1 -> auto: 0.4 of the device L2 in gathered rows (D * bytes per element; R24,
+    the rule of mega.auto_block_rows).  Pure arithmetic: the reference arm uses it too."""
     if block_rows >= 0:
         return block_rows
-    from paper_conf_icdcs_dengr24_b200 import mega as M
     if l2_bytes is None:
+        l2_bytes = 126 * 1024 * 1024
         try:
             import torch
-            l2_bytes = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
+            if torch.cuda.is_available():
+                l2_bytes = torch.cuda.get_device_properties(torch.cuda.current_device()).L2_cache_size
         except Exception:  # noqa: BLE001 - no device: the B200 figure
-            l2_bytes = 126 * 1024 * 1024
-    return M.auto_block_rows(cfg.dim * (2 if dtype == "bf16" else 4), l2_bytes)
+            pass
+    return max(1, int(0.4 * l2_bytes) // max(1, cfg.dim * (2 if dtype == "bf16" else 4)))
 
 
-def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1, graph_only=False):
+def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=0, block_rows=-1):
     import synth
     cfg = synth.get_config(cfg_name)
     block_rows = block_rows_for(cfg, dtype, block_rows)
@@ -164,9 +166,6 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=
                                block_rows=block_rows)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
-    if graph_only:  # the CPU reference arm needs the graph and its layout only
-        return {"cfg": cfg, "indptr": indptr, "indices": indices, "layout": layout, "perm": perm,
-                "gen_s": t_gen, "pre_s": t_pre, "graph_stats": gstats}
     layers = []
     in_dim = cfg.f_in
     for li in range(cfg.layers):
@@ -236,61 +235,84 @@ class Model:
 
 
 # ------------------------------------------------------------------ CPU oracle
-def cpu_sample(wl, seconds_target, H, F):
-    """Bounded sample for the CPU oracle: the first R destination rows of the MEGA
-    order with all their in-edges, one GAT layer fwd+bwd.  The sample is compacted to
-    the nodes it touches (its rows and their sources), so the oracle's per-call O(n)
-    work (fp64 copies of n-row arrays) does not swamp the per-edge work being timed."""
+def cpu_sample(cfg, indptr, indices, seconds_target):
+    """Bounded sample of the workload for the CPU oracle (oracle/ only; no libmega.so):
+    the first R destination rows of the INPUT order (mega-synth permutes ids at random,
+    so this is a uniform sample of destinations) with all their in-edges, compacted to
+    the nodes they touch, run through every layer of the config as one step: projection
+    (oracle.gat.project_forward), attention forward and backward (oracle/c, fp64, OpenMP)
+    and projection backward, with the config's layer widths.  Returns (run, R, describe)
+    where run(R) -> (seconds, sample edges)."""
     from oracle import coracle
+    from oracle import gat as og
     import synth
-    ip = wl["layout"].view(0)
-    indptr_new = ip["indptr"].astype(np.int64)
-    src_new = ip["src"]
-    n = len(indptr_new) - 1
+    indptr = np.asarray(indptr, np.int64)
+    indices = np.asarray(indices)
+    n = len(indptr) - 1
+    H, F, D = cfg.heads, cfg.head_dim, cfg.dim
     rng = np.random.default_rng(0)
+    widths = [cfg.f_in_pad] + [D] * (cfg.layers - 1)
+    ws = [synth.bf16_round(rng.uniform(-0.05, 0.05, (k, D)).astype(np.float32)) for k in widths]
     a_l = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
     a_r = (rng.standard_normal((H, F)) / np.sqrt(F)).astype(np.float32)
-    base_wh = synth.bf16_round(rng.standard_normal((4096, H, F)).astype(np.float32))
-    base_g = synth.bf16_round(rng.standard_normal((4096, H, F)).astype(np.float32))
+    base_x = synth.bf16_round(rng.standard_normal((4096, max(widths))).astype(np.float32))
+    base_g = synth.bf16_round(rng.standard_normal((4096, D)).astype(np.float32))
 
-    def run(R):
-        e = int(indptr_new[R])
-        nodes, inv = np.unique(np.concatenate([np.arange(R, dtype=np.int64), src_new[:e].astype(np.int64)]),
+    def sub(R):
+        e = int(indptr[R])
+        nodes, inv = np.unique(np.concatenate([np.arange(R, dtype=np.int64), indices[:e].astype(np.int64)]),
                                return_inverse=True)   # ids 0..R-1 keep their positions
         k = len(nodes)
-        ptr = np.concatenate([indptr_new[:R + 1], np.full(k - R, e, np.int64)])
-        idx = inv[R:].astype(np.int32)
-        Wh, g = base_wh[nodes & 4095], base_g[nodes & 4095]   # values do not change the work
+        ptr = np.concatenate([indptr[:R + 1], np.full(k - R, e, np.int64)])
+        return ptr, inv[R:].astype(np.int32), nodes, e
+
+    def run(R):
+        ptr, idx, nodes, e = sub(R)
+        k = len(nodes)
+        g = base_g[nodes & 4095].reshape(k, H, F)     # values do not change the work
+        Wh = base_g[nodes & 4095].copy()              # rows of sources outside the sample (values only)
         t0 = time.perf_counter()
-        f = coracle.gat_forward(ptr, idx, Wh, a_l, a_r)
-        coracle.gat_backward(ptr, idx, Wh, a_l, a_r, g, fwd=f)
+        for li, w in enumerate(ws):
+            # the sample owns its R destination rows: their projection (fwd and bwd) is its share of the
+            # layer's dense work, so GEMM work per edge matches the full workload (N/E rows per edge)
+            x = base_x[nodes[:R] & 4095, :w.shape[0]]
+            Wh[:R] = og.project_forward(x, w)
+            f = coracle.gat_forward(ptr, idx, Wh.reshape(k, H, F), a_l, a_r)
+            b = coracle.gat_backward(ptr, idx, Wh.reshape(k, H, F), a_l, a_r, g, fwd=f)
+            og.project_backward(x, w, b["grad_feat"].reshape(k, D)[:R])
         return time.perf_counter() - t0, e
 
-    # host-memory bound: the oracle holds ~6 fp64 [k, H, F] arrays for the k touched nodes
-    try:
+    try:   # host-memory bound: ~8 fp64 [k, D] arrays for the k touched nodes
         import psutil
         cap = 0.4 * psutil.virtual_memory().available
     except Exception:  # pragma: no cover
         cap = 16e9
 
     def fits(R):
-        k = len(np.unique(np.concatenate([np.arange(R, dtype=np.int64), src_new[:indptr_new[R]]])))
-        return k * H * F * 8 * 6 + 32 * int(indptr_new[R]) <= cap
+        k = len(np.unique(np.concatenate([np.arange(R, dtype=np.int64), indices[:indptr[R]]])))
+        return k * D * 8 * 8 + 32 * int(indptr[R]) <= cap
 
-    R = max(1, min(n, int(np.searchsorted(indptr_new, 200000))))
+    R = max(1, min(n, int(np.searchsorted(indptr, 50000))))
     t, e = run(R)
     for _ in range(3):
         if t >= seconds_target / 2 or R >= n:
             break
         e_want = int(e * seconds_target / max(t, 1e-3))
-        R2 = max(R + 1, min(n, int(np.searchsorted(indptr_new, min(wl["cfg"].m, e_want)))))
+        R2 = max(R + 1, min(n, int(np.searchsorted(indptr, min(len(indices), e_want)))))
         while R2 > R + 1 and not fits(R2):
             R2 = R + (R2 - R) // 2
         if R2 <= R + 1 and not fits(R2):
             break
         R = R2
         t, e = run(R)
-    return run, R
+
+    def describe(R, e, t=None):
+        return (f"oracle/ fp64 (oracle/c OpenMP attention + numpy projection), one step of all {cfg.layers} "
+                f"layers (projection fwd, GAT fwd+bwd, projection bwd; H={H}, F={F}) over the first {R} "
+                f"destination rows of the input order and their {e} in-edges, compacted to the nodes they touch; "
+                f"the projection runs on the sample's own R rows"
+                + ("" if t is None else f"; {t:.1f} s"))
+    return run, R, describe
 
 
 def cores():
@@ -301,14 +323,27 @@ def cores():
 
 
 # ------------------------------------------------------------------ main paths
+def workload_config(cfg, args, block_rows, flush_note):
+    """The `config` object of the JSON line, shared by both arms."""
+    return {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m, "layers": cfg.layers,
+            "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in, "order": args.order,
+            "block_rows": block_rows,
+            "value_definition": "layers * E / step time (each layer's edges fwd+bwd; max over ranks)",
+            "l2": flush_note,
+            **({"batch": cfg.batch, "num_graphs": cfg.num_graphs, "edge_drop": cfg.drop} if cfg.batch else {})}
+
+
 def run_reference(args):
+    """--impl reference: the CPU oracle (oracle/, never libmega.so) timed on this box's
+    host cores, on bounded samples of the same workload; rank 0 only."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
-    wl = build_workload(args.config, args.dtype, args.order, block_rows=args.block_rows, graph_only=True)
-    cfg = wl["cfg"]
+    import synth
+    cfg = synth.get_config(args.config)
+    indptr, indices, _ = synth.make_graph(cfg)
     per_step = max(2.0, min(10.0, 150.0 / max(1, args.steps + args.warmup)))
-    run, R = cpu_sample(wl, per_step, cfg.heads, cfg.head_dim)
+    run, R, describe = cpu_sample(cfg, indptr, indices, per_step)
     for _ in range(args.warmup):
         run(R)
     times, edges = [], 0
@@ -317,13 +352,14 @@ def run_reference(args):
         times.append(t)
         edges = e
     tot = float(np.sum(times))
-    value = edges * args.steps / tot
-    sample = (f"oracle/c fp64 GAT fwd+bwd (one layer, H={cfg.heads}, F={cfg.head_dim}) over the first {R} "
-              f"destination rows of the MEGA order ({edges} edges; compacted to the nodes it touches)")
+    value = cfg.layers * edges * args.steps / tot
+    sample = describe(R, edges)
+    conf = workload_config(cfg, args, block_rows_for(cfg, args.dtype, args.block_rows), "host memory (no device)")
+    conf.update({"parallelism": "host cores (oracle)", "sample": sample})
     line = {"impl": "reference", "metric": METRIC, "value": value, "unit": "edges/s", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * tot / args.steps,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic (mega-synth v1)", "config": {"workload": f"{cfg.name}-shaped sample", "sample": sample},
+            "data": "synthetic (mega-synth v1, seeded; random-init weights)", "config": conf,
             "cpu_baseline": {"value": value, "unit": "edges/s", "cores": cores(), "kind": "oracle", "sample": sample},
             "e2e": {"value": value, "unit": "edges/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -481,11 +517,10 @@ def run_mega(args):
     # ---- CPU oracle baseline (bounded sample; rank 0 at N = 1 only) ----
     cpu = None
     if not args.no_cpu_baseline and world == 1:
-        run, R = cpu_sample(wl, args.cpu_seconds, cfg.heads, cfg.head_dim)
+        run, R, describe = cpu_sample(cfg, wl["indptr"], wl["indices"], args.cpu_seconds)
         t, e = run(R)
-        cpu = {"value": e / t, "unit": "edges/s", "cores": cores(), "kind": "oracle",
-               "sample": f"oracle/c fp64 one-layer GAT fwd+bwd over the first {R} destination rows of the MEGA "
-                         f"order ({e} edges; the sample is compacted to the nodes it touches); {t:.1f} s"}
+        cpu = {"value": cfg.layers * e / t, "unit": "edges/s", "cores": cores(), "kind": "oracle",
+               "sample": describe(R, e, t)}
     if rank == 0:
         st = wl["layout"].stats()
         line = {
@@ -494,18 +529,13 @@ def run_mega(args):
             "vs_baseline": None, "dtype": args.dtype,
             "data": ("synthetic (mega-synth v1: Table II-shaped block-diagonal batch, seeded; random-init weights)"
                      if cfg.batch else "synthetic (mega-synth v1: DC-SBM power-law graph, seeded; random-init weights)"),
-            "config": {"workload": f"{cfg.name}-shaped synthetic GAT", "nodes": cfg.n, "edges": cfg.m,
-                       "layers": cfg.layers, "heads": cfg.heads, "head_dim": cfg.head_dim, "f_in": cfg.f_in,
-                       "order": args.order, "block_rows": st["block_rows"],
+            "config": {**workload_config(cfg, args, st["block_rows"],
+                                         "no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)
+                                         if flush is None else "L2 flushed between timed steps (%d MB write, "
+                                         "outside the events)" % (flush.numel() * 4 >> 20)),
                        "parallelism": "single GPU" if world == 1 else
                        f"dst-partitioned x{world} (NCCL all-gather-v of [Wh|er], reduce-to-owner of [dWh|der])",
-                       "value_definition": "layers * E / step time (each layer's edges fwd+bwd; max over ranks)",
-                       "l2": ("no flush: inputs larger than L2 (Wh %.2f GB)" % (cfg.n * cfg.dim * sb / 1e9)
-                              if flush is None else "L2 flushed between timed steps (%d MB write, outside the "
-                              "events)" % (flush.numel() * 4 >> 20)),
-                       "cuda_graph": graph is not None,
-                       **({"batch": cfg.batch, "num_graphs": cfg.num_graphs, "edge_drop": cfg.drop}
-                          if cfg.batch else {})},
+                       "cuda_graph": graph is not None},
             "roofline": roofline, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": model.launches * args.steps,
             "clocks": clk.summary(), "calls_ms_per_step": per_step_calls,
             "layout": {k: st[k] for k in ("window", "seg_edges", "path_length", "revisits", "jumps",

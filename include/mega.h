@@ -1,7 +1,7 @@
 /*
  * mega.h — C ABI of libmega.so, the B200-native hot path of MEGA
  * (Deng & Rao, "MEGA: More Efficient Graph Attention for GNNs", ICDCS'24).
- * ABI version 1.  C linkage; plain pointers and sizes; no C++ or torch types.
+ * ABI version 2.  C linkage; plain pointers and sizes; no C++ or torch types.
  *
  * Citations "PAPER.md:L" are lines of the paper text;
  * DESIGN.md "Rn" are the documented readings of ambiguous passages.
@@ -61,7 +61,7 @@
 extern "C" {
 #endif
 
-#define MEGA_ABI_VERSION 1
+#define MEGA_ABI_VERSION 2 /* 2: projection backward takes a workspace (tcgen05 dW split) */
 
 typedef struct CUstream_st *mega_stream_t; /* == cudaStream_t */
 
@@ -209,15 +209,29 @@ mega_status mega_layout_bind_device(mega_layout *layout, int32_t part, void *dev
 mega_status mega_gat_workspace_bytes(const mega_layout *layout, int32_t part, int heads, int head_dim,
                                      mega_dtype dtype, size_t *fwd_ws, size_t *bwd_ws);
 
-/* a2. Projection (neural operator): feat = x * w on tensor
- * cores (bf16 inputs, fp32 accumulation; MEGA_F32 = true fp32, no TF32),
- * then el/er of every projected row into ctx rows [ctx_row0, ctx_row0+rows).
- *   x    device [rows][ldx] dtype, w device [in_dim][heads*head_dim] dtype,
+/* a2. Projection (neural operator; the "sgemm" the paper finds
+ * efficient): feat = x * w, then el = feat.a_l and er = feat.a_r
+ * of every projected row into ctx rows [ctx_row0, ctx_row0+rows).
+ *   MEGA_BF16: tcgen05 tensor-core GEMM (bf16 operands, fp32 accumulation in
+ *     TMEM, TMA-staged operands); el/er are computed in its epilogue from the
+ *     stored (bf16-rounded) feat.  Requires heads*head_dim a multiple of 64,
+ *     head_dim a multiple of 8 dividing min(heads*head_dim, 256), in_dim, ldx and
+ *     ldf multiples of 8, 16-byte aligned x, w, feat.
+ *   MEGA_F32: true fp32 (no TF32) on CUDA cores (cuBLAS pedantic; the tensor
+ *     cores have no fp32 kind), then an el/er pass.
+ *   x    device [rows][ldx] dtype (columns >= in_dim are ignored),
+ *   w    device [in_dim][heads*head_dim] dtype (dense rows),
  *   feat device [rows][ldf] dtype, ctx device fp32 [MEGA_CTX_PLANES][ctx_n][heads].
  * Errors: INVALID_ARGUMENT, UNSUPPORTED, CUDA. */
 mega_status mega_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
                              int head_dim, const float *attn_l, const float *attn_r, mega_dtype dtype, void *feat,
                              int64_t ldf, float *ctx, int64_t ctx_n, int64_t ctx_row0, mega_stream_t stream);
+
+/* Device workspace (bytes) of mega_project_bwd for this shape: the bf16 dW GEMM
+ * is split over the rows (the reduction dimension) and its fp32 partial tiles
+ * are summed in a fixed order (deterministic).  256 for MEGA_F32. */
+mega_status mega_project_workspace_bytes(int64_t rows, int in_dim, int heads, int head_dim, mega_dtype dtype,
+                                         size_t *bwd_ws);
 
 /* a3-a5. Fused forward over `part`: per-edge score, per-destination online
  * softmax and attention-weighted aggregation, one pass over the edges
@@ -253,13 +267,15 @@ mega_status mega_gat_bwd(const mega_layout *layout, int32_t part, const void *fe
                          int64_t ldlp, float *grad_attn_l, float *grad_attn_r, void *ws, size_t ws_bytes,
                          mega_stream_t stream);
 
-/* a9. Projection backward on tensor cores: grad_w = x^T grad_feat (fp32
- * [in_dim][D], written) and, if grad_x != NULL, grad_x = grad_feat w^T
- * (dtype [rows][ldgx]).  grad_feat is fp32 for MEGA_F32 and the bf16 copy
- * (grad_feat_lp of mega_gat_bwd) for MEGA_BF16.  Errors as mega_project_fwd. */
+/* a9. Projection backward: grad_w = x^T grad_feat (fp32 [in_dim][D], written)
+ * and, if grad_x != NULL, grad_x = grad_feat w^T (dtype [rows][ldgx]).
+ * MEGA_BF16: tcgen05 GEMMs (grad_feat is the bf16 copy, grad_feat_lp of
+ * mega_gat_bwd); the dW partials use `ws` (>= mega_project_workspace_bytes).
+ * MEGA_F32: fp32 on CUDA cores as in mega_project_fwd (ws unused).
+ * Errors as mega_project_fwd, plus OUT_OF_MEMORY (workspace too small). */
 mega_status mega_project_bwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
                              int head_dim, mega_dtype dtype, const void *grad_feat, int64_t ldgf, void *grad_x,
-                             int64_t ldgx, float *grad_w, mega_stream_t stream);
+                             int64_t ldgx, float *grad_w, void *ws, size_t ws_bytes, mega_stream_t stream);
 
 /* NEXT-3: Graph Transformer edge attention, the paper's
  * headline model (Table I; DESIGN.md R-gt), over the same layout:

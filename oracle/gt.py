@@ -1,5 +1,6 @@
 """Graph Transformer attention over a graph, fp64, per edge — the plain definition
-(oracle only, the CUDA kernel is not built yet).
+(SURVEY.md §8(f) NEXT-3).  The CUDA path it checks is csrc/gt_kernels.cu
+(mega_gt_fwd / mega_gt_bwd), compared against this file in tests/test_gpu_gt.py.
 
 Test infrastructure only (see oracle/__init__.py).
 

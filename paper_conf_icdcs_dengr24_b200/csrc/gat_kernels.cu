@@ -2037,8 +2037,9 @@ int ring_blocks(size_t smem) {
 mega_status check_launch(cudaStream_t s, const char *what) {
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
-  if (debug_sync()) {
-    e = cudaStreamSynchronize(s);
+  cudaStreamCaptureStatus cap = cudaStreamCaptureStatusNone;
+  if (debug_sync() && cudaStreamIsCapturing(s, &cap) == cudaSuccess && cap == cudaStreamCaptureStatusNone) {
+    e = cudaStreamSynchronize(s);  // never inside a CUDA-graph capture (illegal there)
     if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + " (sync): " + cudaGetErrorString(e));
   }
   return MEGA_OK;

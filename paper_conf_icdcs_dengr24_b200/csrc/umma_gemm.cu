@@ -1,0 +1,487 @@
+// a2 / a9: the dense node projection and its backward on the 5th-generation
+// tensor cores — the one real contraction of the path (north_star: tensor
+// cores only here; PAPER.md:55 neural operator, PAPER.md:142 sgemm).
+//
+//   fwd  Wh[N,D] = X[N,K] W[K,D]           + epilogue el = Wh.a_l, er = Wh.a_r (per head)
+//   dX   dX[N,K] = dWh[N,D] W^T
+//   dW   dW[K,D] = X^T dWh                  (split over N, fixed-order reduction)
+//
+// One CTA computes a 128 x BN output tile with tcgen05.mma (kind::f16: bf16
+// operands, fp32 accumulator in TMEM), operands staged in shared memory by TMA
+// (cp.async.bulk.tensor, 128-byte swizzle) through an mbarrier ring of STAGES
+// slots.  128 threads: lane 0 of warp 0 is the TMA producer, lane 0 of warp 1
+// issues the MMAs (one thread per CTA, as tcgen05 requires); then all four
+// warps drain TMEM with tcgen05.ld (warp w owns TMEM lanes = tile rows
+// 32w..32w+31, one row per thread) for the epilogue.  Several CTAs share an SM
+// (<= 256 TMEM columns and ~100 KB of shared memory each), so one CTA's
+// epilogue overlaps another's main loop.
+//
+// Operand majors (UMMA descriptors, SWIZZLE_128B canonical layouts):
+//   fwd: A = X   K-major (rows of X contiguous in K),  B = W   MN-major (W[k][n], n contiguous)
+//   dX : A = dWh K-major,                              B = W   K-major  (W[n=k_in][k=d])
+//   dW : A = X   MN-major (X[k=row][m=k_in]),          B = dWh MN-major (dWh[k=row][n=d])
+// K-major SW128 atom: 8 rows x 128 B (64 bf16 of K), 8-row groups 1024 B apart
+// (SBO); the k-th UMMA_K = 16 slice starts 32 B further.  MN-major SW128 atom:
+// 8 k-rows x 128 B (64 bf16 of M/N); 64-wide M/N groups LBO apart (one TMA
+// box = 64 k-rows x 128 B = 8 KB), 8-k-row groups 1024 B apart (SBO); the
+// k-th UMMA_K slice starts 16 rows x 128 B = 2 KB further.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstring>
+#include <mutex>
+
+#include "mega_internal.h"
+
+namespace mega {
+namespace umma {
+
+constexpr int BM = 128, BK = 64, THREADS = 128;
+enum Mode { FWD = 0, DX = 1, DW = 2 };
+
+struct Args {
+  int64_t M;        // output rows (fwd/dX: N; dW: K_in)
+  int Nc;           // output columns (fwd: D; dX: K_in; dW: D)
+  int64_t kb_total; // 64-wide K blocks of the whole reduction
+  int64_t kb_split; // K blocks per CTA along z (dW split; else = kb_total)
+  void *out;        // fwd / dX: bf16 [M][ldo]; dW: fp32 partials [z][Mpad][Nc]
+  int64_t ldo;
+  int64_t mpad;     // dW: rows per partial slab
+  // fwd epilogue: el/er into the ctx planes
+  float *el, *er;
+  const float *al, *ar;
+  int H, F;
+  int64_t ctx_row0;
+};
+
+// ------------------------------------------------------------------ PTX helpers
+__device__ __forceinline__ uint32_t smem_u32(const void *p) { return (uint32_t)__cvta_generic_to_shared(p); }
+
+__device__ __forceinline__ void mbar_init(uint32_t bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(bar), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_expect_tx(uint32_t bar, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t bar, uint32_t parity) {
+  asm volatile(
+      "{\n"
+      ".reg .pred P1;\n"
+      "WAIT_%=:\n"
+      "mbarrier.try_wait.parity.shared::cta.b64 P1, [%0], %1;\n"
+      "@P1 bra DONE_%=;\n"
+      "bra WAIT_%=;\n"
+      "DONE_%=:\n"
+      "}\n" ::"r"(bar),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map, int32_t x, int32_t y, uint32_t bar) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
+      "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(bar)
+      : "memory");
+}
+__device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
+  asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
+}
+// shared-memory matrix descriptor, SWIZZLE_128B, sm_100 version bits
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t sbo) {
+  return (uint64_t)((saddr >> 4) & 0x3FFFu) | ((uint64_t)((lbo >> 4) & 0x3FFFu) << 16) |
+         ((uint64_t)((sbo >> 4) & 0x3FFFu) << 32) | ((uint64_t)1 << 46) | ((uint64_t)2 << 61);
+}
+__device__ __forceinline__ void umma_f16(uint32_t tmem_d, uint64_t a, uint64_t b, uint32_t idesc, uint32_t accum) {
+  asm volatile(
+      "{\n"
+      ".reg .pred p;\n"
+      "setp.ne.b32 p, %4, 0;\n"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n"
+      "}\n" ::"r"(tmem_d),
+      "l"(a), "l"(b), "r"(idesc), "r"(accum)
+      : "memory");
+}
+__device__ __forceinline__ void umma_commit(uint32_t bar) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
+__device__ __forceinline__ void tc_fence_after() { asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory"); }
+
+// 32 consecutive fp32 TMEM columns of this thread's lane
+__device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
+      "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]), "=r"(r[8]),
+        "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]), "=r"(r[15]), "=r"(r[16]),
+        "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]),
+        "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(taddr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+__device__ __forceinline__ uint32_t bf2(float a, float b) {
+  __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
+  return *reinterpret_cast<uint32_t *>(&t);
+}
+
+template <int BN> struct Tiles {
+  static constexpr int A_BYTES = BM * BK * 2;          // 16 KB
+  static constexpr int B_BYTES = BN * BK * 2;
+  static constexpr int STAGE = A_BYTES + B_BYTES;
+  static constexpr int STAGES = STAGE >= 40 * 1024 ? 2 : (STAGE >= 28 * 1024 ? 3 : 4);
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + 256 + 2 * BN * 4;
+};
+
+// MODE: FWD/DX/DW.  BN: tile columns (<= 256, multiple of 16; a multiple of 64
+// when B is MN-major).  FH: fwd only, min(head_dim, 32) (heads per 32-column chunk).
+template <int MODE, int BN, int FH>
+__global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constant__ CUtensorMap tmA,
+                                                            const __grid_constant__ CUtensorMap tmB, const Args g) {
+  using TL = Tiles<BN>;
+  constexpr int STAGES = TL::STAGES;
+  constexpr bool A_MN = MODE == DW, B_MN = MODE != DX;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  uint64_t *bars = reinterpret_cast<uint64_t *>(smem + STAGES * TL::STAGE);   // full[S], empty[S], done
+  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 1);
+  float *s_al = reinterpret_cast<float *>(smem + STAGES * TL::STAGE + 256);
+  float *s_ar = s_al + BN;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t m0 = (int64_t)blockIdx.x * BM;
+  const int n0 = blockIdx.y * BN;
+  const int64_t kb0 = (int64_t)blockIdx.z * g.kb_split;
+  const int64_t kb1 = g.kb_total < kb0 + g.kb_split ? g.kb_total : kb0 + g.kb_split;
+  const int nkb = kb1 > kb0 ? (int)(kb1 - kb0) : 0;
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES), done = smem_u32(bars + 2 * STAGES);
+
+  if (MODE == FWD) {
+    for (int c = threadIdx.x; c < BN; c += THREADS) {
+      const bool ok = n0 + c < g.Nc;
+      s_al[c] = ok ? g.al[n0 + c] : 0.f;
+      s_ar[c] = ok ? g.ar[n0 + c] : 0.f;
+    }
+  }
+  if (warp == 0) {
+    if (lane == 0) {
+      prefetch_tmap(&tmA);
+      prefetch_tmap(&tmB);
+      for (int s = 0; s < STAGES; ++s) {
+        mbar_init(full0 + 8 * s, 1);
+        mbar_init(empty0 + 8 * s, 1);
+      }
+      mbar_init(done, 1);
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+    }
+    __syncwarp();
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)),
+                 "r"((uint32_t)TL::TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0 && lane == 0) {
+    // ---- TMA producer ----
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % STAGES;
+      const uint32_t ph = (uint32_t)(i / STAGES) & 1u;
+      mbar_wait(empty0 + 8 * s, ph ^ 1u);
+      const uint32_t full = full0 + 8 * s;
+      mbar_expect_tx(full, TL::STAGE);
+      const uint32_t sa = smem_u32(smem + s * TL::STAGE), sb = sa + TL::A_BYTES;
+      const int32_t k = (int32_t)((kb0 + i) * BK);
+      if constexpr (A_MN) {          // dW: X[row = k][k_in = m], two 64-wide m boxes
+        tma_load_2d(sa, &tmA, (int32_t)m0, k, full);
+        tma_load_2d(sa + 8192, &tmA, (int32_t)m0 + 64, k, full);
+      } else {                        // K-major A: one 128-row box of 64 K
+        tma_load_2d(sa, &tmA, k, (int32_t)m0, full);
+      }
+      if constexpr (B_MN) {          // B[k][n]: BN/64 boxes of 64 k-rows x 64 n
+#pragma unroll
+        for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * 8192, &tmB, n0 + 64 * j, k, full);
+      } else {                        // K-major B: one BN-row box of 64 K
+        tma_load_2d(sb, &tmB, k, n0, full);
+      }
+    }
+  } else if (warp == 1 && lane == 0) {
+    // ---- MMA issuer (one thread) ----
+    constexpr uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((A_MN ? 1u : 0u) << 15) |
+                               ((B_MN ? 1u : 0u) << 16) | ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+    for (int i = 0; i < nkb; ++i) {
+      const int s = i % STAGES;
+      const uint32_t ph = (uint32_t)(i / STAGES) & 1u;
+      mbar_wait(full0 + 8 * s, ph);
+      tc_fence_after();
+      const uint32_t sa = smem_u32(smem + s * TL::STAGE), sb = sa + TL::A_BYTES;
+#pragma unroll
+      for (int kk = 0; kk < BK / 16; ++kk) {
+        const uint64_t da = A_MN ? sdesc(sa + kk * 2048, 8192, 1024) : sdesc(sa + kk * 32, 16, 1024);
+        const uint64_t db = B_MN ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
+        umma_f16(tmem, da, db, idesc, (i | kk) ? 1u : 0u);
+      }
+      umma_commit(empty0 + 8 * s);   // frees the slot once these MMAs have read it
+    }
+    umma_commit(done);                // accumulator complete
+  }
+  __syncwarp();
+
+  // ---- epilogue: TMEM -> registers -> global ----
+  if (nkb > 0) mbar_wait(done, 0);
+  tc_fence_after();
+  const int row = warp * 32 + lane;
+  const int64_t grow = m0 + row;
+  const uint32_t taddr = tmem + ((uint32_t)(warp * 32) << 16);
+  if constexpr (MODE == DW) {
+    float *dst = static_cast<float *>(g.out) + ((int64_t)blockIdx.z * g.mpad + grow) * g.Nc + n0;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 32) {
+      uint32_t r[32];
+      if (nkb > 0) tmem_ld32(taddr + c0, r);
+      else
+#pragma unroll
+        for (int q = 0; q < 32; ++q) r[q] = 0u;
+#pragma unroll
+      for (int q = 0; q < 8; ++q)
+        *reinterpret_cast<uint4 *>(dst + c0 + 4 * q) = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+    }
+  } else {
+    __nv_bfloat16 *orow = static_cast<__nv_bfloat16 *>(g.out) + grow * g.ldo + n0;
+    const bool live = grow < g.M;
+    float el_acc = 0.f, er_acc = 0.f;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 32) {
+      uint32_t r[32];
+      tmem_ld32(taddr + c0, r);
+      uint32_t p[16];
+#pragma unroll
+      for (int q = 0; q < 16; ++q) p[q] = bf2(__uint_as_float(r[2 * q]), __uint_as_float(r[2 * q + 1]));
+      if (live) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+          if (MODE == FWD || n0 + c0 + 8 * q < g.Nc)
+            *reinterpret_cast<uint4 *>(orow + c0 + 8 * q) = make_uint4(p[4 * q], p[4 * q + 1], p[4 * q + 2], p[4 * q + 3]);
+      }
+      if constexpr (MODE == FWD) {
+        // el/er from the STORED (bf16-rounded) Wh, head by head (FH values per head segment)
+#pragma unroll
+        for (int sgm = 0; sgm < 32 / FH; ++sgm) {
+#pragma unroll
+          for (int q = 0; q < FH; q += 2) {
+            const uint32_t w2 = p[(sgm * FH + q) / 2];
+            const float x0 = __uint_as_float(w2 << 16), x1 = __uint_as_float(w2 & 0xffff0000u);
+            const int c = c0 + sgm * FH + q;
+            el_acc = fmaf(s_al[c], x0, el_acc);
+            el_acc = fmaf(s_al[c + 1], x1, el_acc);
+            er_acc = fmaf(s_ar[c], x0, er_acc);
+            er_acc = fmaf(s_ar[c + 1], x1, er_acc);
+          }
+          const int cend = c0 + (sgm + 1) * FH;       // columns of this tile consumed so far
+          if (cend % g.F == 0) {                       // a head is complete
+            const int h = (n0 + cend) / g.F - 1;
+            if (live && n0 + cend <= g.Nc) {
+              g.el[(g.ctx_row0 + grow) * g.H + h] = el_acc;
+              g.er[(g.ctx_row0 + grow) * g.H + h] = er_acc;
+            }
+            el_acc = 0.f;
+            er_acc = 0.f;
+          }
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 0) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)TL::TMEM_COLS)
+                 : "memory");
+  }
+}
+
+// dW: fixed-order sum of the split partials (deterministic), fp32
+__global__ void __launch_bounds__(256) dw_reduce_kernel(const float *parts, int splits, int64_t mpad, int K, int D,
+                                                        float *out) {
+  const int64_t n4 = (int64_t)K * D / 4;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t e = 4 * i;
+    const int64_t k = e / D, d = e % D;
+    float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int z = 0; z < splits; ++z) {
+      const float4 v = *reinterpret_cast<const float4 *>(parts + ((int64_t)z * mpad + k) * D + d);
+      s.x += v.x; s.y += v.y; s.z += v.z; s.w += v.w;
+    }
+    *reinterpret_cast<float4 *>(out + e) = s;
+  }
+}
+
+// ------------------------------------------------------------------ host side
+PFN_cuTensorMapEncodeTiled_v12000 encoder() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    void *p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+// 2-D bf16 tensor map: `inner` contiguous elements per row, `outer` rows `ld` elements apart,
+// box {box_inner (<= 64: 128 B), box_outer}, 128-byte swizzle, zero fill out of bounds
+mega_status tmap_2d(CUtensorMap *m, const void *base, uint64_t inner, uint64_t outer, int64_t ld, uint32_t box_inner,
+                    uint32_t box_outer) {
+  auto enc = encoder();
+  if (!enc) return fail(MEGA_ERR_CUDA, "cuTensorMapEncodeTiled unavailable (driver entry point)");
+  const cuuint64_t dims[2] = {inner, outer};
+  const cuuint64_t strides[1] = {(cuuint64_t)ld * 2};
+  const cuuint32_t box[2] = {box_inner, box_outer};
+  const cuuint32_t es[2] = {1, 1};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void *>(base), dims, strides, box, es,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                   CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) return fail(MEGA_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return MEGA_OK;
+}
+
+int sm_count() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+template <int MODE, int BN, int FH>
+mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const Args &g, dim3 grid, cudaStream_t st) {
+  auto k = umma_gemm_kernel<MODE, BN, FH>;
+  const size_t smem = Tiles<BN>::SMEM;
+  static bool attr = false;  // per instantiation
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma smem attribute: ") + cudaGetErrorString(e));
+    attr = true;
+  }
+  k<<<grid, THREADS, smem, st>>>(a, b, g);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma_gemm_kernel: ") + cudaGetErrorString(e));
+  return MEGA_OK;
+}
+
+}  // namespace umma
+
+using namespace umma;
+
+// Wh = X W (+ el/er of each head into the ctx planes).  bf16.  D <= 256 per tile:
+// BN = min(D, 256) must be a multiple of head_dim (so a tile holds whole heads) and of 64.
+mega_status umma_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
+                             int head_dim, const float *al, const float *ar, void *feat, int64_t ldf, float *el,
+                             float *er, int64_t ctx_row0, cudaStream_t st) {
+  const int D = heads * head_dim;
+  const int BN = std::min(D, 256);
+  if (D % 64 || BN % head_dim || head_dim % 8)
+    return fail(MEGA_ERR_UNSUPPORTED, "tcgen05 projection: D must be a multiple of 64 and head_dim divide min(D, 256)");
+  CUtensorMap ta, tb;
+  mega_status rc;
+  if ((rc = tmap_2d(&ta, x, (uint64_t)in_dim, (uint64_t)rows, ldx, 64, BM)) != MEGA_OK) return rc;
+  if ((rc = tmap_2d(&tb, w, (uint64_t)D, (uint64_t)in_dim, D, 64, 64)) != MEGA_OK) return rc;
+  Args g{};
+  g.M = rows; g.Nc = D; g.kb_total = (in_dim + BK - 1) / BK; g.kb_split = g.kb_total;
+  g.out = feat; g.ldo = ldf; g.el = el; g.er = er; g.al = al; g.ar = ar; g.H = heads; g.F = head_dim;
+  g.ctx_row0 = ctx_row0;
+  const dim3 grid((unsigned)((rows + BM - 1) / BM), (unsigned)(D / BN), 1);
+  const int fh = std::min(head_dim, 32);
+  if (BN == 256) {
+    if (fh == 32) return launch<FWD, 256, 32>(ta, tb, g, grid, st);
+    if (fh == 16) return launch<FWD, 256, 16>(ta, tb, g, grid, st);
+    return launch<FWD, 256, 8>(ta, tb, g, grid, st);
+  }
+  if (BN == 128) {
+    if (fh == 32) return launch<FWD, 128, 32>(ta, tb, g, grid, st);
+    if (fh == 16) return launch<FWD, 128, 16>(ta, tb, g, grid, st);
+    return launch<FWD, 128, 8>(ta, tb, g, grid, st);
+  }
+  if (BN == 192) {
+    if (fh == 32) return launch<FWD, 192, 32>(ta, tb, g, grid, st);
+    if (fh == 16) return launch<FWD, 192, 16>(ta, tb, g, grid, st);
+    return launch<FWD, 192, 8>(ta, tb, g, grid, st);
+  }
+  if (fh == 32) return launch<FWD, 64, 32>(ta, tb, g, grid, st);
+  if (fh == 16) return launch<FWD, 64, 16>(ta, tb, g, grid, st);
+  return launch<FWD, 64, 8>(ta, tb, g, grid, st);
+}
+
+// dX[rows][in_dim] = dWh W^T (bf16 out).  K = D (multiple of 64).  Columns are written in
+// 8-wide (16-byte) vectors up to round_up(in_dim, 8) (<= ldgx): the ones past in_dim get 0
+// (W rows past in_dim read as zeros), i.e. the zero padding of a padded X.
+mega_status umma_project_dx(const void *gf, int64_t ldgf, int64_t rows, int in_dim, const void *w, int D, void *gx,
+                            int64_t ldgx, cudaStream_t st) {
+  if (D % 64) return fail(MEGA_ERR_UNSUPPORTED, "tcgen05 dX: D % 64 required");
+  const int BN = in_dim >= 256 ? 256 : (in_dim >= 128 ? 128 : 64);
+  CUtensorMap ta, tb;
+  mega_status rc;
+  if ((rc = tmap_2d(&ta, gf, (uint64_t)D, (uint64_t)rows, ldgf, 64, BM)) != MEGA_OK) return rc;
+  if ((rc = tmap_2d(&tb, w, (uint64_t)D, (uint64_t)in_dim, D, 64, BN)) != MEGA_OK) return rc;
+  Args g{};
+  g.M = rows; g.Nc = (in_dim + 7) / 8 * 8; g.kb_total = D / BK; g.kb_split = g.kb_total; g.out = gx; g.ldo = ldgx;
+  const dim3 grid((unsigned)((rows + BM - 1) / BM), (unsigned)((in_dim + BN - 1) / BN), 1);
+  if (BN == 256) return launch<DX, 256, 32>(ta, tb, g, grid, st);
+  if (BN == 128) return launch<DX, 128, 32>(ta, tb, g, grid, st);
+  return launch<DX, 64, 32>(ta, tb, g, grid, st);
+}
+
+// workspace of umma_project_dw: split partials
+void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, size_t &bytes) {
+  const int BN = std::min(D, 256);
+  const int64_t mt = (in_dim + BM - 1) / BM, nt = (D + BN - 1) / BN;
+  const int64_t kbt = (rows + BK - 1) / BK;
+  int64_t s = (2 * (int64_t)sm_count() + mt * nt - 1) / (mt * nt);
+  s = std::max<int64_t>(1, std::min<int64_t>(s, kbt));
+  const int64_t per = (kbt + s - 1) / s;
+  splits = (int)((kbt + per - 1) / per);   // every split non-empty
+  mpad = mt * BM;
+  bytes = (size_t)splits * (size_t)mpad * (size_t)D * 4;
+}
+
+// dW[in_dim][D] = X^T dWh (fp32 out), split over rows, fixed-order reduce.
+mega_status umma_project_dw(const void *x, int64_t ldx, const void *gf, int64_t ldgf, int64_t rows, int in_dim, int D,
+                            float *gw, void *ws, size_t ws_bytes, cudaStream_t st) {
+  if (D % 64) return fail(MEGA_ERR_UNSUPPORTED, "tcgen05 dW: D % 64 required");
+  int splits;
+  int64_t mpad;
+  size_t need;
+  umma_dw_plan(rows, in_dim, D, splits, mpad, need);
+  if (ws_bytes < need) return fail(MEGA_ERR_OUT_OF_MEMORY, "projection workspace too small (mega_project_workspace_bytes)");
+  const int BN = std::min(D, 256);
+  CUtensorMap ta, tb;
+  mega_status rc;
+  if ((rc = tmap_2d(&ta, x, (uint64_t)in_dim, (uint64_t)rows, ldx, 64, 64)) != MEGA_OK) return rc;
+  if ((rc = tmap_2d(&tb, gf, (uint64_t)D, (uint64_t)rows, ldgf, 64, 64)) != MEGA_OK) return rc;
+  Args g{};
+  g.M = mpad; g.Nc = D; g.kb_total = (rows + BK - 1) / BK; g.kb_split = (g.kb_total + splits - 1) / splits;
+  g.out = ws; g.mpad = mpad;
+  const dim3 grid((unsigned)(mpad / BM), (unsigned)(D / BN), (unsigned)splits);
+  if (BN == 256) rc = launch<DW, 256, 32>(ta, tb, g, grid, st);
+  else if (BN == 128) rc = launch<DW, 128, 32>(ta, tb, g, grid, st);
+  else if (BN == 192) rc = launch<DW, 192, 32>(ta, tb, g, grid, st);
+  else rc = launch<DW, 64, 32>(ta, tb, g, grid, st);
+  if (rc != MEGA_OK) return rc;
+  const int64_t n4 = (int64_t)in_dim * D / 4;
+  const int blocks = (int)std::min<int64_t>((n4 + 255) / 256, 4 * sm_count());
+  dw_reduce_kernel<<<std::max(blocks, 1), 256, 0, st>>>(static_cast<const float *>(ws), splits, mpad, in_dim, D, gw);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("dw_reduce_kernel: ") + cudaGetErrorString(e));
+  return MEGA_OK;
+}
+
+}  // namespace mega

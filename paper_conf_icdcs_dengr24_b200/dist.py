@@ -42,10 +42,11 @@ def allgather_rows(t: torch.Tensor, bounds, group=None):
     for q in range(world):
         if q == rank:
             continue
+        peer = dist.get_global_rank(group, q) if group is not None else q   # P2P ops take global ranks
         if b[rank + 1] > b[rank]:
-            ops.append(dist.P2POp(dist.isend, mine, q, group))
+            ops.append(dist.P2POp(dist.isend, mine, peer, group))
         if b[q + 1] > b[q]:
-            ops.append(dist.P2POp(dist.irecv, t[b[q]:b[q + 1]], q, group))
+            ops.append(dist.P2POp(dist.irecv, t[b[q]:b[q + 1]], peer, group))
     if ops:
         for r in dist.batch_isend_irecv(ops):
             r.wait()

@@ -42,8 +42,11 @@ class GATLayer:
         self.grad_feat_lp = torch.empty(n, D, dtype=self.dtype, device=dev) if self.dtype == torch.bfloat16 else None
         self.grad_attn_l = torch.empty(D, dtype=torch.float32, device=dev)
         self.grad_attn_r = torch.empty(D, dtype=torch.float32, device=dev)
-        self.grad_w = torch.empty(self.w.shape[0], D, dtype=torch.float32, device=dev)
+        # rows >= in_dim (zero padding of W) are never written by mega_project_bwd: keep them 0
+        self.grad_w = torch.zeros(self.w.shape[0], D, dtype=torch.float32, device=dev)
         self.grad_x = torch.empty_like(self.x) if want_grad_x else None
+        pws = M.mega_project_workspace_bytes(self.x.shape[0], self.in_dim, heads, head_dim, M._dtype_code(x))
+        self.ws_p = torch.empty(max(pws, 256), dtype=torch.uint8, device=dev)
 
     # a2
     def project(self, stream=None):
@@ -70,7 +73,7 @@ class GATLayer:
         gf = self.grad_feat_lp if self.dtype == torch.bfloat16 else self.grad_feat
         rows = slice(self.row_begin, self.row_end) if self.x.shape[0] != self.n else slice(None)
         M.mega_project_bwd(self.x, self.w, self.H, self.F, gf[rows], self.grad_w, self.grad_x,
-                           in_dim=self.in_dim, stream=stream)
+                           in_dim=self.in_dim, ws=self.ws_p, stream=stream)
 
     def forward(self, stream=None):
         self.project(stream)
@@ -86,7 +89,11 @@ class GATLayer:
         self.backward(grad_out, stream)
 
     def launches_per_step(self) -> int:
-        """Our kernels per step (cuBLAS GEMMs excluded): eler, fwd, [fwd merge], dlt, bwd_src,
-        [bwd_src merge], bwd_dst, reduce(a_l, a_r)."""
+        """Our kernels per step.  bf16: projection GEMM (el/er in its epilogue), fwd, [fwd merge], dlt,
+        bwd_src, [bwd_src merge], bwd_dst, reduce(a_l, a_r), dW GEMM + its reduce, [dX GEMM].
+        fp32: eler, fwd, [merge], dlt, bwd_src, [merge], bwd_dst, reduce (the fp32 GEMMs are cuBLAS's)."""
         v = self.layout.view(self.part, arrays=False)
-        return 6 + (1 if v["num_fwd_splits"] > 0 else 0) + (1 if v["num_bwd_splits"] > 0 else 0)
+        splits = (1 if v["num_fwd_splits"] > 0 else 0) + (1 if v["num_bwd_splits"] > 0 else 0)
+        if self.dtype == torch.bfloat16:
+            return 8 + splits + (1 if self.grad_x is not None else 0)
+        return 6 + splits

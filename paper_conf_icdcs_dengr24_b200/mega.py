@@ -95,7 +95,9 @@ def lib():
                                  P, P, _c.c_size_t, P]),
             "mega_gat_bwd": (S, [P, _c.c_int32, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64,
                                  P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P]),
-            "mega_project_bwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, S, P, I64, P, I64, P, P]),
+            "mega_project_workspace_bytes": (S, [I64, _c.c_int, _c.c_int, _c.c_int, S, P]),
+            "mega_project_bwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, S, P, I64, P, I64, P, P,
+                                     _c.c_size_t, P]),
             "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P]),
             "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, P]),
             "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P, I64, P, P, P, I64,
@@ -275,11 +277,18 @@ def mega_gat_bwd(layout: Layout, part, feat, attn_l, attn_r, heads, head_dim, ou
                               _stream(stream)))
 
 
-def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_dim=None, stream=None):
+def mega_project_workspace_bytes(rows, in_dim, heads, head_dim, dtype) -> int:
+    b = _c.c_size_t()
+    _check(lib().mega_project_workspace_bytes(rows, in_dim, heads, head_dim, dtype, _c.byref(b)))
+    return b.value
+
+
+def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_dim=None, ws=None, stream=None):
     dt = _dtype_code(x)
     _check(lib().mega_project_bwd(_ptr(x), x.stride(0), x.shape[0], in_dim or w.shape[0], _ptr(w), heads, head_dim,
                                   dt, _ptr(grad_feat), grad_feat.stride(0), _ptr(grad_x),
-                                  grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _stream(stream)))
+                                  grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _ptr(ws),
+                                  0 if ws is None else ws.numel() * ws.element_size(), _stream(stream)))
 
 
 # NEXT-3: Graph Transformer edge attention (include/mega.h mega_gt_*; fp32)
@@ -289,13 +298,27 @@ def mega_gt_workspace_bytes(layout: Layout, part: int, heads: int):
     return b.value
 
 
+def _gt_check(name, tensors, ld_group):
+    """mega_gt_* take fp32 row-major operands with ONE leading dimension per group:
+    refuse anything else instead of letting the kernels read it as the wrong data."""
+    import torch
+    for t in tensors:
+        if t.dtype != torch.float32 or not t.is_cuda or t.dim() != 2 or t.stride(1) != 1:
+            raise TypeError(f"{name}: operands must be fp32 CUDA 2-D tensors with unit column stride")
+    if len({t.stride(0) for t in ld_group}) != 1:
+        raise ValueError(f"{name}: {len(ld_group)} operands sharing one leading dimension have different strides")
+
+
 def mega_gt_fwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, stream=None):
+    _gt_check("mega_gt_fwd", (q, k, v, out, lse), (q, k, v))
     _check(lib().mega_gt_fwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
                              out.stride(0), _ptr(lse), _stream(stream)))
 
 
 def mega_gt_bwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, grad_out, grad_q, grad_k, grad_v, ws,
                 stream=None):
+    _gt_check("mega_gt_bwd", (q, k, v, out, lse, grad_out, grad_q, grad_k, grad_v), (q, k, v))
+    _gt_check("mega_gt_bwd", (grad_q, grad_k, grad_v), (grad_q, grad_k, grad_v))
     _check(lib().mega_gt_bwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
                              out.stride(0), _ptr(lse), _ptr(grad_out), grad_out.stride(0), _ptr(grad_q), _ptr(grad_k),
                              _ptr(grad_v), grad_k.stride(0), _ptr(ws), ws.numel() * ws.element_size(),

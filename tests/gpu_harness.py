@@ -106,39 +106,80 @@ def assert_fp32_close(got, ref, name):
     assert not bad.any(), f"{name}: {bad.sum()} elements out of tolerance, max err {err.max():.3e}"
 
 
-def assert_bf16_close(got, ref, name):
-    """north_star bf16 bar: max|gpu - ref| <= 2e-2 max|ref| per tensor."""
+def assert_bf16_close(got, ref, name, extra=None):
+    """north_star bf16 bar: max|gpu - ref| <= 2e-2 max|ref| per tensor.
+    `extra` (elementwise, optional) adds a derived error bound (see dlt_bf16_bound)."""
     got = np.asarray(got, np.float64)
     ref = np.asarray(ref, np.float64)
     fin = np.isfinite(ref)
     assert np.array_equal(fin, np.isfinite(got)), f"{name}: finiteness differs"
     scale = np.max(np.abs(ref[fin])) if fin.any() else 0.0
-    err = np.max(np.abs(got[fin] - ref[fin])) if fin.any() else 0.0
-    # + the fp32 absolute term (DESIGN.md R-tol): the bf16 path accumulates in fp32, and a tensor whose
-    # reference is exactly 0 by cancellation (e.g. all in-edges of a row from one source) keeps fp32 noise
-    assert err <= 2e-2 * scale + 1e-4, f"{name}: max err {err:.3e} > 2e-2 * {scale:.3e} + 1e-4"
+    err = np.abs(got[fin] - ref[fin])
+    tol = 2e-2 * scale + (0.0 if extra is None else np.asarray(extra, np.float64)[fin])
+    bad = err > tol
+    assert not bad.any(), (f"{name}: {bad.sum()} elements out of tolerance, max err {err.max():.3e} "
+                           f"(2e-2 * {scale:.3e}{'' if extra is None else ' + derived bound'})")
 
 
-def assert_fp32_close_reduction(got, ref, name):
-    """fp32 bar for the parameter gradients (DESIGN.md R-tol): they are sums over all N
-    rows of terms whose own fp32 relative error is ~1e-6 (exp/log chains), so the
-    relative part is taken against the tensor's scale: |d| <= 1e-4 + 1e-5 max|ref|."""
-    got = np.asarray(got, np.float64)
-    ref = np.asarray(ref, np.float64)
-    err = np.abs(got - ref)
-    tol = 1e-4 + 1e-5 * np.max(np.abs(ref))
-    assert np.all(err <= tol), f"{name}: max err {err.max():.3e} > {tol:.3e}"
+def dlt_bf16_bound(ip, ix, Wh, a_l, a_r, g, slope=M.SLOPE):
+    """Elementwise bound on the grad_attn_l / grad_attn_r error that bf16 storage of
+    `out` introduces (DESIGN.md R-prec, "Dlt bound").  The GPU forms Dlt_i = g_i . out_i
+    from the STORED bf16 out (a6 saves an edge pass that way), so its grad_attn carry
+    the effect of that rounding, which does not vanish where the exact result is 0 by
+    cancellation.  The bound has three parts, all computed from the fp64 oracle
+    (never from the GPU):
+      1. the exact effect of rounding out to bf16: |da(Dlt from bf16(out)) - da(exact)|;
+      2. elements of out within 2^-16 relative of a bf16 rounding midpoint may round the
+         other way on the GPU (its fp32 out differs from the exact one by ~2^-20
+         relative): each costs at most one bf16 ulp, |g_i,f| ulp(out_i,f), in Dlt_i;
+      3. the two F-term fp32 dot products (dalpha_e = g_i . Wh_j, Dlt_i):
+         F 2^-23 (A_i + B_e), A_i = sum_f |g_i||out_i|, B_e = sum_f |g_i||Wh_j|.
+    Parts 2-3 give eps_e per edge and head; dz_e = alpha_e (dalpha_e - Dlt_i) lf_e with
+    lf_e <= 1 gives |d del_i| <= sum_In alpha eps, |d der_j| <= sum_Out alpha eps and
+    |d da_l[h,f]| <= sum_i |d del_i,h| |Wh_i,h,f| (da_r likewise with der)."""
+    import synth as _synth
+    from oracle import gat as og
+    Wh = np.asarray(Wh, np.float64)
+    g = np.asarray(g, np.float64)
+    n, H, F = Wh.shape
+    f = og.gat_forward(ip, ix, Wh, a_l, a_r, slope)
+    b = og.gat_backward(ip, ix, Wh, a_l, a_r, g, slope, fwd=f)
+    out = f["out"]
+    outb = _synth.bf16_round(out.astype(np.float32)).astype(np.float64)
+    b_r = og.gat_backward(ip, ix, Wh, a_l, a_r, g, slope, fwd={**f, "out": outb})     # part 1
+    # part 2: distance to the nearest bf16 rounding midpoint, relative
+    ulp = np.where(out != 0, 2.0 ** (np.floor(np.log2(np.abs(np.where(out != 0, out, 1.0)))) - 7), 0.0)
+    mid_dist = np.abs(np.abs(out - outb) - 0.5 * ulp)
+    near = mid_dist <= 2.0 ** -16 * np.abs(out)
+    flip = np.einsum("nhf,nhf->nh", np.abs(g), np.where(near, ulp, 0.0))
+    deg = np.diff(np.asarray(ip, np.int64))
+    dst = np.repeat(np.arange(n), deg)
+    src = np.asarray(ix, np.int64)
+    A = np.einsum("nhf,nhf->nh", np.abs(g), np.abs(out))
+    B = np.einsum("ehf,ehf->eh", np.abs(g[dst]), np.abs(Wh[src]))
+    eps = flip[dst] + F * 2.0 ** -23 * (A[dst] + B)                                 # parts 2 + 3
+    t = f["alpha"] * eps
+    ddel = np.zeros((n, H))
+    np.add.at(ddel, dst, t)
+    dder = np.zeros((n, H))
+    np.add.at(dder, src, t)
+    aW = np.abs(Wh)
+    return {"grad_attn_l": np.abs(b_r["grad_attn_l"] - b["grad_attn_l"]) + np.einsum("nh,nhf->hf", ddel, aW),
+            "grad_attn_r": np.abs(b_r["grad_attn_r"] - b["grad_attn_r"]) + np.einsum("nh,nhf->hf", dder, aW)}
 
 
 REDUCTIONS = ("grad_attn_l", "grad_attn_r", "grad_w")
 
 
-def check(got, ref, dtype, keys=("out", "lse", "grad_feat", "grad_attn_l", "grad_attn_r")):
+def check(got, ref, dtype, keys=("out", "lse", "grad_feat", "grad_attn_l", "grad_attn_r"), graph=None):
+    """graph = (indptr, indices, Wh, a_l, a_r, g) in old ids: in bf16 mode the attention-parameter
+    gradients then also get the derived Dlt bound (dlt_bf16_bound)."""
+    bound = dlt_bf16_bound(*graph) if (graph is not None and dtype == "bf16") else {}
     for k in keys:
         if dtype == "fp32":
             (assert_fp32_close_reduction if k in REDUCTIONS else assert_fp32_close)(got[k], ref[k], k)
         else:
-            assert_bf16_close(got[k], ref[k], k)
+            assert_bf16_close(got[k], ref[k], k, extra=bound.get(k))
 
 
 def layer(layout, x_new, w, a_l, a_r, H, F, dtype, want_grad_x=True):

@@ -129,4 +129,4 @@ def test_gpu_parity_batches(cuda_device, dtype, cfg_name, H, F):
     got = hz.run_attention(lay, Wh, a_l, a_r, g, dtype)
     f = coracle.gat_forward(ip, ix, Wh, a_l, a_r)
     ref = {**f, **coracle.gat_backward(ip, ix, Wh, a_l, a_r, g, fwd=f)}
-    hz.check(got, ref, dtype)
+    hz.check(got, ref, dtype, graph=(ip, ix, Wh, a_l, a_r, g))

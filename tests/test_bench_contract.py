@@ -42,6 +42,19 @@ def test_gpu_arm_line():
     assert {"sm_mhz", "sm_max_mhz", "reasons"} <= set(d["clocks"])
 
 
+def test_reference_arm_runs_no_product_code():
+    """The reference arm is the oracle alone: it must not import the package or load libmega.so."""
+    code = ("import sys, json; sys.argv = ['bench.py', '--impl', 'reference', '--config', 'cora', '--steps', '1', "
+            "'--warmup', '0']; import bench; bench.main(); "
+            "maps = open('/proc/self/maps').read(); "
+            "print(json.dumps({'pkg': any(m.startswith('paper_conf_icdcs_dengr24_b200') for m in sys.modules), "
+            "'so': 'libmega.so' in maps}))")
+    r = subprocess.run([sys.executable, "-c", code], capture_output=True, text=True, timeout=600, cwd=ROOT)
+    assert r.returncode == 0, r.stderr[-2000:]
+    res = json.loads(r.stdout.strip().splitlines()[-1])
+    assert res == {"pkg": False, "so": False}
+
+
 def test_reference_arm_batch_config():
     d = _run(["--impl", "reference", "--config", "aqsol-b128-drop20", "--steps", "2", "--warmup", "1"], 600)
     assert KEYS <= set(d) and d["impl"] == "reference" and d["value"] > 0

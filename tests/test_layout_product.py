@@ -25,7 +25,7 @@ def test_exports_every_declared_symbol():
     L = M.lib()
     for name in sorted(declared):
         assert hasattr(L, name), name
-    assert M.mega_abi_version() == 1
+    assert M.mega_abi_version() == 2
 
 
 def test_invalid_inputs_are_rejected():
