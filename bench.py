@@ -188,7 +188,7 @@ class Model:
 
     def __init__(self, wl, dtype, dev, rank=0, world=1):
         import torch
-        from paper_conf_icdcs_dengr24_b200.dist import DistGATLayer
+        from paper_conf_icdcs_dengr24_b200.dist import DistGATLayer, make_comm
         self.torch = torch
         cfg = wl["cfg"]
         tdt = torch.bfloat16 if dtype == "bf16" else torch.float32
@@ -200,12 +200,13 @@ class Model:
         self.x0 = torch.tensor(wl["x0"][self.b0:self.b1], device=dev).to(tdt).contiguous()
         self.g = torch.tensor(wl["g_last"][self.b0:self.b1], device=dev).to(tdt).contiguous()
         self.layers = []
+        self.comm = make_comm() if world > 1 else None   # library-owned NCCL communicator
         x = self.x0
         for li, inp in enumerate(wl["layers"]):
             w = torch.tensor(inp["w"], device=dev).to(tdt).contiguous()
             Ld = DistGATLayer(lay, rank, x, w, torch.tensor(inp["a_l"], device=dev),
                               torch.tensor(inp["a_r"], device=dev), cfg.heads, cfg.head_dim, in_dim=inp["in_dim"],
-                              want_grad_x=li > 0, lp_only=dtype == "bf16")
+                              want_grad_x=li > 0, lp_only=dtype == "bf16", comm=self.comm)
             self.layers.append(Ld)
             x = Ld.L.out
         self.launches = sum(Ld.L.launches_per_step() for Ld in self.layers)
@@ -376,6 +377,8 @@ def run_mega(args):
     torch.cuda.set_device(local)
     dev = torch.device("cuda", local)
     if world > 1:
+        if args.gpus != world:
+            raise SystemExit(f"bench.py --gpus {args.gpus} launched with WORLD_SIZE={world}")
         dist.init_process_group("nccl", device_id=dev)
 
     def sync_all():
@@ -549,8 +552,37 @@ def run_mega(args):
         dist.destroy_process_group()
 
 
+def free_port():
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def launch_cmd(argv, n, port):
+    """The one-process-per-GPU relaunch of `bench.py argv` on n GPUs of this node."""
+    return [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}", "--master-addr",
+            "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *argv]
+
+
+def maybe_spawn(args, argv):
+    """`bench.py --gpus N` without a torchrun environment: re-launch itself as N ranks
+    (one per GPU, NCCL) and exit with their status.  Fails loudly without N devices."""
+    if args.impl != "mega" or args.gpus <= 1 or "WORLD_SIZE" in os.environ:
+        return
+    import torch
+    have = torch.cuda.device_count()
+    if have < args.gpus:
+        raise SystemExit(f"bench.py --gpus {args.gpus}: only {have} CUDA device(s) visible")
+    r = subprocess.run(launch_cmd(argv, args.gpus, free_port()))
+    raise SystemExit(r.returncode)
+
+
 def main():
     args = parse()
+    maybe_spawn(args, sys.argv[1:])
     if args.impl == "reference":
         run_reference(args)
     else:

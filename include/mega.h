@@ -73,7 +73,8 @@ typedef enum {
   MEGA_ERR_OUT_OF_MEMORY = 4,    /* host allocation failed, or a caller buffer is too small */
   MEGA_ERR_CUDA = 5,             /* a CUDA runtime / cuBLAS call failed (message has details) */
   MEGA_ERR_STATE = 6,            /* layout part not bound, or bound to another device */
-  MEGA_ERR_IO = 7                /* mega_layout_save / _load file errors or bad format */
+  MEGA_ERR_IO = 7,               /* mega_layout_save / _load file errors or bad format */
+  MEGA_ERR_NCCL = 8              /* NCCL could not be loaded or an NCCL call failed (message has details) */
 } mega_status;
 
 typedef enum { MEGA_F32 = 0, MEGA_BF16 = 1 } mega_dtype;
@@ -169,6 +170,8 @@ typedef struct {
 #define MEGA_BWD_PHASE_DST 4u    /* mega_gat_bwd: destination pass over this part's rows -> adds
                                     del_i a_l to grad_feat, writes grad_feat_lp, grad_attn_l and
                                     grad_attn_r (partials of this part for k > 1).  Neither flag = both. */
+#define MEGA_DIST_PHASE_SEND 16u  /* mega_gat_*_dist: only the first half (see below); neither = both */
+#define MEGA_DIST_PHASE_RECV 32u
 #define MEGA_BWD_LP_ONLY 8u      /* mega_gat_bwd with grad_feat_lp != NULL: the final rows are written
                                     only to grad_feat_lp (the GEMM operand of mega_project_bwd);
                                     grad_feat keeps the fp32 source-phase partial.  Saves a D*4-byte
@@ -276,6 +279,90 @@ mega_status mega_gat_bwd(const mega_layout *layout, int32_t part, const void *fe
 mega_status mega_project_bwd(const void *x, int64_t ldx, int64_t rows, int in_dim, const void *w, int heads,
                              int head_dim, mega_dtype dtype, const void *grad_feat, int64_t ldgf, void *grad_x,
                              int64_t ldgx, float *grad_w, void *ws, size_t ws_bytes, mega_stream_t stream);
+
+/* ---------------- k GPUs: destination partitions ----------------
+ * The exact counterpart of the paper's "partition of the path representation
+ * ... only two communications for adjacent path partitions":
+ * a layout with num_parts = k gives rank p the contiguous, edge-balanced rows
+ * [bounds[p], bounds[p+1]) of the MEGA order (R23) and every
+ * in-edge of those rows.  Per layer, rank p exchanges the projected source
+ * rows [Wh | er] in the forward and the partial [dWh | der] of other ranks'
+ * rows in the backward.  The library owns the communicator. */
+typedef struct mega_comm mega_comm;
+
+/* NCCL transport (one process per GPU).  Rank 0 calls mega_comm_unique_id and
+ * broadcasts the 128 bytes over the caller's own process group; every rank
+ * then calls mega_comm_init with its rank and CUDA device.  libnccl.so.2 is
+ * loaded on first use (the copy the process already has, else the system's).
+ * Errors: NCCL (library missing or a call failed), CUDA, INVALID_ARGUMENT. */
+mega_status mega_comm_unique_id(uint8_t id[128]);
+mega_status mega_comm_init(const uint8_t id[128], int nranks, int rank, int device, mega_comm **out);
+/* LOCAL transport: all `nranks` ranks driven by ONE process (devices[r], or
+ * the current device for every rank when devices == NULL).  Messages are
+ * stream-ordered device-to-device copies from the peer's buffers (peer
+ * memory when ranks sit on different GPUs).  The caller runs every dist call
+ * with MEGA_DIST_PHASE_SEND on all ranks, then with MEGA_DIST_PHASE_RECV on all
+ * ranks, and must not modify a sent buffer until the receiving phase is done.
+ * out[0..nranks) receive the communicators. */
+mega_status mega_comm_init_local(int nranks, const int *devices, mega_comm **out);
+void mega_comm_destroy(mega_comm *comm);
+/* transport: 0 = NCCL, 1 = LOCAL */
+mega_status mega_comm_info(const mega_comm *comm, int *nranks, int *rank, int *device, int *transport);
+
+/* Read-only host view of the k-GPU work split of one part (for tests): the
+ * forward items of the local pass (sources this part owns) and the remote pass,
+ * as [n][4] (row, e_begin, e_end, slot | -1) over the part's CSR positions, the
+ * merge records [n][3] (row, first_slot, nseg), and the ranges of bwd_items /
+ * bwd_splits that belong to the part's own sources.  Empty for k = 1. */
+typedef struct {
+  uint32_t struct_size;
+  int64_t num_local_items, num_remote_items, num_splits, num_slots;
+  int64_t bwd_own_items_begin, bwd_own_items_end, bwd_own_splits_begin, bwd_own_splits_end;
+  const int32_t *local_items, *remote_items, *splits;
+} mega_layout_dist_view;
+mega_status mega_layout_dist_view_get(mega_layout *layout, int32_t part, mega_layout_dist_view *out);
+
+/* Workspaces of the dist calls on part `part` (fwd: slots of the split rows;
+ * bwd: mega_gat_bwd's plus a receive area of (k-1) * rows_p * (D + heads) fp32). */
+mega_status mega_gat_dist_workspace_bytes(const mega_layout *layout, int32_t part, int heads, int head_dim,
+                                          mega_dtype dtype, size_t *fwd_ws, size_t *bwd_ws);
+
+/* Forward on rank `part` (= the comm rank) of a k-part layout, overlapped with
+ * the exchange (SURVEY §8(e) forward steps 2-4):
+ *   1. on comm_stream: send this rank's projected rows [Wh | er] (feat rows and
+ *      the er plane of ctx, rows [bounds[p], bounds[p+1])) to every peer and
+ *      receive the peers' rows into the same global arrays;
+ *   2. meanwhile on `stream`: fused score/softmax/aggregation over block (p,p),
+ *      the in-edges whose source this rank owns;
+ *   3. after the receives: the remote blocks, then a fixed-order merge (KB7) of
+ *      the rows whose edges were split between the passes.
+ * feat (device [num_nodes][ldf], GLOBAL rows, written for the peers' rows) must
+ * hold this rank's projected rows; ctx holds their el/er with
+ * MEGA_FLAG_ELER_IN_CTX (from mega_project_fwd), else they are computed first.
+ * Other arguments as mega_gat_fwd.  PHASE flags: SEND = steps 1-2, RECV = step 3. */
+mega_status mega_gat_fwd_dist(const mega_layout *layout, int32_t part, mega_comm *comm, void *feat, int64_t ldf,
+                              const float *attn_l, const float *attn_r, int heads, int head_dim, mega_dtype dtype,
+                              float negative_slope, uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws,
+                              size_t ws_bytes, mega_stream_t stream, mega_stream_t comm_stream);
+
+/* Backward of mega_gat_fwd_dist (SURVEY §8(e) backward):
+ *   SEND: Dlt; the source-major pass for the sources OTHER ranks own, whose
+ *     partial [dWh | der] rows then travel to their owners on comm_stream
+ *     (a reduce-scatter-v done as grouped point-to-point messages) while the
+ *     source pass for this rank's own sources runs on `stream`;
+ *   RECV: the peers' partials of this rank's rows are added in fixed peer
+ *     order, then the destination pass on this rank's rows.
+ * grad_feat: device fp32 [num_nodes][D] (ldgf == D), GLOBAL rows: on return
+ * rows [bounds[p], bounds[p+1]) are final (other rows hold this rank's partial).
+ * grad_attn_l/r are THIS RANK'S PARTIAL sums: the caller all-reduces them with
+ * the projection's grad_w (data-parallel parameter gradients).
+ * Other arguments as mega_gat_bwd. */
+mega_status mega_gat_bwd_dist(const mega_layout *layout, int32_t part, mega_comm *comm, const void *feat,
+                              int64_t ldf, const float *attn_l, const float *attn_r, int heads, int head_dim,
+                              mega_dtype dtype, float negative_slope, uint32_t flags, const void *out, int64_t ldo,
+                              const void *grad_out, int64_t ldg, float *ctx, float *grad_feat, int64_t ldgf,
+                              void *grad_feat_lp, int64_t ldlp, float *grad_attn_l, float *grad_attn_r, void *ws,
+                              size_t ws_bytes, mega_stream_t stream, mega_stream_t comm_stream);
 
 /* NEXT-3: Graph Transformer edge attention, the paper's
  * headline model (Table I; DESIGN.md R-gt), over the same layout:

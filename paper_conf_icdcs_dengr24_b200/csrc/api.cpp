@@ -53,12 +53,58 @@ std::vector<int32_t> make_tiles(const std::vector<int32_t> &items) {
   return t;
 }
 
+// Forward work split by source owner for the k-GPU path:
+// part p's row r has its edges sorted by new source id, so the edges from p's own
+// rows [b_p, b_{p+1}) (block (p,p), computable before any exchange) are one
+// contiguous range [l0, l1) and the remote ones are [e0, l0) and [l1, e1).
+// Each range is cut into segments of <= S edges.  A row whose edges form a single
+// segment is finalised by the pass that owns it (slot -1); every other row gets a
+// contiguous block of slots (local segments first) and a split record
+// (row, first_slot, nseg) for the fixed-order merge after the remote pass.  Rows
+// without edges are finalised (out = 0, lse = -inf) by the local pass.
+void dist_items(const mega_layout *L, int part, std::vector<int32_t> &local, std::vector<int32_t> &remote,
+                std::vector<int32_t> &splits, int32_t &nslots) {
+  const Part &P = L->parts[part];
+  const int32_t b0 = L->bounds[part], b1 = L->bounds[part + 1];
+  const int32_t S = (int32_t)std::max<int64_t>(1, L->stats.seg_edges);
+  local.clear(); remote.clear(); splits.clear();
+  nslots = 0;
+  const int64_t rows = (int64_t)P.indptr.size() - 1;
+  for (int64_t r = 0; r < rows; ++r) {
+    const int32_t e0 = P.indptr[r], e1 = P.indptr[r + 1];
+    if (e1 == e0) { local.insert(local.end(), {(int32_t)r, e0, e0, -1}); continue; }
+    const int32_t *sb = P.src.data() + e0, *se = P.src.data() + e1;
+    const int32_t l0 = e0 + (int32_t)(std::lower_bound(sb, se, b0) - sb);
+    const int32_t l1 = e0 + (int32_t)(std::lower_bound(sb, se, b1) - sb);
+    const int32_t rng[3][3] = {{l0, l1, 1}, {e0, l0, 0}, {l1, e1, 0}};   // (begin, end, is_local)
+    int32_t nseg = 0;
+    for (auto &q : rng) if (q[1] > q[0]) nseg += (q[1] - q[0] + S - 1) / S;
+    const bool single = nseg == 1;
+    const int32_t base = single ? -1 : nslots;
+    int32_t k = 0;
+    for (auto &q : rng)
+      for (int32_t b = q[0]; b < q[1]; b += S) {
+        std::vector<int32_t> &dst = q[2] ? local : remote;
+        dst.insert(dst.end(), {(int32_t)r, b, std::min(q[1], b + S), single ? -1 : base + k});
+        ++k;
+      }
+    if (!single) {
+      splits.insert(splits.end(), {(int32_t)r, base, nseg});
+      nslots += nseg;
+    }
+  }
+}
+
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]) {
   const Part &P = L->parts[part];
+  std::vector<int32_t> dl, dr, ds;
+  int32_t nsl = 0;
+  if (L->parts.size() > 1) dist_items(L, part, dl, dr, ds, nsl);
   const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
                                       P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
-                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size()};
+                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size(),
+                                      dl.size(), dr.size(), ds.size()};
   size_t off = 0;
   for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
@@ -84,6 +130,7 @@ const char *mega_status_string(mega_status s) {
     case MEGA_ERR_CUDA: return "MEGA_ERR_CUDA";
     case MEGA_ERR_STATE: return "MEGA_ERR_STATE";
     case MEGA_ERR_IO: return "MEGA_ERR_IO";
+    case MEGA_ERR_NCCL: return "MEGA_ERR_NCCL";
   }
   return "MEGA_ERR_UNKNOWN";
 }
@@ -177,6 +224,35 @@ mega_status mega_layout_view_get(const mega_layout *L, int32_t part, mega_layout
   return MEGA_OK;
 }
 
+mega_status mega_layout_dist_view_get(mega_layout *L, int32_t part, mega_layout_dist_view *v) {
+  clear_error();
+  if (!L || !v) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  Part &P = L->parts[part];
+  std::memset(v, 0, sizeof *v);
+  v->struct_size = sizeof *v;
+  if (L->parts.size() > 1) {
+    dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
+    auto first_ge = [](const std::vector<int32_t> &a, int stride, int32_t x) {
+      int64_t lo = 0, hi = (int64_t)a.size() / stride;
+      while (lo < hi) { int64_t mid = (lo + hi) / 2; if (a[mid * stride] < x) lo = mid + 1; else hi = mid; }
+      return lo;
+    };
+    v->bwd_own_items_begin = first_ge(P.bwd_items, 4, (int32_t)P.row_begin);
+    v->bwd_own_items_end = first_ge(P.bwd_items, 4, (int32_t)P.row_end);
+    v->bwd_own_splits_begin = first_ge(P.bwd_splits, 3, (int32_t)P.row_begin);
+    v->bwd_own_splits_end = first_ge(P.bwd_splits, 3, (int32_t)P.row_end);
+  }
+  v->num_local_items = (int64_t)P.dl_items.size() / 4;
+  v->num_remote_items = (int64_t)P.dr_items.size() / 4;
+  v->num_splits = (int64_t)P.d_splits.size() / 3;
+  v->num_slots = P.n_d_slots;
+  v->local_items = P.dl_items.data();
+  v->remote_items = P.dr_items.data();
+  v->splits = P.d_splits.data();
+  return MEGA_OK;
+}
+
 mega_status mega_layout_device_bytes(const mega_layout *L, int32_t part, size_t *bytes) {
   clear_error();
   if (!L || !bytes) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
@@ -221,9 +297,11 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   for (int64_t v = 0; v < L->n; ++v)
     for (int32_t q = P.cindptr[v]; q < P.cindptr[v + 1]; ++q) csrc[q] = (int32_t)v;
   const std::vector<int32_t> ftiles = make_tiles(P.fwd_items), btiles = make_tiles(P.bwd_items);
+  if (L->parts.size() > 1) dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
-      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos};
+      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos,
+      &P.dl_items, &P.dr_items, &P.d_splits};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
@@ -261,6 +339,24 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.n_bwd_splits = (int32_t)(P.bwd_splits.size() / 3);
   D.n_bwd_slots = P.n_bwd_slots;
   D.id_mask = packed ? ((1u << 26) - 1u) : 0x7fffffffu;
+  D.dl_items = reinterpret_cast<const int4 *>(base + offs[14]);
+  D.dr_items = reinterpret_cast<const int4 *>(base + offs[15]);
+  D.d_splits = reinterpret_cast<const int32_t *>(base + offs[16]);
+  D.n_dl_items = (int32_t)(P.dl_items.size() / 4);
+  D.n_dr_items = (int32_t)(P.dr_items.size() / 4);
+  D.n_d_splits = (int32_t)(P.d_splits.size() / 3);
+  D.n_d_slots = P.n_d_slots;
+  {  // own-source ranges of the CSC work (items and splits are sorted by source id)
+    auto first_ge = [](const std::vector<int32_t> &v, int stride, int32_t x) {
+      int64_t lo = 0, hi = (int64_t)v.size() / stride;
+      while (lo < hi) { int64_t mid = (lo + hi) / 2; if (v[mid * stride] < x) lo = mid + 1; else hi = mid; }
+      return (int32_t)lo;
+    };
+    D.bwd_own0 = first_ge(P.bwd_items, 4, (int32_t)P.row_begin);
+    D.bwd_own1 = first_ge(P.bwd_items, 4, (int32_t)P.row_end);
+    D.bsplit_own0 = first_ge(P.bwd_splits, 3, (int32_t)P.row_begin);
+    D.bsplit_own1 = first_ge(P.bwd_splits, 3, (int32_t)P.row_end);
+  }
   // pageable-memory copies return once staged, so the packed temporaries may go
   return MEGA_OK;
 }

@@ -221,7 +221,6 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
   const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
-  const uint32_t row_bytes = (uint32_t)(a.D * sizeof(T));
   const float *sp_v[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
@@ -253,8 +252,6 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   auto stage_er = [&](int b, int4 itm, int bse) {
     const uint32_t jj = (uint32_t)s_src[b][w][rb + gl];
     cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
-    if (bse + gl < itm.z && gl < a.pf_rows)
-      prefetch_l2_bulk(feat + (jj & idm) * ldf, row_bytes, (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row);
     cp_async_commit();
   };
   // prologue: descriptor batches 0 and 1, chunk 0 staged
@@ -411,144 +408,6 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
     base = nbase;
     q = nq;
     buf = nb_;
-  }
-  cp_async_wait<0>();
-}
-
-// ---- a3+a4+a5 for wide rows (G = 32 lanes per row): cp.async ring pipeline ----
-// Each warp streams its source rows through a private shared-memory ring of P
-// quads (4 rows each) with cp.async (LDGSTS, L2 cache-policy hints): every lane
-// copies and later reads back exactly its own 16-byte pieces, so the ring
-// needs no barriers; P quads stay in flight without holding registers.
-template <typename T, int V, int HT, int P>
-__global__ void __launch_bounds__(TPB, 2) gat_fwd_ring_kernel(const FwdArgs a) {
-  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, SP = HT + 1, RSLOT = 4 * P;
-  extern __shared__ uint4 ring_all[];   // [WPB][RSLOT][V][32]
-  __shared__ float s_p[WPB][32][SP];
-  __shared__ int s_j[WPB][32];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-  uint4 *ring = ring_all + (size_t)w * RSLOT * V * 32;
-  const int H = a.H;
-  const uint32_t idm = a.L.id_mask;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
-  int hv[V];
-#pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / FF;
-  const T *featl = static_cast<const T *>(a.feat) + lane * EPV;
-  const uint32_t ldf = (uint32_t)a.ldf;
-  const int64_t stride = (int64_t)gridDim.x * WPB;
-  auto issue_quad = [&](int q, int cnt) {
-#pragma unroll
-    for (int r = 0; r < 4; ++r) {
-      const int k = min(4 * q + r, cnt - 1);  // the tail re-reads the last row (weight p = 0)
-      const uint32_t jj = (uint32_t)s_j[w][k];
-      const T *rp = featl + (jj & idm) * ldf;
-      const uint64_t pol = (int)(jj >> 26) >= a.hot_cls ? pol_hot : pol_row;
-      uint4 *dst = ring + ((q % P) * 4 + r) * V * 32 + lane;
-#pragma unroll
-      for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
-    }
-    cp_async_commit();
-  };
-  for (int64_t it = (int64_t)blockIdx.x * WPB + w; it < a.L.n_fwd_items; it += stride) {
-    const int4 item = a.L.fwd_items[it];
-    const int64_t grow = a.L.row_begin + item.x;
-    float elr[HT], mrun[HT], lrun[HT];
-    load_h<HT>(a.el + grow * H, H, elr);
-#pragma unroll
-    for (int h = 0; h < HT; ++h) { mrun[h] = -INFINITY; lrun[h] = 0.f; }
-    float acc[V][EPV];
-#pragma unroll
-    for (int v = 0; v < V; ++v)
-#pragma unroll
-      for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
-    for (int base = item.y; base < item.z; base += G) {
-      const int e = base + lane;
-      const bool valid = e < item.z;
-      const int jr = ld_stream(a.L.src + min(e, item.z - 1), pol_cold);
-      const int cnt = min(G, item.z - base), nq = (cnt + 3) >> 2;
-      float erj[HT];
-      load_h<HT>(a.er + (int64_t)((uint32_t)jr & idm) * H, H, erj);
-      s_j[w][lane] = jr;
-      __syncwarp();
-#pragma unroll
-      for (int q = 0; q < P; ++q) {
-        if (q < nq) issue_quad(q, cnt);
-        else cp_async_commit();
-      }
-      float sc[HT];
-#pragma unroll
-      for (int h = 0; h < HT; ++h) {
-        sc[h] = 1.f;
-        if (h < H) {
-          const float s = valid ? leaky(elr[h] + erj[h], a.slope) : -INFINITY;
-          const float mn = fmaxf(mrun[h], gmax<G>(s, 0xffffffffu));
-          sc[h] = fexp(mrun[h] - mn);
-          const float p = valid ? fexp(s - mn) : 0.f;
-          lrun[h] = fmaf(lrun[h], sc[h], p);
-          mrun[h] = mn;
-          s_p[w][lane][h] = p;
-        }
-      }
-#pragma unroll
-      for (int v = 0; v < V; ++v) {
-        const float f = sel<HT>(sc, hv[v]);
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
-      }
-      __syncwarp();
-      for (int q = 0; q < nq; ++q) {
-        cp_async_wait<P - 1>();
-#pragma unroll
-        for (int r = 0; r < 4; ++r) {
-          const int k = 4 * q + r;
-          const uint4 *src = ring + ((q % P) * 4 + r) * V * 32 + lane;
-#pragma unroll
-          for (int v = 0; v < V; ++v) {
-            const float pw = s_p[w][k][hv[v]];
-            float x[EPV];
-            unpack(src[v * 32], x, T());
-#pragma unroll
-            for (int kk = 0; kk < EPV; kk += 2) ffma2s(acc[v][kk], acc[v][kk + 1], x[kk], x[kk + 1], pw);
-          }
-        }
-        if (q + P < nq) issue_quad(q + P, cnt);
-        else cp_async_commit();
-      }
-      __syncwarp();
-    }
-    float lt[HT];
-#pragma unroll
-    for (int h = 0; h < HT; ++h) lt[h] = h < H ? gsum<G>(lrun[h], 0xffffffffu) : 0.f;
-    if (item.w < 0) {
-      T *orow = static_cast<T *>(a.out) + (int64_t)item.x * a.ldo + lane * EPV;
-#pragma unroll
-      for (int v = 0; v < V; ++v) {
-        const float Lh = sel<HT>(lt, hv[v]);
-        const float inv = Lh > 0.f ? 1.f / Lh : 0.f;
-        float y[EPV];
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) y[k] = acc[v][k] * inv;
-        st16(orow + v * G * EPV, pack(y, T()));
-      }
-      for (int h = lane; h < H; h += G) {
-        const float Lh = sel<HT>(lt, h);
-        a.lse[grow * H + h] = Lh > 0.f ? sel<HT>(mrun, h) + flog(Lh) : -INFINITY;
-      }
-    } else {
-      const int64_t slot = item.w;
-      for (int h = lane; h < H; h += G) {
-        a.ws_m[slot * H + h] = sel<HT>(mrun, h);
-        a.ws_l[slot * H + h] = sel<HT>(lt, h);
-      }
-      float *pr = a.ws_acc + slot * a.D + lane * EPV;
-#pragma unroll
-      for (int v = 0; v < V; ++v)
-#pragma unroll
-        for (int k = 0; k < EPV; k += 4)
-          *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
-              make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
-    }
   }
   cp_async_wait<0>();
 }
@@ -880,10 +739,8 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
           y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-          if (!a.lp_partial)
-            *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
         }
-        if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
@@ -1091,10 +948,8 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
           y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-          if (!a.lp_partial)
-            *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
         }
-        if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
@@ -1110,590 +965,6 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       }
     }
   }
-}
-
-// ---- a7, chunk-pipelined (G = 32, H <= 4) ----
-// gat_bwd_src_kernel's arithmetic with the fwd pipe kernel's staging: while
-// chunk c runs, the next chunk's destination ids, their (el, lse, Dlt) and
-// (for a new source) er_j are staged in shared memory with cp.async, and the
-// next chunk's g rows and the next source's Wh row are prefetched into L2.
-template <typename T, int V, int HT>
-__global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_pipe_kernel(const BwdArgs a) {
-  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
-  constexpr int U1 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U1 < G ? U1 : G;
-  constexpr int NB = U * V;
-  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
-  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
-  __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
-  __shared__ float s_z[WPB][32][SP];  // dz out
-  __shared__ int4 s_desc[2][WPB][32];
-  __shared__ int s_i[2][WPB][32];     // packed destination rows of a chunk
-  __shared__ __align__(16) float s_el[2][WPB][32][HT];
-  __shared__ __align__(16) float s_ls[2][WPB][32][HT];
-  __shared__ __align__(16) float s_dl[2][WPB][32][HT];
-  __shared__ __align__(16) float s_er[2][WPB][HT];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
-  const unsigned gmask = 0xffffffffu;
-  const int H = a.H;
-  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
-  const uint32_t grow_bytes = (uint32_t)(a.D * sizeof(T));
-  int hv[V];
-#pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
-  int bidx = 0;
-#pragma unroll
-  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
-  const int bu = bidx / V, bv = bidx % V;
-  const int bhead = ((bv * G + gl) * EPV) / FF;
-  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
-  const T *feat = static_cast<const T *>(a.feat);
-  const T *gout = static_cast<const T *>(a.gout);
-  const T *goutl = gout + gl * EPV;
-  const int64_t stride = (int64_t)gridDim.x * WPB;
-  const int64_t it0 = (int64_t)blockIdx.x * WPB + w, n_items = a.L.n_bwd_items;
-  if (it0 >= n_items) return;
-  auto row_load = [&](uint4 (&r)[V], uint32_t ii) {
-    const T *rp = goutl + (ii & idm) * ldg;
-    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
-#pragma unroll
-    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
-  };
-  auto stage_desc = [&](int k) {
-    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
-    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][gl], a.L.bwd_items + itq);
-    cp_async_commit();
-  };
-  // chunk (itm, bse): destination ids; for the first chunk of a source its er, and its Wh row into L2
-  auto stage_ids = [&](int b, int4 itm, int bse) {
-    if (itm.z > itm.y) cp_async_small<4>(&s_i[b][w][gl], a.L.cdst + min(bse + gl, itm.z - 1));
-    else s_i[b][w][gl] = 0;
-    if (bse == itm.y && gl == 0) {
-      cp_async_h<HT>(&s_er[b][w][0], a.er + (int64_t)itm.x * H);
-      prefetch_l2_bulk(feat + (int64_t)itm.x * a.ldf, grow_bytes, pol_row);
-    }
-    cp_async_commit();
-  };
-  // the staged chunk's destination values, and its g rows into L2
-  auto stage_dst = [&](int b, int4 itm, int bse) {
-    const uint32_t ii = (uint32_t)s_i[b][w][gl];
-    const int64_t gi = a.L.row_begin + (int)(ii & idm);
-    cp_async_h<HT>(&s_el[b][w][gl][0], a.el + gi * H);
-    cp_async_h<HT>(&s_ls[b][w][gl][0], a.lse + gi * H);
-    cp_async_h<HT>(&s_dl[b][w][gl][0], a.dlt + gi * H);
-    cp_async_commit();
-    // the chunk's first pf_rows g rows into L2, one 128-byte line per lane per step
-    constexpr int LPR = (32 * V * 16) / 128, RPS = 32 / LPR;
-    const int cnt_n = min(a.pf_rows, itm.z - bse);
-    for (int r0 = 0; r0 < cnt_n; r0 += RPS) {
-      const int r = r0 + gl / LPR;
-      if (r < cnt_n)
-        prefetch_l2_line(reinterpret_cast<const char *>(gout + ((uint32_t)s_i[b][w][r] & idm) * ldg) + (gl % LPR) * 128);
-    }
-  };
-  stage_desc(0);
-  stage_desc(1);
-  cp_async_wait<1>();
-  __syncwarp();
-  int q = 0;
-  int4 item = s_desc[0][w][0];
-  int base = item.y, buf = 0;
-  stage_ids(0, item, base);
-  cp_async_wait<0>();
-  __syncwarp();
-  stage_dst(0, item, base);
-  cp_async_wait<0>();
-  __syncwarp();
-  float whf[V][EPV], acc[V][EPV], derv[V], erj[HT], dacc = 0.f;
-  while (true) {
-    int4 nitem = item;
-    int nbase = base + G;
-    int nq = q;
-    bool has_next = true;
-    if (nbase >= item.z) {
-      nq = q + 1;
-      if (it0 + (int64_t)nq * stride >= n_items) {
-        has_next = false;
-      } else {
-        if (nq % G == 0) {
-          cp_async_wait<0>();
-          __syncwarp();
-          nitem = s_desc[(nq / G) & 1][w][0];
-          __syncwarp();
-          stage_desc(nq / G + 1);
-        } else {
-          nitem = s_desc[(nq / G) & 1][w][nq % G];
-        }
-        nbase = nitem.y;
-      }
-    }
-    const int nb_ = buf ^ 1;
-    if (has_next) stage_ids(nb_, nitem, nbase);
-    const int64_t j = item.x;
-    if (base == item.y) {
-      const T *rp = feat + j * a.ldf + gl * EPV;
-#pragma unroll
-      for (int v = 0; v < V; ++v) {
-        unpack(ldg16(rp + v * G * EPV), whf[v], T());
-        derv[v] = 0.f;
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
-      }
-#pragma unroll
-      for (int h = 0; h < HT; ++h) erj[h] = s_er[buf][w][h];
-      dacc = 0.f;
-    }
-    const int *si = &s_i[buf][w][0];
-    const int c = base + gl;
-    const bool valid = c < item.z;
-    const int cp_c = item.z > item.y ? ld_stream(a.L.cpos + min(c, item.z - 1), policy_first()) : 0;
-    const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
-    uint4 ra[U][V], rz[U][V];
-    if (cnt > 0) {
-#pragma unroll
-      for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)si[min(u, cnt - 1)]);
-      if (nbt > 1) {
-#pragma unroll
-        for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)si[min(U + u, cnt - 1)]);
-      }
-    }
-#pragma unroll
-    for (int h = 0; h < HT; ++h)
-      if (h < H) {
-        const float z = s_el[buf][w][gl][h] + erj[h];
-        const float al = valid ? fexp(leaky(z, a.slope) - s_ls[buf][w][gl][h]) : 0.f;
-        s_a[w][lane][h] = z > 0.f ? al : -al;
-      }
-    cp_async_wait<0>();
-    __syncwarp();
-    if (has_next) stage_dst(nb_, nitem, nbase);
-    const float(*sd)[HT] = s_dl[buf][w];
-    auto consume = [&](const uint4 (&raw)[U][V], int k0) {
-      float p[U][V];
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const float al = fabsf(s_a[w][k0 + u][hv[v]]);
-          float x[EPV];
-          unpack(raw[u][v], x, T());
-          float s0 = 0.f, s1 = 0.f;
-#pragma unroll
-          for (int k = 0; k < EPV; k += 2) {
-            ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
-            ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
-          }
-          p[u][v] = s0 + s1;
-        }
-      if constexpr (BFLY) {
-        float qv[NB];
-#pragma unroll
-        for (int i = 0; i < NB; ++i) qv[i] = p[i / V][i % V];
-#pragma unroll
-        for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
-          if (n > 1) {
-            const bool up = (gl & o) != 0;
-#pragma unroll
-            for (int i = 0; i < n / 2; ++i) {
-              const float send = up ? qv[i] : qv[i + n / 2];
-              const float keep = up ? qv[i + n / 2] : qv[i];
-              qv[i] = keep + __shfl_xor_sync(gmask, send, o);
-            }
-            n /= 2;
-          } else {
-            qv[0] += __shfl_xor_sync(gmask, qv[0], o);
-          }
-        }
-        const int er_ = k0 + bu;
-        const float sa = s_a[w][er_][bhead];
-        const float dz = fabsf(sa) * (qv[0] - sd[er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
-        dacc += dz;
-        if (bwriter) s_z[w][er_][bhead] = dz;
-      } else {
-        head_reduce<G, U, V, LPH>(p, gmask);
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int er_ = k0 + u;
-#pragma unroll
-          for (int v = 0; v < V; ++v) {
-            const float sa = s_a[w][er_][hv[v]];
-            const float dz = fabsf(sa) * (p[u][v] - sd[er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
-            derv[v] += dz;
-            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
-          }
-        }
-      }
-    };
-    for (int b = 0; b < nbt; b += 2) {
-      consume(ra, b * U);
-      if (b + 2 < nbt) {
-#pragma unroll
-        for (int u = 0; u < U; ++u) row_load(ra[u], (uint32_t)si[min((b + 2) * U + u, cnt - 1)]);
-      }
-      if (b + 1 < nbt) {
-        consume(rz, (b + 1) * U);
-        if (b + 3 < nbt) {
-#pragma unroll
-          for (int u = 0; u < U; ++u) row_load(rz[u], (uint32_t)si[min((b + 3) * U + u, cnt - 1)]);
-        }
-      }
-    }
-    __syncwarp();
-    if (valid) {
-      float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
-      if constexpr (HT == 4) {
-        reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
-      } else {
-        for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
-      }
-    }
-    if (base + G >= item.z) {  // last chunk of this source: finalise
-      if constexpr (BFLY) {
-        float dsum = dacc;
-#pragma unroll
-        for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o);
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          int src = gl;
-#pragma unroll
-          for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
-            const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
-            src = bit ? (src | o) : (src & ~o);
-          }
-          derv[v] = __shfl_sync(gmask, dsum, src);
-        }
-      }
-      if (item.w < 0) {
-        float *orow = a.gfeat + j * a.ldgf + gl * EPV;
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const float *arp = a.ar + (v * G + gl) * EPV;
-          float y[EPV];
-#pragma unroll
-          for (int k = 0; k < EPV; k += 4) {
-            const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
-            y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
-            y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-            if (!a.lp_partial)
-              *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
-          }
-          if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
-          if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
-        }
-      } else {
-        const int64_t slot = item.w;
-        float *pr = a.ws_bacc + slot * a.D + gl * EPV;
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-#pragma unroll
-          for (int k = 0; k < EPV; k += 4)
-            *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
-                make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
-          if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
-        }
-      }
-    }
-    if (!has_next) break;
-    cp_async_wait<0>();
-    __syncwarp();
-    item = nitem;
-    base = nbase;
-    q = nq;
-    buf = nb_;
-  }
-  cp_async_wait<0>();
-}
-
-// ---- a7, chunk-pipelined with a shared-memory ring (G = 32, H <= 4) ----
-// gat_bwd_src_pipe_kernel's staging of the next chunk (ids, el / lse / Dlt, er)
-// combined with gat_bwd_src_ring_kernel's cp.async ring for the g rows.
-// gat_bwd_src_kernel's arithmetic with the fwd pipe kernel's staging: while
-// chunk c runs, the next chunk's destination ids, their (el, lse, Dlt) and
-// (for a new source) er_j are staged in shared memory with cp.async, and the
-// next chunk's g rows and the next source's Wh row are prefetched into L2.
-template <typename T, int V, int HT, int NBF>
-__global__ void __launch_bounds__(TPB, 2) gat_bwd_src_pipering_kernel(const BwdArgs a) {
-  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
-  constexpr int U1 = V >= 4 ? 1 : (V == 2 ? 2 : 4), U = U1 < G ? U1 : G;
-  constexpr int NB = U * V;
-  constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
-  constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
-  extern __shared__ uint4 ring_all[];  // [WPB][NBF * U][V][32]
-  __shared__ float s_a[WPB][32][SP];  // alpha, sign bit = (z <= 0)
-  __shared__ float s_z[WPB][32][SP];  // dz out
-  __shared__ int4 s_desc[2][WPB][32];
-  __shared__ int s_i[2][WPB][32];     // packed destination rows of a chunk
-  __shared__ __align__(16) float s_el[2][WPB][32][HT];
-  __shared__ __align__(16) float s_ls[2][WPB][32][HT];
-  __shared__ __align__(16) float s_dl[2][WPB][32][HT];
-  __shared__ __align__(16) float s_er[2][WPB][HT];
-  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
-  const unsigned gmask = 0xffffffffu;
-  const int H = a.H;
-  const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
-  const uint32_t grow_bytes = (uint32_t)(a.D * sizeof(T));
-  int hv[V];
-#pragma unroll
-  for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
-  int bidx = 0;
-#pragma unroll
-  for (int s = 0, o = LPH >> 1; (1 << s) < NB; ++s, o >>= 1) bidx = 2 * bidx + ((gl & o) ? 1 : 0);
-  const int bu = bidx / V, bv = bidx % V;
-  const int bhead = ((bv * G + gl) * EPV) / FF;
-  const bool bwriter = (gl & (LPH / (NB > 0 ? NB : 1) - 1)) == 0;
-  const T *feat = static_cast<const T *>(a.feat);
-  const T *gout = static_cast<const T *>(a.gout);
-  const T *goutl = gout + gl * EPV;
-  const int64_t stride = (int64_t)gridDim.x * WPB;
-  const int64_t it0 = (int64_t)blockIdx.x * WPB + w, n_items = a.L.n_bwd_items;
-  if (it0 >= n_items) return;
-  uint4 *ring = ring_all + (size_t)w * NBF * U * V * 32;
-  // batch b of the current chunk -> ring slots (b % NBF) U ..; one cp.async group per batch (empty past the chunk)
-  auto issue = [&](const int *ids, int b, int cnt) {
-    if (b * U < cnt) {
-#pragma unroll
-      for (int u = 0; u < U; ++u) {
-        const uint32_t ii = (uint32_t)ids[min(b * U + u, cnt - 1)];
-        const T *rp = goutl + (ii & idm) * ldg;
-        const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
-        uint4 *dst = ring + (((b % NBF) * U + u) * V) * 32 + lane;
-#pragma unroll
-        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
-      }
-    }
-    cp_async_commit();
-  };
-  auto stage_desc = [&](int k) {
-    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
-    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][gl], a.L.bwd_items + itq);
-    cp_async_commit();
-  };
-  // chunk (itm, bse): destination ids; for the first chunk of a source its er, and its Wh row into L2
-  auto stage_ids = [&](int b, int4 itm, int bse) {
-    if (itm.z > itm.y) cp_async_small<4>(&s_i[b][w][gl], a.L.cdst + min(bse + gl, itm.z - 1));
-    else s_i[b][w][gl] = 0;
-    if (bse == itm.y && gl == 0) {
-      cp_async_h<HT>(&s_er[b][w][0], a.er + (int64_t)itm.x * H);
-      prefetch_l2_bulk(feat + (int64_t)itm.x * a.ldf, grow_bytes, pol_row);
-    }
-    cp_async_commit();
-  };
-  // the staged chunk's destination values, and its g rows into L2
-  auto stage_dst = [&](int b, int4 itm, int bse) {
-    const uint32_t ii = (uint32_t)s_i[b][w][gl];
-    const int64_t gi = a.L.row_begin + (int)(ii & idm);
-    cp_async_h<HT>(&s_el[b][w][gl][0], a.el + gi * H);
-    cp_async_h<HT>(&s_ls[b][w][gl][0], a.lse + gi * H);
-    cp_async_h<HT>(&s_dl[b][w][gl][0], a.dlt + gi * H);
-    cp_async_commit();
-    // the chunk's first pf_rows g rows into L2, one 128-byte line per lane per step
-    constexpr int LPR = (32 * V * 16) / 128, RPS = 32 / LPR;
-    const int cnt_n = min(a.pf_rows, itm.z - bse);
-    for (int r0 = 0; r0 < cnt_n; r0 += RPS) {
-      const int r = r0 + gl / LPR;
-      if (r < cnt_n)
-        prefetch_l2_line(reinterpret_cast<const char *>(gout + ((uint32_t)s_i[b][w][r] & idm) * ldg) + (gl % LPR) * 128);
-    }
-  };
-  stage_desc(0);
-  stage_desc(1);
-  cp_async_wait<1>();
-  __syncwarp();
-  int q = 0;
-  int4 item = s_desc[0][w][0];
-  int base = item.y, buf = 0;
-  stage_ids(0, item, base);
-  cp_async_wait<0>();
-  __syncwarp();
-  stage_dst(0, item, base);
-  cp_async_wait<0>();
-  __syncwarp();
-  float whf[V][EPV], acc[V][EPV], derv[V], erj[HT], dacc = 0.f;
-  while (true) {
-    int4 nitem = item;
-    int nbase = base + G;
-    int nq = q;
-    bool has_next = true;
-    if (nbase >= item.z) {
-      nq = q + 1;
-      if (it0 + (int64_t)nq * stride >= n_items) {
-        has_next = false;
-      } else {
-        if (nq % G == 0) {
-          cp_async_wait<0>();
-          __syncwarp();
-          nitem = s_desc[(nq / G) & 1][w][0];
-          __syncwarp();
-          stage_desc(nq / G + 1);
-        } else {
-          nitem = s_desc[(nq / G) & 1][w][nq % G];
-        }
-        nbase = nitem.y;
-      }
-    }
-    const int nb_ = buf ^ 1;
-    if (has_next) stage_ids(nb_, nitem, nbase);
-    const int64_t j = item.x;
-    if (base == item.y) {
-      const T *rp = feat + j * a.ldf + gl * EPV;
-#pragma unroll
-      for (int v = 0; v < V; ++v) {
-        unpack(ldg16(rp + v * G * EPV), whf[v], T());
-        derv[v] = 0.f;
-#pragma unroll
-        for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
-      }
-#pragma unroll
-      for (int h = 0; h < HT; ++h) erj[h] = s_er[buf][w][h];
-      dacc = 0.f;
-    }
-    const int *si = &s_i[buf][w][0];
-    const int c = base + gl;
-    const bool valid = c < item.z;
-    const int cp_c = item.z > item.y ? ld_stream(a.L.cpos + min(c, item.z - 1), policy_first()) : 0;
-    const int cnt = max(0, min(G, item.z - base)), nbt = (cnt + U - 1) / U;
-#pragma unroll
-    for (int b = 0; b < NBF; ++b) issue(si, b, cnt);
-#pragma unroll
-    for (int h = 0; h < HT; ++h)
-      if (h < H) {
-        const float z = s_el[buf][w][gl][h] + erj[h];
-        const float al = valid ? fexp(leaky(z, a.slope) - s_ls[buf][w][gl][h]) : 0.f;
-        s_a[w][lane][h] = z > 0.f ? al : -al;
-      }
-    cp_async_wait<NBF>();  // the next chunk's ids (older than the NBF ring groups) have landed
-    __syncwarp();
-    if (has_next) stage_dst(nb_, nitem, nbase);
-    else cp_async_commit();  // keep the group count uniform
-    const float(*sd)[HT] = s_dl[buf][w];
-    auto consume = [&](const uint4 *slot, int k0) {
-      float p[U][V];
-#pragma unroll
-      for (int u = 0; u < U; ++u)
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const float al = fabsf(s_a[w][k0 + u][hv[v]]);
-          float x[EPV];
-          unpack(slot[(u * V + v) * 32], x, T());
-          float s0 = 0.f, s1 = 0.f;
-#pragma unroll
-          for (int k = 0; k < EPV; k += 2) {
-            ffma2v(s0, s1, x[k], x[k + 1], whf[v][k], whf[v][k + 1]);
-            ffma2s(acc[v][k], acc[v][k + 1], x[k], x[k + 1], al);
-          }
-          p[u][v] = s0 + s1;
-        }
-      if constexpr (BFLY) {
-        float qv[NB];
-#pragma unroll
-        for (int i = 0; i < NB; ++i) qv[i] = p[i / V][i % V];
-#pragma unroll
-        for (int n = NB, o = LPH >> 1; o > 0; o >>= 1) {
-          if (n > 1) {
-            const bool up = (gl & o) != 0;
-#pragma unroll
-            for (int i = 0; i < n / 2; ++i) {
-              const float send = up ? qv[i] : qv[i + n / 2];
-              const float keep = up ? qv[i + n / 2] : qv[i];
-              qv[i] = keep + __shfl_xor_sync(gmask, send, o);
-            }
-            n /= 2;
-          } else {
-            qv[0] += __shfl_xor_sync(gmask, qv[0], o);
-          }
-        }
-        const int er_ = k0 + bu;
-        const float sa = s_a[w][er_][bhead];
-        const float dz = fabsf(sa) * (qv[0] - sd[er_][bhead]) * (signbit(sa) ? a.slope : 1.f);
-        dacc += dz;
-        if (bwriter) s_z[w][er_][bhead] = dz;
-      } else {
-        head_reduce<G, U, V, LPH>(p, gmask);
-#pragma unroll
-        for (int u = 0; u < U; ++u) {
-          const int er_ = k0 + u;
-#pragma unroll
-          for (int v = 0; v < V; ++v) {
-            const float sa = s_a[w][er_][hv[v]];
-            const float dz = fabsf(sa) * (p[u][v] - sd[er_][hv[v]]) * (signbit(sa) ? a.slope : 1.f);
-            derv[v] += dz;
-            if (head_lead<G, LPH>(gl, v)) s_z[w][er_][hv[v]] = dz;
-          }
-        }
-      }
-    };
-    for (int b = 0; b < nbt; ++b) {
-      cp_async_wait<NBF>();  // groups after batch b: NBF - 1 - b ring batches, the dst staging, b refills
-      consume(ring + ((b % NBF) * U * V) * 32 + lane, b * U);
-      issue(si, b + NBF, cnt);
-    }
-    __syncwarp();
-    if (valid) {
-      float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
-      if constexpr (HT == 4) {
-        reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
-      } else {
-        for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
-      }
-    }
-    if (base + G >= item.z) {  // last chunk of this source: finalise
-      if constexpr (BFLY) {
-        float dsum = dacc;
-#pragma unroll
-        for (int s = 0, o = LPH >> 1; s < UB; ++s, o >>= 1) dsum += __shfl_xor_sync(gmask, dsum, o);
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          int src = gl;
-#pragma unroll
-          for (int t = 0, o = LPH >> (1 + UB); (1 << t) < V; ++t, o >>= 1) {
-            const int bit = (v >> ((V == 2 ? 1 : (V == 4 ? 2 : 3)) - 1 - t)) & 1;
-            src = bit ? (src | o) : (src & ~o);
-          }
-          derv[v] = __shfl_sync(gmask, dsum, src);
-        }
-      }
-      if (item.w < 0) {
-        float *orow = a.gfeat + j * a.ldgf + gl * EPV;
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-          const float *arp = a.ar + (v * G + gl) * EPV;
-          float y[EPV];
-#pragma unroll
-          for (int k = 0; k < EPV; k += 4) {
-            const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
-            y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
-            y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-            if (!a.lp_partial)
-              *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
-          }
-          if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
-          if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
-        }
-      } else {
-        const int64_t slot = item.w;
-        float *pr = a.ws_bacc + slot * a.D + gl * EPV;
-#pragma unroll
-        for (int v = 0; v < V; ++v) {
-#pragma unroll
-          for (int k = 0; k < EPV; k += 4)
-            *reinterpret_cast<float4 *>(pr + v * G * EPV + k) =
-                make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
-          if (head_lead<G, LPH>(gl, v)) a.ws_bder[slot * H + hv[v]] = derv[v];
-        }
-      }
-    }
-    if (!has_next) break;
-    cp_async_wait<0>();
-    __syncwarp();
-    item = nitem;
-    base = nbase;
-    q = nq;
-    buf = nb_;
-  }
-  cp_async_wait<0>();
 }
 
 // Split sources: dWh_j = sum_k acc_k + der_j a_r, der_j = sum_k der_k.
@@ -1726,12 +997,8 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
       float *orow = a.gfeat + j * a.ldgf + col;
 #pragma unroll
       for (int k = 0; k < EPV; ++k) y[k] = fmaf(der, a.ar[col + k], y[k]);
-      if (a.lp_partial) {
-        st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + col, pack(y, T()));
-      } else {
 #pragma unroll
-        for (int k = 0; k < EPV; ++k) orow[k] = y[k];
-      }
+      for (int k = 0; k < EPV; ++k) orow[k] = y[k];
     }
   }
 }
@@ -1779,16 +1046,8 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       whp[v] = ldg16(wr + v * G * EPV);
-      if (a.lp_partial) {  // bf16 partial (one-call training path, k = 1)
-        float t[EPV];
-        unpack(*reinterpret_cast<const uint4 *>(static_cast<const T *>(a.gfeat_lp) + grow * a.ldlp +
-                                                 (v * G + gl) * EPV), t, T());
 #pragma unroll
-        for (int k = 0; k < EPV / 4; ++k) part[v][k] = make_float4(t[4 * k], t[4 * k + 1], t[4 * k + 2], t[4 * k + 3]);
-      } else {
-#pragma unroll
-        for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
-      }
+      for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
     }
     float derr[HT];
     load_h<HT>(a.der + grow * H, H, derr);
@@ -1865,6 +1124,30 @@ __global__ void __launch_bounds__(1024) param_reduce_kernel(const double *parts_
 #pragma unroll
     for (int k = 0; k < 32; ++k) t += sh[k][tx];
     out[d] = (float)t;
+  }
+}
+
+// k-GPU backward: add the peers' partial [dWh | der] of this
+// part's own rows (received into `stage`, one [rows][ld] block per peer) to
+// the local partial, peers in ascending order (fixed order: deterministic).
+__global__ void __launch_bounds__(256) dist_combine_kernel(float *gfeat, int64_t ldgf, float *der, const float *stage,
+                                                           const float *stage_der, int npeers, int64_t rows,
+                                                           int64_t row0, int D, int H) {
+  const int64_t nv = rows * (D / 4);
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / (D / 4), c = 4 * (i % (D / 4));
+    float4 *dst = reinterpret_cast<float4 *>(gfeat + (row0 + r) * ldgf + c);
+    float4 acc = *dst;
+    for (int q = 0; q < npeers; ++q) {
+      const float4 v = *reinterpret_cast<const float4 *>(stage + ((int64_t)q * rows + r) * ldgf + c);
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    *dst = acc;
+  }
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < rows * H; i += (int64_t)gridDim.x * blockDim.x) {
+    float acc = der[row0 * H + i];
+    for (int q = 0; q < npeers; ++q) acc += stage_der[(int64_t)q * rows * H + i];
+    der[row0 * H + i] = acc;
   }
 }
 
@@ -1972,15 +1255,8 @@ int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
   return c;
 }
 
-// cp.async ring kernels for wide rows (opt-in with MEGA_RING=1; the register-batch kernels measure faster)
-bool use_ring() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_RING");
-    v = (e && e[0] == '1') ? 1 : 0;
-  }
-  return v == 1;
-}
+// L2 policy of gathered rows (ablation knob MEGA_L2_POLICY): 0 = hot rows evict_last, the rest
+// evict_first (default); 1 = all evict_normal; 2 = hot evict_last, rest evict_normal
 int l2_policy_mode() {
   static int v = -1;
   if (v < 0) {
@@ -1988,50 +1264,6 @@ int l2_policy_mode() {
     v = e ? std::atoi(e) : 0;
   }
   return v;
-}
-// forward kernel: 3 = chunk-pipelined gat_fwd_pipe_kernel (default; products 3 layers: 25.5 vs 29.3 ms/step),
-// 0/1/2 = gat_fwd_kernel batch variants
-int fwd_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_FWD_VAR");
-    v = e ? std::atoi(e) : 3;
-  }
-  return v;
-}
-// edge-streaming TMA forward for wide rows (gat_stream.cu), opt-in with MEGA_FWD_STREAM=1: measured
-// 46.7 vs 29.2 ms/step for the fused kernel on products (3 layers)
-bool use_stream_fwd() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_FWD_STREAM");
-    v = (e && e[0] == '1') ? 1 : 0;
-  }
-  return v == 1;
-}
-int pf_rows() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_PF_ROWS");
-    v = e ? std::atoi(e) : 0;  // 0..32 rows measured within 1% (the staging of ids/el/er is what pays)
-  }
-  return v;
-}
-// source pass: 4 = gat_bwd_src_ring_kernel with 4 batches in flight (default where G = 32 and V <= 2;
-// products 3 layers: gat_bwd 60.5 -> 52.9 ms/step), 5 = the ring with 6 batches (56.6), 0 = register-batch
-// gat_bwd_src_kernel (the default elsewhere), 1 = its single-batch variant, 3 = gat_bwd_src_pipe_kernel (60.3),
-// 6 = gat_bwd_src_pipering_kernel (staged chain + ring: 49.7-50.1 vs 48.1 for 4; the staging costs more than it hides)
-int bwd_variant() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_BWD_VAR");
-    v = e ? std::atoi(e) : 4;
-  }
-  return v;
-}
-int ring_blocks(size_t smem) {
-  const size_t per_sm = 227 * 1024;
-  return (int)std::max<size_t>(1, per_sm / (smem + 12 * 1024));
 }
 
 mega_status check_launch(cudaStream_t s, const char *what) {
@@ -2086,15 +1318,14 @@ mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
   return MEGA_OK;
 }
 
-struct WsFwd { size_t m, l, acc, alpha, total; };
+struct WsFwd { size_t m, l, acc, total; };
 WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   WsFwd w;
   size_t slots = (size_t)std::max(1, D.n_fwd_slots);
   w.m = 0;
   w.l = align256(w.m + slots * s.H * 4);
   w.acc = align256(w.l + slots * s.H * 4);
-  w.alpha = align256(w.acc + slots * s.D * 4);
-  w.total = align256(w.alpha + (s.G == 32 ? (size_t)std::max<int64_t>(1, D.edges) * s.H * 4 : 0));
+  w.total = align256(w.acc + slots * s.D * 4);
   return w;
 }
 struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
@@ -2156,46 +1387,17 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
   mega_status rc = MEGA_OK;
   dispatch_gv(s.nv, [&](auto g, auto v) {
     constexpr int G = decltype(g)::value, V = decltype(v)::value;
-    if constexpr (G == 32) {
-      if (use_stream_fwd() && !use_ring()) {
-        rc = run_fwd_stream(a, s.nv, s.H, std::is_same<T, __nv_bfloat16>::value, st, dev_info(dev).sms);
-        return;
-      }
-    }
     if (a.L.n_fwd_items > 0) {
       dispatch_h(s.H, [&](auto ht) {
         constexpr int HT = decltype(ht)::value;
-        if constexpr (G == 32) {
-          if (use_ring()) {
-            constexpr int RB = 32 * V * 16;                       // bytes per row
-            constexpr int P = RB >= 4096 ? 1 : (RB >= 2048 ? 1 : (RB >= 1024 ? 3 : 6));  // <= 96 KB ring per CTA, 2 CTAs/SM
-            auto k = gat_fwd_ring_kernel<T, V, HT, P>;
-            const size_t smem = (size_t)WPB * 4 * P * RB;
-            static bool attr = false;
-            if (!attr) {
-              cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-              attr = true;
-            }
-            const int grid = (int)std::min<int64_t>((a.L.n_fwd_items + WPB - 1) / WPB,
-                                                    (int64_t)dev_info(dev).sms * ring_blocks(smem));
-            k<<<std::max(grid, 1), TPB, smem, st>>>(a);
-            rc = check_launch(st, "gat_fwd_ring_kernel");
-            return;
-          }
-        }
         auto launch = [&](auto kern_fn) {
           kern_fn<<<grid_for(kern_fn, a.L.n_fwd_items, 32 / G, dev), TPB, 0, st>>>(a);
           rc = check_launch(st, "gat_fwd_kernel");
         };
-        switch (fwd_variant()) {
-          case 3:
-            if constexpr (G >= 8) launch(gat_fwd_pipe_kernel<T, G, V, HT>);  // (narrow rows: static smem)
-            else launch(gat_fwd_kernel<T, G, V, HT, 0>);
-            break;
-          case 1: launch(gat_fwd_kernel<T, G, V, HT, 1>); break;
-          case 2: launch(gat_fwd_kernel<T, G, V, HT, 2>); break;
-          default: launch(gat_fwd_kernel<T, G, V, HT, 0>); break;
-        }
+        // chunk-pipelined kernel for groups of >= 8 lanes (products 3 layers: 25.5 vs 29.3 ms/step for the
+        // register-batch kernel, which stays for narrow rows: static shared memory of the pipe kernel)
+        if constexpr (G >= 8) launch(gat_fwd_pipe_kernel<T, G, V, HT>);
+        else launch(gat_fwd_kernel<T, G, V, HT, 0>);
       });
       if (rc != MEGA_OK) return;
     }
@@ -2209,7 +1411,7 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
 }
 
 template <typename T>
-mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, int dev) {
+mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, int dev, bool with_dlt = true) {
   mega_status rc = MEGA_OK;
   const uint32_t ph = flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST);
   const bool src_phase = ph == 0 || (ph & MEGA_BWD_PHASE_SRC);
@@ -2219,52 +1421,30 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
     dispatch_h(s.H, [&](auto ht) {
       constexpr int HT = decltype(ht)::value;
       if (src_phase) {
-        if (a.L.rows > 0) {
+        if (with_dlt && a.L.rows > 0) {
           auto k = dlt_kernel<T, G, V, HT>;
           k<<<grid_for(k, a.L.rows, 32 / G, dev), TPB, 0, st>>>(a);
           if ((rc = check_launch(st, "dlt_kernel")) != MEGA_OK) return;
         }
         if (a.L.n_bwd_items > 0) {
-          auto launch = [&](auto ks) { ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a); };
-          bool piped = false;
-          if constexpr (G == 32 && HT <= 4) {
-            if (bwd_variant() == 3) { launch(gat_bwd_src_pipe_kernel<T, V, HT>); piped = true; }
-            if constexpr (V <= 2) {
-              if (bwd_variant() == 6) {  // staged chain + shared-memory ring (4 batches in flight)
-                constexpr int U = V == 2 ? 2 : 4, NBF = 4;
-                auto kr = gat_bwd_src_pipering_kernel<T, V, HT, NBF>;
-                const size_t smem = (size_t)WPB * NBF * U * V * 32 * 16;
-                cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-                int nblk = 0;
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
-                const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
-                                                        (int64_t)dev_info(dev).sms * std::max(nblk, 1));
-                kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
-                piped = true;
-              }
-            }
-          }
+          bool ring = false;
           if constexpr (G == 32 && V <= 2) {
-            const int bv = bwd_variant();
-            if (bv == 4 || bv == 5) {  // shared-memory ring: 4 = 4 batches in flight, 5 = 6 batches
-              auto ring_launch = [&](auto kr, int nbf) {
-                constexpr int U = V == 2 ? 2 : 4;
-                const size_t smem = (size_t)WPB * nbf * U * V * 32 * 16;
-                cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-                int nblk = 0;
-                cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
-                const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
-                                                        (int64_t)dev_info(dev).sms * std::max(nblk, 1));
-                kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
-              };
-              if (bv == 4) ring_launch(gat_bwd_src_ring_kernel<T, V, HT, 4>, 4);
-              else ring_launch(gat_bwd_src_ring_kernel<T, V, HT, 6>, 6);
-              piped = true;
-            }
+            // shared-memory ring, 4 batches in flight (products 3 layers: gat_bwd 60.5 -> 52.9 ms/step)
+            constexpr int U = V == 2 ? 2 : 4, NBF = 4;
+            auto kr = gat_bwd_src_ring_kernel<T, V, HT, NBF>;
+            const size_t smem = (size_t)WPB * NBF * U * V * 32 * 16;
+            cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+            int nblk = 0;
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
+            const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
+                                                    (int64_t)dev_info(dev).sms * std::max(nblk, 1));
+            kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
+            ring = true;
           }
-          if (piped) {
-          } else if (bwd_variant() == 1) launch(gat_bwd_src_kernel<T, G, V, HT, 1>);
-          else launch(gat_bwd_src_kernel<T, G, V, HT, 0>);
+          if (!ring) {
+            auto ks = gat_bwd_src_kernel<T, G, V, HT, 0>;
+            ks<<<grid_for(ks, a.L.n_bwd_items, 32 / G, dev), TPB, 0, st>>>(a);
+          }
           if ((rc = check_launch(st, "gat_bwd_src_kernel")) != MEGA_OK) return;
         }
         if (a.L.n_bwd_splits > 0) {
@@ -2343,10 +1523,8 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.alpha = reinterpret_cast<float *>(wb + w.alpha);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
-  a.pf_rows = pf_rows();
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -2394,12 +1572,251 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
-  a.lp_partial = 0;  // bf16 partial measured no faster than the fp32 partial (latency-bound); kept off
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
-  a.pf_rows = pf_rows();
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
+}
+
+}  // extern "C"
+
+// ---------------- k-GPU path ----------------
+namespace mega {
+namespace {
+struct DistWs { size_t fwd, bwd_base, stage, stage_der, bwd_total; };
+DistWs dist_ws(const mega_layout *L, int32_t part, const Shape &s) {
+  const Part &P = L->parts[part];
+  DevPart D = host_counts(P, L->n);
+  int32_t nslots = P.n_d_slots;
+  if (L->parts.size() > 1 && P.dl_items.empty() && P.dr_items.empty()) {
+    std::vector<int32_t> a, b, c;
+    dist_items(L, part, a, b, c, nslots);
+  }
+  D.n_fwd_slots = std::max(D.n_fwd_slots, nslots);
+  DistWs w;
+  w.fwd = ws_fwd(D, s).total;
+  w.bwd_base = ws_bwd(D, s).total;
+  const size_t k1 = L->parts.size() - 1, rows = (size_t)(P.row_end - P.row_begin);
+  w.stage = w.bwd_base;
+  w.stage_der = align256(w.stage + k1 * rows * (size_t)s.D * 4);
+  w.bwd_total = align256(w.stage_der + k1 * rows * (size_t)s.H * 4);
+  return w;
+}
+bool phase_flags(uint32_t flags, bool &snd, bool &rcv) {
+  const uint32_t ph = flags & (MEGA_DIST_PHASE_SEND | MEGA_DIST_PHASE_RECV);
+  snd = ph == 0 || (ph & MEGA_DIST_PHASE_SEND);
+  rcv = ph == 0 || (ph & MEGA_DIST_PHASE_RECV);
+  return true;
+}
+mega_status check_comm(const mega_layout *L, int32_t part, mega_comm *c) {
+  if (!c) return fail(MEGA_ERR_INVALID_ARGUMENT, "null comm");
+  if (comm_size(c) != (int)L->parts.size())
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "comm size != layout num_parts");
+  if (comm_rank(c) != part) return fail(MEGA_ERR_INVALID_ARGUMENT, "part must equal the comm rank");
+  return MEGA_OK;
+}
+}  // namespace
+}  // namespace mega
+
+extern "C" {
+
+mega_status mega_gat_dist_workspace_bytes(const mega_layout *L, int32_t part, int heads, int head_dim, mega_dtype dtype,
+                                          size_t *fwd_ws, size_t *bwd_ws) {
+  clear_error();
+  if (!L || !fwd_ws || !bwd_ws) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
+  if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
+  Shape s;
+  mega_status rc = check_shape(heads, head_dim, dtype, s);
+  if (rc != MEGA_OK) return rc;
+  const DistWs w = dist_ws(L, part, s);
+  *fwd_ws = w.fwd;
+  *bwd_ws = w.bwd_total;
+  return MEGA_OK;
+}
+
+mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *comm, void *feat, int64_t ldf,
+                              const float *attn_l, const float *attn_r, int heads, int head_dim, mega_dtype dtype,
+                              float negative_slope, uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws,
+                              size_t ws_bytes, mega_stream_t stream, mega_stream_t comm_stream) {
+  clear_error();
+  int dev = 0;
+  mega_status rc = check_part(L, part, dev);
+  if (rc != MEGA_OK) return rc;
+  if ((rc = check_comm(L, part, comm)) != MEGA_OK) return rc;
+  if (L->parts.size() == 1)   // nothing to exchange
+    return mega_gat_fwd(L, part, feat, ldf, attn_l, attn_r, heads, head_dim, dtype, negative_slope,
+                        flags & MEGA_FLAG_ELER_IN_CTX, out, ldo, ctx, ws, ws_bytes, stream);
+  Shape s;
+  if ((rc = check_shape(heads, head_dim, dtype, s)) != MEGA_OK) return rc;
+  if (!feat || !attn_l || !attn_r || !out || !ctx || !ws) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  const int esz = dtype == MEGA_BF16 ? 2 : 4;
+  if (ldf < s.D || ldo < s.D || (ldf * esz) % 16 || (ldo * esz) % 16)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "ldf/ldo must be >= D and a multiple of 16 bytes");
+  if ((uint64_t)L->n * (uint64_t)ldf >= (1ULL << 32))
+    return fail(MEGA_ERR_UNSUPPORTED, "num_nodes * ldf must be < 2^32 elements (32-bit row offsets)");
+  if (!al16(feat) || !al16(out) || !al16(ctx) || !al16(ws)) return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
+  const Part &P = L->parts[part];
+  const DistWs dw = dist_ws(L, part, s);
+  if (ws_bytes < dw.fwd) return fail(MEGA_ERR_OUT_OF_MEMORY, "fwd workspace too small (mega_gat_dist_workspace_bytes)");
+  bool snd, rcv;
+  phase_flags(flags, snd, rcv);
+  cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
+  const int64_t n = L->n, plane = n * s.H, b0 = P.row_begin, rows = P.row_end - P.row_begin;
+  char *fb = static_cast<char *>(feat);
+  kern::FwdArgs a;
+  a.L = P.dev;
+  a.feat = feat; a.ldf = ldf;
+  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane;
+  a.H = s.H; a.F = s.F; a.D = s.D; a.slope = negative_slope;
+  a.out = out; a.ldo = ldo;
+  DevPart Dw = P.dev;
+  Dw.n_fwd_slots = std::max(P.dev.n_fwd_slots, P.dev.n_d_slots);
+  const WsFwd w = ws_fwd(Dw, s);
+  char *wb = static_cast<char *>(ws);
+  a.ws_m = reinterpret_cast<float *>(wb + w.m);
+  a.ws_l = reinterpret_cast<float *>(wb + w.l);
+  a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
+  a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
+  a.pol_mode = l2_policy_mode();
+  auto pass = [&](const int4 *items, int32_t nitems, const int32_t *splits, int32_t nsplits) {
+    kern::FwdArgs b = a;
+    b.L.fwd_items = items; b.L.n_fwd_items = nitems;
+    b.L.fwd_splits = splits; b.L.n_fwd_splits = nsplits;
+    return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(b, s, st, dev) : run_fwd<float>(b, s, st, dev);
+  };
+  const int k = (int)L->parts.size(), p = part;
+  std::vector<CommMsg> sends, recvs;
+  for (int q = 0; q < k; ++q) {
+    if (q == p) continue;
+    const int64_t q0 = L->bounds[q], qn = L->bounds[q + 1] - q0;
+    sends.push_back({q, 0, fb + b0 * ldf * esz, (size_t)(rows * ldf * esz)});
+    sends.push_back({q, 1, ctx + plane + b0 * s.H, (size_t)(rows * s.H * 4)});
+    recvs.push_back({q, 0, fb + q0 * ldf * esz, (size_t)(qn * ldf * esz)});
+    recvs.push_back({q, 1, ctx + plane + q0 * s.H, (size_t)(qn * s.H * 4)});
+  }
+  if (snd) {
+    if (!(flags & MEGA_FLAG_ELER_IN_CTX) && rows > 0) {   // el/er of the own rows (those we send)
+      rc = launch_eler_any(dtype, fb + b0 * ldf * esz, ldf, rows, b0, attn_l, attn_r, heads, head_dim, ctx, ctx + plane, st);
+      if (rc != MEGA_OK) return rc;
+    }
+    // [Wh | er] of the own rows to every peer on the comm stream, the peers' rows back ...
+    if ((rc = comm_exchange(comm, sends, recvs, st, cs, true, false)) != MEGA_OK) return rc;
+    // ... while block (p, p) (sources this rank owns) runs on the compute stream
+    if ((rc = pass(P.dev.dl_items, P.dev.n_dl_items, nullptr, 0)) != MEGA_OK) return rc;
+  }
+  if (rcv) {
+    if ((rc = comm_exchange(comm, sends, recvs, st, cs, false, true)) != MEGA_OK) return rc;
+    cudaError_t ce = cudaStreamWaitEvent(st, comm_done_event(comm), 0);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("wait comm: ") + cudaGetErrorString(ce));
+    // remote blocks, then the fixed-order merge of the rows split across passes / segments (KB7)
+    if ((rc = pass(P.dev.dr_items, P.dev.n_dr_items, nullptr, 0)) != MEGA_OK) return rc;
+    if ((rc = pass(nullptr, 0, P.dev.d_splits, P.dev.n_d_splits)) != MEGA_OK) return rc;
+  }
+  return MEGA_OK;
+}
+
+mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *comm, const void *feat, int64_t ldf,
+                              const float *attn_l, const float *attn_r, int heads, int head_dim, mega_dtype dtype,
+                              float negative_slope, uint32_t flags, const void *out, int64_t ldo, const void *grad_out,
+                              int64_t ldg, float *ctx, float *grad_feat, int64_t ldgf, void *grad_feat_lp,
+                              int64_t ldlp, float *grad_attn_l, float *grad_attn_r, void *ws, size_t ws_bytes,
+                              mega_stream_t stream, mega_stream_t comm_stream) {
+  clear_error();
+  int dev = 0;
+  mega_status rc = check_part(L, part, dev);
+  if (rc != MEGA_OK) return rc;
+  if ((rc = check_comm(L, part, comm)) != MEGA_OK) return rc;
+  if (L->parts.size() == 1)
+    return mega_gat_bwd(L, part, feat, ldf, attn_l, attn_r, heads, head_dim, dtype, negative_slope,
+                        flags & MEGA_BWD_LP_ONLY, out, ldo, grad_out, ldg, ctx, grad_feat, ldgf, grad_feat_lp, ldlp,
+                        grad_attn_l, grad_attn_r, ws, ws_bytes, stream);
+  Shape s;
+  if ((rc = check_shape(heads, head_dim, dtype, s)) != MEGA_OK) return rc;
+  if (!feat || !attn_l || !attn_r || !out || !grad_out || !ctx || !grad_feat || !grad_attn_l || !grad_attn_r || !ws)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  const int esz = dtype == MEGA_BF16 ? 2 : 4;
+  if (ldf < s.D || ldo < s.D || ldg < s.D || ldgf != s.D || (ldf * esz) % 16 || (ldo * esz) % 16 ||
+      (ldg * esz) % 16 || (ldgf * 4) % 16)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "leading dimensions must be >= D (ldgf == D) and multiples of 16 bytes");
+  if ((uint64_t)L->n * (uint64_t)std::max(ldf, ldg) >= (1ULL << 32))
+    return fail(MEGA_ERR_UNSUPPORTED, "num_nodes * ld must be < 2^32 elements (32-bit row offsets)");
+  if (grad_feat_lp && (ldlp < s.D || (ldlp * esz) % 16 || !al16(grad_feat_lp)))
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "grad_feat_lp: bad ld or alignment");
+  if (!al16(feat) || !al16(out) || !al16(grad_out) || !al16(ctx) || !al16(grad_feat) || !al16(ws) ||
+      !al16(attn_l) || !al16(attn_r))
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
+  const Part &P = L->parts[part];
+  const DistWs dw = dist_ws(L, part, s);
+  if (ws_bytes < dw.bwd_total) return fail(MEGA_ERR_OUT_OF_MEMORY, "bwd workspace too small (mega_gat_dist_workspace_bytes)");
+  bool snd, rcv;
+  phase_flags(flags, snd, rcv);
+  const int64_t plane = L->n * s.H, b0 = P.row_begin, rows = P.row_end - P.row_begin;
+  kern::BwdArgs a;
+  a.L = P.dev;
+  a.feat = feat; a.ldf = ldf; a.al = attn_l; a.ar = attn_r;
+  a.H = s.H; a.F = s.F; a.D = s.D; a.slope = negative_slope;
+  a.out = out; a.ldo = ldo; a.gout = grad_out; a.ldg = ldg;
+  a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane; a.dlt = ctx + 3 * plane; a.der = ctx + 4 * plane;
+  a.gfeat = grad_feat; a.ldgf = ldgf; a.gfeat_lp = grad_feat_lp; a.ldlp = ldlp;
+  const WsBwd w = ws_bwd(P.dev, s);
+  char *wb = static_cast<char *>(ws);
+  a.dz = reinterpret_cast<float *>(wb + w.dz);
+  a.ws_bacc = reinterpret_cast<float *>(wb + w.bacc);
+  a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
+  a.ws_dal = reinterpret_cast<double *>(wb + w.dal);
+  a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
+  a.gal = grad_attn_l; a.gar = grad_attn_r;
+  a.nb_dst = 0;
+  a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
+  a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
+  a.pol_mode = l2_policy_mode();
+  float *stage = reinterpret_cast<float *>(wb + dw.stage), *stage_der = reinterpret_cast<float *>(wb + dw.stage_der);
+  cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
+  // source-phase launches over a range of CSC items [i0, i1) and splits [s0, s1)
+  auto src_range = [&](int32_t i0, int32_t i1, int32_t s0, int32_t s1, bool dlt) {
+    kern::BwdArgs b = a;
+    b.L.bwd_items = P.dev.bwd_items + i0; b.L.n_bwd_items = std::max(0, i1 - i0);
+    b.L.bwd_splits = P.dev.bwd_splits + 3 * s0; b.L.n_bwd_splits = std::max(0, s1 - s0);
+    return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt)
+                              : run_bwd<float>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt);
+  };
+  const int k = (int)L->parts.size(), p = part;
+  std::vector<CommMsg> sends, recvs;
+  int slot = 0;
+  for (int q = 0; q < k; ++q) {
+    if (q == p) continue;
+    const int64_t q0 = L->bounds[q], qn = L->bounds[q + 1] - q0;
+    // this rank's partial [dWh | der] of q's rows -> q; q's partial of our rows -> stage slot
+    sends.push_back({q, 2, grad_feat + q0 * ldgf, (size_t)(qn * ldgf * 4)});
+    sends.push_back({q, 3, ctx + 4 * plane + q0 * s.H, (size_t)(qn * s.H * 4)});
+    recvs.push_back({q, 2, stage + (int64_t)slot * rows * ldgf, (size_t)(rows * ldgf * 4)});
+    recvs.push_back({q, 3, stage_der + (int64_t)slot * rows * s.H, (size_t)(rows * s.H * 4)});
+    ++slot;
+  }
+  const DevPart &D = P.dev;
+  if (snd) {
+    // Dlt, then the sources other ranks own (their partials travel while ours are computed)
+    if ((rc = src_range(0, D.bwd_own0, 0, D.bsplit_own0, true)) != MEGA_OK) return rc;
+    if ((rc = src_range(D.bwd_own1, D.n_bwd_items, D.bsplit_own1, D.n_bwd_splits, false)) != MEGA_OK) return rc;
+    if ((rc = comm_exchange(comm, sends, recvs, st, cs, true, false)) != MEGA_OK) return rc;
+    if ((rc = src_range(D.bwd_own0, D.bwd_own1, D.bsplit_own0, D.bsplit_own1, false)) != MEGA_OK) return rc;
+  }
+  if (rcv) {
+    if ((rc = comm_exchange(comm, sends, recvs, st, cs, false, true)) != MEGA_OK) return rc;
+    cudaError_t ce = cudaStreamWaitEvent(st, comm_done_event(comm), 0);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("wait comm: ") + cudaGetErrorString(ce));
+    if (k > 1 && rows > 0) {
+      const int64_t nv = rows * (s.D / 4);
+      const int blocks = (int)std::min<int64_t>((nv + 255) / 256, 4 * dev_info(dev).sms);
+      kern::dist_combine_kernel<<<std::max(blocks, 1), 256, 0, st>>>(grad_feat, ldgf, ctx + 4 * plane, stage, stage_der,
+                                                                     k - 1, rows, b0, s.D, s.H);
+      if ((rc = check_launch(st, "dist_combine_kernel")) != MEGA_OK) return rc;
+    }
+    rc = dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, MEGA_BWD_PHASE_DST, st, dev)
+                            : run_bwd<float>(a, s, MEGA_BWD_PHASE_DST, st, dev);
+    if (rc != MEGA_OK) return rc;
+  }
+  return MEGA_OK;
 }
 
 }  // extern "C"

@@ -1,5 +1,5 @@
 // Device helpers and kernel argument blocks shared by the attention kernels
-// (gat_kernels.cu, gat_stream.cu).  Internal to libmega.so.
+// (gat_kernels.cu).  Internal to libmega.so.
 #pragma once
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
@@ -288,10 +288,8 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
-  float *alpha;    // edge-streaming forward: [E_p][H] fp32 attention weights in CSR order
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
   int pol_mode; // MEGA_L2_POLICY
-  int pf_rows;  // gat_fwd_pipe_kernel: rows of the next chunk prefetched into L2 (MEGA_PF_ROWS)
 };
 
 struct BwdArgs {
@@ -316,14 +314,10 @@ struct BwdArgs {
   float *gal, *gar;
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
-  int lp_partial;  // ... and (both phases in one call) the source-phase partial lives in gfeat_lp too
-  int pf_rows;     // gat_bwd_src_pipe_kernel: g rows of the next chunk prefetched into L2 (MEGA_PF_ROWS)
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int pol_mode; // MEGA_L2_POLICY
 };
 
 }  // namespace kern
 
-// gat_stream.cu: the edge-streaming forward for rows of nv = 32..256 16-byte vectors
-mega_status run_fwd_stream(const kern::FwdArgs &a, int nv, int H, bool bf16, cudaStream_t st, int sms);
 }  // namespace mega

@@ -4,6 +4,7 @@
 #include <string>
 #include <vector>
 
+#include <cuda_runtime.h>
 #include <vector_types.h>
 
 #include "../../include/mega.h"
@@ -38,10 +39,22 @@ struct DevPart {
   uint32_t id_mask = 0x7fffffffu;
   int32_t n_fwd_items = 0, n_fwd_splits = 0, n_fwd_slots = 0;
   int32_t n_bwd_items = 0, n_bwd_splits = 0, n_bwd_slots = 0;
+  // k > 1 (destination-partitioned): the forward split by source owner.
+  // Local pass items read only this part's own source rows (block (p,p)); remote pass
+  // items the rest; rows with both (or long segments) go to slots merged by d_splits.
+  const int4 *dl_items = nullptr, *dr_items = nullptr;
+  const int32_t *d_splits = nullptr;
+  int32_t n_dl_items = 0, n_dr_items = 0, n_d_splits = 0, n_d_slots = 0;
+  // backward: items / splits of this part's own sources (rows [row_begin, row_end)) are the
+  // contiguous ranges [bwd_own0, bwd_own1) of bwd_items and [bsplit_own0, bsplit_own1) of bwd_splits
+  int32_t bwd_own0 = 0, bwd_own1 = 0, bsplit_own0 = 0, bsplit_own1 = 0;
 };
 
 struct Part {
   int64_t row_begin = 0, row_end = 0;
+  // k > 1 dist items (derived from indptr/src/bounds at bind time; host copies for the view)
+  std::vector<int32_t> dl_items, dr_items, d_splits;
+  int32_t n_d_slots = 0;
   std::vector<int32_t> indptr, src, eid, cindptr, cdst, cpos, csr2csc;
   std::vector<int32_t> fwd_items, fwd_splits, bwd_items, bwd_splits;
   int32_t n_fwd_slots = 0, n_bwd_slots = 0;
@@ -69,7 +82,22 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-constexpr int kImageArrays = 14;
+constexpr int kImageArrays = 17;
+// dist items of part p (k > 1): see DevPart; S = the layout's segment size
+void dist_items(const mega_layout *L, int part, std::vector<int32_t> &local, std::vector<int32_t> &remote,
+                std::vector<int32_t> &splits, int32_t &nslots);
+// comm.cpp: one exchange of (peer, pointer, bytes) messages (see mega_comm)
+struct CommMsg { int peer; int tag; const void *ptr; size_t bytes; };
+}  // namespace mega
+struct mega_comm;
+namespace mega {
+int comm_rank(const mega_comm *c);
+int comm_size(const mega_comm *c);
+int comm_device(const mega_comm *c);
+bool comm_is_local(const mega_comm *c);
+mega_status comm_exchange(mega_comm *c, const std::vector<CommMsg> &sends, const std::vector<CommMsg> &recvs,
+                          cudaStream_t ready_on, cudaStream_t cs, bool phase_send, bool phase_recv);
+cudaEvent_t comm_done_event(mega_comm *c);
 // Edge tiles of the streaming kernels: consecutive unsplit work items are
 // merged while their edges stay contiguous and total <= kTileEdges; a split
 // segment (slot >= 0) is a tile of its own; rows without edges are skipped.

@@ -5,20 +5,24 @@ The exact counterpart of the paper's "partition of the path representation
 rank p owns the contiguous, edge-balanced rows [b_p, b_{p+1}) of the MEGA
 order (R23) and part p of the layout (its in-edges, every source).
 
-Per layer and step (torch.distributed over NCCL is the plumbing; every
-computation is a libmega.so call):
-  forward   mega_project_fwd on the owned rows -> all-gather-v of the projected
-            rows [Wh | er] (grouped send/recv: partitions are unequal and NCCL
-            has no all-gather-v) -> mega_gat_fwd on part p;
-  backward  mega_gat_bwd(PHASE_SRC) -> partial dWh and der for every source ->
-            reduce of each owner's row block onto its owner -> mega_gat_bwd
-            (PHASE_DST) on the owned rows -> mega_project_bwd on the owned rows
-            -> all-reduce of dW, da_l, da_r.
-The exchange helpers are also exercised on CPU with gloo (tests/test_dist_cpu.py).
+Per layer and step, every computation and every byte of the exchange is a
+libmega.so call on a library-owned communicator (include/mega.h "k GPUs"):
+  forward   mega_project_fwd on the owned rows -> mega_gat_fwd_dist: the
+            [Wh | er] rows travel to every peer on a comm stream while block
+            (p,p) is aggregated, then the remote blocks and the merge;
+  backward  mega_gat_bwd_dist: partial [dWh | der] of the peers' sources travel
+            to their owners while this rank's own sources are processed, then
+            the destination pass -> mega_project_bwd on the owned rows.
+torch.distributed is the plumbing only: it broadcasts the 128-byte NCCL id
+that bootstraps the library's communicator, and all-reduces the parameter
+gradients (dW, da_l, da_r) as data-parallel training does.
+
+allgather_rows / reduce_to_owners are the same exchange written with
+torch.distributed point-to-point ops; the CPU (gloo) test uses them to check
+the partition semantics against the oracle without a GPU.
 """
 from __future__ import annotations
 
-import numpy as np
 import torch
 import torch.distributed as dist
 
@@ -65,38 +69,71 @@ def reduce_to_owners(t: torch.Tensor, bounds, group=None):
                         op=dist.ReduceOp.SUM, group=group)
 
 
+def make_comm(group=None) -> M.Comm:
+    """Bootstrap the library-owned NCCL communicator from the torch process group:
+    rank 0 draws the unique id, torch broadcasts it, every rank joins."""
+    world, rank = dist.get_world_size(group), dist.get_rank(group)
+    obj = [M.mega_comm_unique_id() if rank == 0 else None]
+    dist.broadcast_object_list(obj, src=dist.get_global_rank(group, 0) if group is not None else 0, group=group)
+    return M.mega_comm_init(obj[0], world, rank, torch.cuda.current_device())
+
+
 class DistGATLayer:
-    """One GAT layer on part `rank` of a k-part layout."""
+    """One GAT layer on part `rank` of a k-part layout (k = 1: the single-GPU layer)."""
 
     def __init__(self, layout: M.Layout, rank, x_local, w, attn_l, attn_r, heads, head_dim, in_dim=None,
-                 want_grad_x=False, group=None, lp_only=False):
+                 want_grad_x=False, group=None, lp_only=False, comm: M.Comm | None = None):
         self.group = group
-        self.bounds = layout.view(rank)["bounds"]
+        self.rank = rank
+        self.k = layout.view(rank, arrays=False)["num_parts"]
+        self.comm = comm
+        if self.k > 1 and comm is None:
+            raise ValueError("a k-part layout needs a mega communicator (dist.make_comm)")
         self.L = GATLayer(layout, x_local, w, attn_l, attn_r, heads, head_dim, part=rank, in_dim=in_dim,
                           want_grad_x=want_grad_x, lp_only=lp_only)
+        if self.k > 1:
+            L = self.L
+            fws, bws = M.mega_gat_dist_workspace_bytes(layout, rank, heads, head_dim, M._dtype_code(x_local))
+            L.ws_f = torch.empty(max(fws, 256), dtype=torch.uint8, device=x_local.device)
+            L.ws_b = torch.empty(max(bws, 256), dtype=torch.uint8, device=x_local.device)
+            self.cs = torch.cuda.Stream(device=x_local.device)
+        # parameter gradients all-reduced in one flat buffer
+        L = self.L
+        self._pg = [L.grad_w, L.grad_attn_l, L.grad_attn_r]
 
     def forward(self, timed=None):
         """timed(name, fn): optional wrapper used by bench.py to time each call."""
         L = self.L
         t = timed or (lambda name, fn: fn())
         t("project_fwd", L.project)
-        t("comm_fwd", lambda: (allgather_rows(L.feat, self.bounds, self.group),
-                               allgather_rows(L.ctx[1], self.bounds, self.group)))  # [Wh | er] rows
-        t("gat_fwd", lambda: L.attend(True))
+        if self.k == 1:
+            t("gat_fwd", lambda: L.attend(True))
+        else:   # exchange of [Wh | er] overlapped with block (p, p), remote blocks, merge
+            t("gat_fwd", lambda: M.mega_gat_fwd_dist(L.layout, self.rank, self.comm, L.feat, L.attn_l, L.attn_r, L.H,
+                                                     L.F, L.out, L.ctx, L.ws_f, L.slope, M.MEGA_FLAG_ELER_IN_CTX,
+                                                     comm_stream=self.cs))
         return L.out
 
     def backward(self, grad_out_local, timed=None):
         L = self.L
         t = timed or (lambda name, fn: fn())
-        if _world(self.group) == 1:  # one call: lets LP_ONLY keep the partial in the bf16 operand
+        if self.k == 1:   # one call: lets LP_ONLY keep the partial in the bf16 operand
             t("gat_bwd", lambda: L.attend_backward(grad_out_local, 0))
         else:
-            t("gat_bwd_src", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_SRC))
-            t("comm_bwd", lambda: (reduce_to_owners(L.grad_feat, self.bounds, self.group),
-                                   reduce_to_owners(L.ctx[4], self.bounds, self.group)))  # [dWh | der]
-            t("gat_bwd_dst", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_DST))
+            flags = M.MEGA_BWD_LP_ONLY if (L.lp_only and L.grad_feat_lp is not None) else 0
+            t("gat_bwd", lambda: M.mega_gat_bwd_dist(L.layout, self.rank, self.comm, L.feat, L.attn_l, L.attn_r, L.H,
+                                                     L.F, L.out, grad_out_local, L.ctx, L.grad_feat, L.grad_attn_l,
+                                                     L.grad_attn_r, L.ws_b, L.grad_feat_lp, L.slope, flags,
+                                                     comm_stream=self.cs))
         t("project_bwd", L.project_backward)
         if _world(self.group) > 1:
-            for x in (L.grad_w, L.grad_attn_l, L.grad_attn_r):
-                dist.all_reduce(x, group=self.group)
+            t("allreduce_params", self._allreduce_params)
         return L.grad_x
+
+    def _allreduce_params(self):
+        flat = torch.cat([p.reshape(-1) for p in self._pg])
+        dist.all_reduce(flat, group=self.group)
+        off = 0
+        for p in self._pg:
+            p.copy_(flat[off:off + p.numel()].view_as(p))
+            off += p.numel()

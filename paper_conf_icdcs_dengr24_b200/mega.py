@@ -22,6 +22,8 @@ MEGA_CTX_PLANES = 5  # el, er, lse, Dlt, der
 MEGA_BWD_PHASE_SRC = 2
 MEGA_BWD_PHASE_DST = 4
 MEGA_BWD_LP_ONLY = 8
+MEGA_DIST_PHASE_SEND = 16
+MEGA_DIST_PHASE_RECV = 32
 SLOPE = float(np.float32(0.2))
 
 _c = ctypes
@@ -57,6 +59,13 @@ _VIEW_INTS = ("num_nodes", "num_edges", "row_begin", "row_end", "part_edges", "n
               "num_bwd_items", "num_bwd_splits", "num_parts")
 _VIEW_PTRS = ("perm", "new_of_old", "bounds", "indptr", "src", "eid", "cindptr", "cdst", "cpos", "csr2csc",
               "fwd_items", "fwd_splits", "bwd_items", "bwd_splits")
+
+
+class mega_layout_dist_view(_c.Structure):
+    _fields_ = [("struct_size", _c.c_uint32)] + [(k, _c.c_int64) for k in (
+        "num_local_items", "num_remote_items", "num_splits", "num_slots", "bwd_own_items_begin", "bwd_own_items_end",
+        "bwd_own_splits_begin", "bwd_own_splits_end")] + [(k, _c.POINTER(_c.c_int32)) for k in (
+        "local_items", "remote_items", "splits")]
 
 
 class mega_layout_view(_c.Structure):
@@ -98,6 +107,17 @@ def lib():
             "mega_project_workspace_bytes": (S, [I64, _c.c_int, _c.c_int, _c.c_int, S, P]),
             "mega_project_bwd": (S, [P, I64, I64, _c.c_int, P, _c.c_int, _c.c_int, S, P, I64, P, I64, P, P,
                                      _c.c_size_t, P]),
+            "mega_layout_dist_view_get": (S, [P, _c.c_int32, P]),
+            "mega_comm_unique_id": (S, [P]),
+            "mega_comm_init": (S, [P, _c.c_int, _c.c_int, _c.c_int, P]),
+            "mega_comm_init_local": (S, [_c.c_int, P, P]),
+            "mega_comm_destroy": (None, [P]),
+            "mega_comm_info": (S, [P, P, P, P, P]),
+            "mega_gat_dist_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, _c.c_int, S, P, P]),
+            "mega_gat_fwd_dist": (S, [P, _c.c_int32, P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32,
+                                      P, I64, P, P, _c.c_size_t, P, P]),
+            "mega_gat_bwd_dist": (S, [P, _c.c_int32, P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32,
+                                      P, I64, P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P, P]),
             "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P]),
             "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, P]),
             "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P, I64, P, P, P, I64,
@@ -289,6 +309,92 @@ def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_d
                                   dt, _ptr(grad_feat), grad_feat.stride(0), _ptr(grad_x),
                                   grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _ptr(ws),
                                   0 if ws is None else ws.numel() * ws.element_size(), _stream(stream)))
+
+
+# ---------------- k GPUs (include/mega.h "k GPUs: destination partitions") ----------------
+def mega_layout_dist_view_get(layout: Layout, part: int = 0) -> dict:
+    """Host copy of the k-GPU work split of one part (local / remote forward items, merge records,
+    own-source ranges of the backward items)."""
+    v = mega_layout_dist_view()
+    _check(lib().mega_layout_dist_view_get(layout.handle, part, _c.byref(v)))
+    d = {k: getattr(v, k) for k, _ in mega_layout_dist_view._fields_[1:9]}
+    for k, w, n in (("local_items", 4, v.num_local_items), ("remote_items", 4, v.num_remote_items),
+                    ("splits", 3, v.num_splits)):
+        ptr = getattr(v, k)
+        d[k] = (np.ctypeslib.as_array(ptr, shape=(n * w,)).copy() if n > 0 else np.zeros(0, np.int32)).reshape(-1, w)
+    return d
+
+
+class Comm:
+    """Owns a mega_comm* (library-owned communicator)."""
+
+    def __init__(self, handle):
+        self._h = _c.c_void_p(handle)
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.mega_comm_destroy(self._h)
+            self._h = _c.c_void_p(None)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self):
+        a, b, c, d = _c.c_int(), _c.c_int(), _c.c_int(), _c.c_int()
+        _check(lib().mega_comm_info(self._h, _c.byref(a), _c.byref(b), _c.byref(c), _c.byref(d)))
+        return {"nranks": a.value, "rank": b.value, "device": c.value, "transport": ("nccl", "local")[d.value]}
+
+
+def mega_comm_unique_id() -> bytes:
+    buf = (_c.c_uint8 * 128)()
+    _check(lib().mega_comm_unique_id(buf))
+    return bytes(buf)
+
+
+def mega_comm_init(uid: bytes, nranks: int, rank: int, device: int) -> Comm:
+    assert len(uid) == 128
+    buf = (_c.c_uint8 * 128).from_buffer_copy(uid)
+    h = _c.c_void_p()
+    _check(lib().mega_comm_init(buf, nranks, rank, device, _c.byref(h)))
+    return Comm(h.value)
+
+
+def mega_comm_init_local(nranks: int, devices=None):
+    """LOCAL transport: all ranks in this process -> list of Comm."""
+    out = (_c.c_void_p * nranks)()
+    devs = None if devices is None else (_c.c_int * nranks)(*devices)
+    _check(lib().mega_comm_init_local(nranks, devs, out))
+    return [Comm(out[r]) for r in range(nranks)]
+
+
+def mega_gat_dist_workspace_bytes(layout: Layout, part: int, heads: int, head_dim: int, dtype: int):
+    f, b = _c.c_size_t(), _c.c_size_t()
+    _check(lib().mega_gat_dist_workspace_bytes(layout.handle, part, heads, head_dim, dtype, _c.byref(f),
+                                               _c.byref(b)))
+    return f.value, b.value
+
+
+def mega_gat_fwd_dist(layout: Layout, part, comm: Comm, feat, attn_l, attn_r, heads, head_dim, out, ctx, ws,
+                      negative_slope=SLOPE, flags=0, stream=None, comm_stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_gat_fwd_dist(layout.handle, part, comm.handle, _ptr(feat), feat.stride(0), _ptr(attn_l),
+                                   _ptr(attn_r), heads, head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0),
+                                   _ptr(ctx), _ptr(ws), ws.numel() * ws.element_size(), _stream(stream),
+                                   _stream(comm_stream)))
+
+
+def mega_gat_bwd_dist(layout: Layout, part, comm: Comm, feat, attn_l, attn_r, heads, head_dim, out, grad_out, ctx,
+                      grad_feat, grad_attn_l, grad_attn_r, ws, grad_feat_lp=None, negative_slope=SLOPE, flags=0,
+                      stream=None, comm_stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_gat_bwd_dist(layout.handle, part, comm.handle, _ptr(feat), feat.stride(0), _ptr(attn_l),
+                                   _ptr(attn_r), heads, head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0),
+                                   _ptr(grad_out), grad_out.stride(0), _ptr(ctx), _ptr(grad_feat),
+                                   grad_feat.stride(0), _ptr(grad_feat_lp),
+                                   grad_feat_lp.stride(0) if grad_feat_lp is not None else 0, _ptr(grad_attn_l),
+                                   _ptr(grad_attn_r), _ptr(ws), ws.numel() * ws.element_size(), _stream(stream),
+                                   _stream(comm_stream)))
 
 
 # NEXT-3: Graph Transformer edge attention (include/mega.h mega_gt_*; fp32)

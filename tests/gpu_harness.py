@@ -115,7 +115,7 @@ def assert_bf16_close(got, ref, name, extra=None):
     assert np.array_equal(fin, np.isfinite(got)), f"{name}: finiteness differs"
     scale = np.max(np.abs(ref[fin])) if fin.any() else 0.0
     err = np.abs(got[fin] - ref[fin])
-    tol = 2e-2 * scale + (0.0 if extra is None else np.asarray(extra, np.float64)[fin])
+    tol = 2e-2 * scale + (0.0 if extra is None else np.asarray(extra, np.float64).reshape(ref.shape)[fin])
     bad = err > tol
     assert not bad.any(), (f"{name}: {bad.sum()} elements out of tolerance, max err {err.max():.3e} "
                            f"(2e-2 * {scale:.3e}{'' if extra is None else ' + derived bound'})")
@@ -166,6 +166,18 @@ def dlt_bf16_bound(ip, ix, Wh, a_l, a_r, g, slope=M.SLOPE):
     aW = np.abs(Wh)
     return {"grad_attn_l": np.abs(b_r["grad_attn_l"] - b["grad_attn_l"]) + np.einsum("nh,nhf->hf", ddel, aW),
             "grad_attn_r": np.abs(b_r["grad_attn_r"] - b["grad_attn_r"]) + np.einsum("nh,nhf->hf", dder, aW)}
+
+
+def assert_fp32_close_reduction(got, ref, name):
+    """fp32 bar for the parameter gradients (DESIGN.md R-tol): they are sums over all N
+    rows of terms whose own fp32 relative error is ~1e-6 (exp/log chains), so the
+    relative part is taken against the tensor's scale: |d| <= 1e-4 + 1e-5 max|ref|
+    (tests/test_tolerance_fp32.py shows the elementwise form is out of reach for fp32)."""
+    got = np.asarray(got, np.float64)
+    ref = np.asarray(ref, np.float64)
+    err = np.abs(got - ref)
+    tol = 1e-4 + 1e-5 * np.max(np.abs(ref))
+    assert np.all(err <= tol), f"{name}: max err {err.max():.3e} > {tol:.3e}"
 
 
 REDUCTIONS = ("grad_attn_l", "grad_attn_r", "grad_w")

@@ -68,3 +68,27 @@ def test_gpu_arm_batch_cuda_graph():
     c = d["config"]
     assert c["cuda_graph"] is True and c["batch"] == "zinc" and c["num_graphs"] == 64
     assert c["l2"].startswith("L2 flushed")
+
+
+def test_gpus_n_relaunches_as_n_ranks(monkeypatch):
+    """--gpus N outside torchrun re-launches bench.py as N ranks (one per GPU), and
+    refuses loudly when fewer than N devices are visible."""
+    import bench
+    cmd = bench.launch_cmd(["--gpus", "2", "--steps", "3"], 2, 29999)
+    assert cmd[1:3] == ["-m", "torch.distributed.run"] and "--nproc-per-node=2" in cmd
+    assert cmd[-4:] == [os.path.join(ROOT, "bench.py"), "--gpus", "2", "--steps", "3"][-4:]
+    assert "127.0.0.1" in cmd
+    monkeypatch.delenv("WORLD_SIZE", raising=False)
+    import torch
+    monkeypatch.setattr(torch.cuda, "device_count", lambda: 1)
+    import argparse
+    ns = argparse.Namespace(impl="mega", gpus=2)
+    with pytest.raises(SystemExit) as e:
+        bench.maybe_spawn(ns, ["--gpus", "2"])
+    assert "only 1 CUDA device" in str(e.value)
+    calls = []
+    monkeypatch.setattr(torch.cuda, "device_count", lambda: 2)
+    monkeypatch.setattr(bench.subprocess, "run", lambda c: calls.append(c) or type("R", (), {"returncode": 0})())
+    with pytest.raises(SystemExit) as e:
+        bench.maybe_spawn(ns, ["--gpus", "2"])
+    assert e.value.code == 0 and "--nproc-per-node=2" in calls[0]

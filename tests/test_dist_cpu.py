@@ -115,3 +115,36 @@ def test_partitioned_layer_equals_single_process(world):
     for rank, ok_out, ok_gf, ok_al, ok_ar, rows, edges in res:
         assert ok_out and ok_gf and ok_al and ok_ar, (rank, ok_out, ok_gf, ok_al, ok_ar)
         assert rows > 0 and edges > 0
+
+
+def _subgroup_worker(rank, world, port, q):
+    """allgather_rows on a subgroup whose group ranks differ from the global ranks."""
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        sub = dist.new_group([1, 2])
+        if rank in (1, 2):
+            gr = dist.get_rank(sub)            # 0 or 1
+            bounds = [0, 3, 7]
+            t = torch.zeros(7, 2)
+            t[bounds[gr]:bounds[gr + 1]] = float(rank)
+            D.allgather_rows(t, bounds, group=sub)
+            ok = torch.equal(t[:3], torch.full((3, 2), 1.0)) and torch.equal(t[3:], torch.full((4, 2), 2.0))
+            q.put((rank, ok))
+        dist.barrier()
+    finally:
+        dist.destroy_process_group()
+
+
+def test_allgather_rows_on_a_subgroup():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_subgroup_worker, args=(r, 3, port, q)) for r in range(3)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=300) for _ in range(2)]
+    for p in procs:
+        p.join(timeout=60)
+    assert all(p.exitcode == 0 for p in procs)
+    assert all(ok for _, ok in res), res
