@@ -116,24 +116,83 @@ def peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "source": "fallback (B200_PROFILING.md)"}
 
 
-def algorithmic_bytes(call, n, m, H, D, sb, rows=None):
-    """Compulsory HBM bytes per launch of each library call:
-    every gathered row counted once (perfect on-chip reuse), per-edge streams once."""
-    rows = n if rows is None else rows
+def floor_bytes(kernel, rows, N, E, H, D, sb, R=None):
+    """SURVEY §8(d)-d3 algorithmic bytes of one launch group, with R row fetches of the
+    gathered operand (R = N: the compulsory floor, every gathered row once; R = E: no
+    reuse).  bf16/fp32 storage sb, out in storage type, fp32 dWh, int32 indices.
+      KB2      B_fwd = 4E + R (D sb + 4H) + rows (8 + 8H + D sb)
+      KB3+KB4  N (2D sb + 4H) + 4E(1+H) + R (D sb + 12H) + N (8 + D sb + 8H + 4D)
+      KB5      4E(1+H) + N (8 + 8D + 4H + D sb)
+    (rows = destination rows of the part; N = rows at k = 1)."""
+    R = N if R is None else R
+    if kernel == "KB2":
+        return 4 * E + R * (D * sb + 4 * H) + rows * (8 + 8 * H + D * sb)
+    if kernel == "KB3+KB4":
+        return rows * (2 * D * sb + 4 * H) + 4 * E * (1 + H) + R * (D * sb + 12 * H) + N * (8 + D * sb + 8 * H + 4 * D)
+    if kernel == "KB5":
+        return 4 * E * (1 + H) + rows * (8 + 8 * D + 4 * H + D * sb)
+    raise KeyError(kernel)
+
+
+def design_bytes(kernel, rows, N, E, H, D, sb):
+    """The design's own compulsory bytes (LP_ONLY training path): what these
+    kernels must move given the layout (16-byte work items, the cpos map, dz in CSR order,
+    the bf16 projection operand written instead of fp32 dWh)."""
     items = 16 * rows
-    if call == "gat_fwd":     # KB2 (+KB7): idx, items, Wh, er, el, out, lse
-        return 4 * m + items + n * D * sb + n * H * 4 + rows * H * 4 + rows * D * sb + rows * H * 4
-    if call == "gat_bwd_src":  # KB3 + KB4 (+merge): g,out -> Dlt; cdst, items, Wh, er, g_i, el/lse/Dlt, dz, dWh
-        return (2 * rows * D * sb + rows * H * 4) + (4 * m + 16 * n + n * D * sb + n * H * 4 + rows * D * sb
-                                                    + 3 * rows * H * 4 + 4 * m * H + n * D * 4)
-    if call == "gat_bwd_dst":  # KB5: indptr, csr2csc, dz, dWh RMW, Wh, bf16 copy
-        return 4 * (rows + 1) + 4 * m + 4 * m * H + 2 * rows * D * 4 + rows * D * sb + (rows * D * sb if sb == 2 else 0)
-    if call == "gat_bwd":      # one call, LP_ONLY (bf16): KB3 + KB4 + KB5 with the partial kept in bf16
+    if kernel == "KB2":   # idx, items, Wh, er (all sources once), el, out, lse
+        return 4 * E + items + N * D * sb + N * H * 4 + rows * H * 4 + rows * D * sb + rows * H * 4
+    if kernel == "KB3+KB4":   # g,out -> Dlt; cdst, cpos, items, Wh, er, g_i, el/lse/Dlt, dz, dWh, der
+        return ((2 * rows * D * sb + rows * H * 4) + (8 * E + 16 * N + N * D * sb + N * H * 4 + rows * D * sb
+                                                       + 3 * rows * H * 4 + 4 * E * H + N * D * 4 + N * H * 4))
+    if kernel == "KB5":   # indptr, dz, dWh partial, der, Wh, bf16 operand
         pb = sb if sb == 2 else 4
-        return ((2 * rows * D * sb + rows * H * 4)
-                + (4 * m + 16 * n + n * D * sb + n * H * 4 + rows * D * sb + 3 * rows * H * 4 + 4 * m * H + n * D * pb)
-                + (4 * (rows + 1) + 4 * m + 4 * m * H + 2 * rows * D * pb + rows * D * sb + rows * H * 4))
-    raise KeyError(call)
+        return 4 * (rows + 1) + 4 * E * H + rows * D * 4 + rows * H * 4 + rows * D * sb + rows * D * pb
+    raise KeyError(kernel)
+
+
+# kernel-name prefixes (ncu launch list) of each launch group
+GROUPS = {"KB2": ("gat_fwd",), "KB3+KB4": ("dlt_kernel", "gat_bwd_src"), "KB5": ("gat_bwd_dst", "param_reduce"),
+          "proj_fwd": ("umma_gemm_kernel<0",), "proj_bwd": ("umma_gemm_kernel<1", "umma_gemm_kernel<2", "dw_reduce")}
+
+
+def ncu_launch_summary(path):
+    """Per launch group: mean DRAM bytes, ncu duration and tensor-pipe % per call, from an
+    ncu --csv launch list (scripts/gpu_prof_r02.sh).  Each kernel type of a group is
+    launched once per call, so a group's per-call figure is the sum of its kernels' means."""
+    import csv
+    if not os.path.exists(path):
+        return None
+    per = {}
+    with open(path) as f:
+        lines = [ln for ln in f if ln.startswith('"')]
+    for row in csv.DictReader(lines):
+        name = row.get("Kernel Name", "")
+        full = name.split("(")[0].replace("void ", "")
+        head = full.split("<")[0]
+        short = head.split("::")[-1] + full[len(head):]     # namespaces dropped, template args kept
+        d = per.setdefault(short, {})
+        try:
+            v = float(row["Metric Value"].replace(",", ""))
+        except (KeyError, ValueError):
+            continue
+        unit = row.get("Metric Unit", "")
+        v *= {"Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "usecond": 1e3, "msecond": 1e6, "second": 1e9}.get(unit, 1.0)
+        d.setdefault(row["Metric Name"], []).append(v)
+    out = {}
+    for g, pref in GROUPS.items():
+        ks = [k for k in per if any(k.startswith(p) for p in pref)]
+        if not ks:
+            continue
+        mean = lambda k, m: float(np.mean(per[k].get(m, [0.0])))   # noqa: E731
+        dur_unit = 1e-6   # gpu__time_duration in ns (ncu default "nsecond")
+        out[g] = {"dram_bytes": sum(mean(k, "dram__bytes_read.sum") + mean(k, "dram__bytes_write.sum") for k in ks),
+                  "ncu_ms": sum(mean(k, "gpu__time_duration.sum") for k in ks) * dur_unit,
+                  "kernels": sorted(ks)}
+        tp = [mean(k, "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed") for k in ks
+              if "sm__pipe_tensor_cycles_active.avg.pct_of_peak_sustained_elapsed" in per[k]]
+        if g.startswith("proj") and tp:
+            out[g]["tensor_pipe_pct"] = max(tp)
+    return out
 
 
 # ------------------------------------------------------------------ workload
@@ -211,9 +270,10 @@ class Model:
             x = Ld.L.out
         self.launches = sum(Ld.L.launches_per_step() for Ld in self.layers)
 
-    def step(self, ev=None, before_bwd=None):
+    def step(self, ev=None, before_bwd=None, split=False):
         """ev: optional dict name -> list of (start, end) event pairs to record into;
-        before_bwd: called between the forward and the backward (e2e: wait for grad_out's copy)."""
+        before_bwd: called between the forward and the backward (e2e: wait for grad_out's copy);
+        split: run the single-GPU backward as its two phases (per-kernel-group timing)."""
         torch = self.torch
 
         def timed(name, fn):
@@ -232,7 +292,7 @@ class Model:
             before_bwd()
         g = self.g
         for Ld in reversed(self.layers):
-            g = Ld.backward(g, timed)
+            g = Ld.backward(g, timed, split=split)
 
 
 # ------------------------------------------------------------------ CPU oracle
@@ -417,14 +477,13 @@ def run_mega(args):
     flush = None
     if cfg.n * cfg.dim * sb0 * 4 < 2 * l2_bytes:
         flush = torch.empty(2 * l2_bytes // 4, dtype=torch.float32, device=dev)
-    ev = {}
     start, end = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(local) as clk:
         sync_all()
         if flush is None and graph is None:
             start.record()
             for _ in range(args.steps):
-                model.step(ev)
+                model.step()
             end.record()
             sync_all()
             ms_step = start.elapsed_time(end) / args.steps
@@ -440,39 +499,62 @@ def run_mega(args):
                 pairs.append((s1, e1))
             sync_all()
             ms_step = float(np.sum([a.elapsed_time(b) for a, b in pairs])) / args.steps
-    if graph is not None or flush is not None:   # per-call breakdown from a separate eager pass
-        sync_all()
-        for _ in range(args.steps):
-            if flush is not None:
-                flush.fill_(1.0)
-            model.step(ev)
-        sync_all()
+    # per-call breakdown from a separate eager pass (CUDA events on the launching stream around
+    # every library call; the backward split into its source and destination phases)
+    ev = {}
+    sync_all()
+    for _ in range(args.steps):
+        if flush is not None:
+            flush.fill_(1.0)
+        model.step(ev, split=True)
+    sync_all()
     ms_t = torch.tensor([ms_step], device=dev)
     if world > 1:
         dist.all_reduce(ms_t, op=dist.ReduceOp.MAX)
     ms = float(ms_t.item())
+    n_launch = {k: len(v) for k, v in ev.items()}
     calls = {k: float(np.mean([s.elapsed_time(e) for s, e in v])) for k, v in ev.items()}
     per_step_calls = {k: float(np.sum([s.elapsed_time(e) for s, e in v])) / args.steps for k, v in ev.items()}
     L = cfg.layers
     value = L * cfg.m / (ms * 1e-3)
-    # roofline of the dominant attention call (this rank's part)
+    # ---- roofline per launch group (SURVEY §8(d)-d3 bytes; this rank's part) ----
     pk = peaks()
     sb = 2 if args.dtype == "bf16" else 4
-    att = {k: per_step_calls[k] for k in ("gat_fwd", "gat_bwd", "gat_bwd_src", "gat_bwd_dst") if k in per_step_calls}
-    dom = max(att, key=att.get)
-    bytes_per_launch = algorithmic_bytes(dom, cfg.n, model.part_edges, cfg.heads, cfg.dim, sb, rows=model.rows)
-    achieved = bytes_per_launch / (calls[dom] * 1e-3) / 1e9
-    traffic = None
-    tp = os.path.join(ROOT, "profiles", f"traffic_{cfg.name}_{args.dtype}.json")
-    if os.path.exists(tp) and world == 1:
-        traffic = json.load(open(tp)).get(dom)
-    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": pk["hbm_gbs"], "unit": "GB/s",
-                "frac": achieved / pk["hbm_gbs"], "traffic": traffic, "algorithmic_bytes": bytes_per_launch,
-                "launch_ms": calls[dom], "peak_source": pk["source"],
-                "note": "algorithmic bytes = compulsory floor (each gathered row once, DESIGN.md §5)"}
-    if traffic:  # measured DRAM bytes of the same kernels (ncu, committed) over this run's live launch time
-        roofline["traffic_gbs"] = traffic / (calls[dom] * 1e-3) / 1e9
-        roofline["traffic_frac"] = roofline["traffic_gbs"] / pk["hbm_gbs"]
+    E, N, rows, H, D = model.part_edges, cfg.n, model.rows, cfg.heads, cfg.dim
+    ncu = ncu_launch_summary(os.path.join(ROOT, "profiles", "r02", f"launches_{cfg.name}_{args.dtype}.csv"))
+    call_of = {"KB2": "gat_fwd", "KB3+KB4": "gat_bwd_src", "KB5": "gat_bwd_dst", "KB3-KB5": "gat_bwd"}
+    kernels = {}
+    for kname, call in call_of.items():
+        if call not in calls:
+            continue
+        t = calls[call] * 1e-3
+        parts = ("KB3+KB4", "KB5") if kname == "KB3-KB5" else (kname,)   # k > 1: the backward is one call
+        fb = sum(floor_bytes(q, rows, N, E, H, D, sb) for q in parts)
+        nb = sum(floor_bytes(q, rows, N, E, H, D, sb, R=E) for q in parts)
+        db = sum(design_bytes(q, rows, N, E, H, D, sb) for q in parts)
+        ent = {"call": call, "ms": calls[call], "floor_bytes": fb, "noreuse_bytes": nb, "design_bytes": db,
+               "achieved_gbs": fb / t / 1e9, "frac": fb / t / 1e9 / pk["hbm_gbs"],
+               "noreuse_frac": nb / t / 1e9 / pk["hbm_gbs"], "design_frac": db / t / 1e9 / pk["hbm_gbs"]}
+        if ncu and kname in ncu and world == 1:
+            ent["traffic"] = ncu[kname]["dram_bytes"]
+            ent["traffic_gbs"] = ncu[kname]["dram_bytes"] / t / 1e9
+            ent["traffic_frac"] = ent["traffic_gbs"] / pk["hbm_gbs"]
+            ent["ncu_ms"] = ncu[kname]["ncu_ms"]
+        kernels[kname] = ent
+    dom = max(kernels, key=lambda k: kernels[k]["ms"])
+    kd = kernels[dom]
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": kd["achieved_gbs"], "peak": pk["hbm_gbs"], "unit": "GB/s",
+                "frac": kd["frac"], "traffic": kd.get("traffic"), "algorithmic_bytes": kd["floor_bytes"],
+                "launch_ms": kd["ms"], "peak_source": pk["source"] + " (hbm_gbs, copy bandwidth)",
+                "note": "algorithmic bytes = SURVEY §8(d)-d3 floor (R = N: every gathered row once) per launch; "
+                        "time = CUDA events around the call on its stream (eager pass, bwd split by phase); "
+                        "traffic = ncu DRAM bytes per launch from profiles/r02/launches_<cfg>_<dtype>.csv",
+                "kernels": kernels}
+    if kd.get("traffic"):
+        roofline["traffic_frac"] = kd["traffic_frac"]
+    if ncu:
+        roofline["gemm"] = {g: {**ncu[g], "ms_per_call": calls.get("project_fwd" if g == "proj_fwd" else "project_bwd")}
+                            for g in ("proj_fwd", "proj_bwd") if g in ncu}
     # ---- e2e: this step's inputs from pinned host memory, parameter grads back ----
     e2e = None
     if not args.no_e2e:

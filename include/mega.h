@@ -319,6 +319,12 @@ typedef struct {
   int64_t num_local_items, num_remote_items, num_splits, num_slots;
   int64_t bwd_own_items_begin, bwd_own_items_end, bwd_own_splits_begin, bwd_own_splits_end;
   const int32_t *local_items, *remote_items, *splits;
+  /* NEXT-1 halo plan: rows sent to / received from each peer (new ids, grouped by peer,
+   * offsets [num_parts+1]); the forward moves these rows of [Wh | er] and the backward the
+   * same rows of partial [dWh | der] the other way.  full_recv_rows = num_nodes - rows of
+   * the part, what an all-gather would receive. */
+  int64_t num_send, num_recv, full_recv_rows;
+  const int32_t *send_idx, *send_off, *recv_idx, *recv_off;
 } mega_layout_dist_view;
 mega_status mega_layout_dist_view_get(mega_layout *layout, int32_t part, mega_layout_dist_view *out);
 

@@ -95,16 +95,53 @@ void dist_items(const mega_layout *L, int part, std::vector<int32_t> &local, std
   }
 }
 
+// NEXT-1: exchange only the rows a peer's edges reference.  Part p's
+// CSC row j is non-empty exactly when some in-edge of p's rows comes from source j, so
+// p needs from q the rows j in [b_q, b_{q+1}) with a non-empty CSC row in part p, and
+// sends to q its own rows with a non-empty CSC row in part q.  The same lists, read the
+// other way, route the backward's partial [dWh | der] rows back to their owners.
+void halo_plan(const mega_layout *L, int part, std::vector<int32_t> &send_idx, std::vector<int32_t> &send_off,
+               std::vector<int32_t> &recv_idx, std::vector<int32_t> &recv_off, std::vector<int32_t> &pos) {
+  const int k = (int)L->parts.size();
+  const Part &P = L->parts[part];
+  const int32_t b0 = L->bounds[part], b1 = L->bounds[part + 1], rows = b1 - b0;
+  send_idx.clear(); recv_idx.clear();
+  send_off.assign(k + 1, 0);
+  recv_off.assign(k + 1, 0);
+  pos.assign((size_t)std::max(0, k - 1) * rows, -1);
+  int slot = 0;
+  for (int q = 0; q < k; ++q) {
+    send_off[q] = (int32_t)send_idx.size();
+    recv_off[q] = (int32_t)recv_idx.size();
+    if (q == part) continue;
+    const Part &Q = L->parts[q];
+    for (int32_t j = b0; j < b1; ++j)   // own rows that q's edges reference
+      if (Q.cindptr[j + 1] > Q.cindptr[j]) send_idx.push_back(j);
+    for (int32_t j = L->bounds[q]; j < L->bounds[q + 1]; ++j)   // q's rows that this part's edges reference
+      if (P.cindptr[j + 1] > P.cindptr[j]) recv_idx.push_back(j);
+    // where q's partial of own row j lands in the receive buffer (q packs its partials of this
+    // part's rows in the order of this list, the buffer holds the peers' blocks in peer order)
+    for (int32_t t = send_off[q]; t < (int32_t)send_idx.size(); ++t)
+      pos[(size_t)slot * rows + (send_idx[t] - b0)] = t;
+    ++slot;
+  }
+  send_off[k] = (int32_t)send_idx.size();
+  recv_off[k] = (int32_t)recv_idx.size();
+}
+
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]) {
   const Part &P = L->parts[part];
-  std::vector<int32_t> dl, dr, ds;
+  std::vector<int32_t> dl, dr, ds, hs, hso, hr, hro, hp;
   int32_t nsl = 0;
-  if (L->parts.size() > 1) dist_items(L, part, dl, dr, ds, nsl);
+  if (L->parts.size() > 1) {
+    dist_items(L, part, dl, dr, ds, nsl);
+    halo_plan(L, part, hs, hso, hr, hro, hp);
+  }
   const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
                                       P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
                                       make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size(),
-                                      dl.size(), dr.size(), ds.size()};
+                                      dl.size(), dr.size(), ds.size(), hs.size(), hr.size(), hp.size()};
   size_t off = 0;
   for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
@@ -233,6 +270,14 @@ mega_status mega_layout_dist_view_get(mega_layout *L, int32_t part, mega_layout_
   v->struct_size = sizeof *v;
   if (L->parts.size() > 1) {
     dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
+    halo_plan(L, part, P.hsend_idx, P.hsend_off, P.hrecv_idx, P.hrecv_off, P.hpos);
+    v->num_send = (int64_t)P.hsend_idx.size();
+    v->num_recv = (int64_t)P.hrecv_idx.size();
+    v->full_recv_rows = L->n - (P.row_end - P.row_begin);
+    v->send_idx = P.hsend_idx.data();
+    v->send_off = P.hsend_off.data();
+    v->recv_idx = P.hrecv_idx.data();
+    v->recv_off = P.hrecv_off.data();
     auto first_ge = [](const std::vector<int32_t> &a, int stride, int32_t x) {
       int64_t lo = 0, hi = (int64_t)a.size() / stride;
       while (lo < hi) { int64_t mid = (lo + hi) / 2; if (a[mid * stride] < x) lo = mid + 1; else hi = mid; }
@@ -297,11 +342,14 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   for (int64_t v = 0; v < L->n; ++v)
     for (int32_t q = P.cindptr[v]; q < P.cindptr[v + 1]; ++q) csrc[q] = (int32_t)v;
   const std::vector<int32_t> ftiles = make_tiles(P.fwd_items), btiles = make_tiles(P.bwd_items);
-  if (L->parts.size() > 1) dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
+  if (L->parts.size() > 1) {
+    dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
+    halo_plan(L, part, P.hsend_idx, P.hsend_off, P.hrecv_idx, P.hrecv_off, P.hpos);
+  }
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
       &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos,
-      &P.dl_items, &P.dr_items, &P.d_splits};
+      &P.dl_items, &P.dr_items, &P.d_splits, &P.hsend_idx, &P.hrecv_idx, &P.hpos};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
@@ -346,6 +394,11 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.n_dr_items = (int32_t)(P.dr_items.size() / 4);
   D.n_d_splits = (int32_t)(P.d_splits.size() / 3);
   D.n_d_slots = P.n_d_slots;
+  D.hsend_idx = reinterpret_cast<const int32_t *>(base + offs[17]);
+  D.hrecv_idx = reinterpret_cast<const int32_t *>(base + offs[18]);
+  D.hpos = reinterpret_cast<const int32_t *>(base + offs[19]);
+  D.n_hsend = (int64_t)P.hsend_idx.size();
+  D.n_hrecv = (int64_t)P.hrecv_idx.size();
   {  // own-source ranges of the CSC work (items and splits are sorted by source id)
     auto first_ge = [](const std::vector<int32_t> &v, int stride, int32_t x) {
       int64_t lo = 0, hi = (int64_t)v.size() / stride;

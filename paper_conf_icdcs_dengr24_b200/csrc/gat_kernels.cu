@@ -1127,26 +1127,52 @@ __global__ void __launch_bounds__(1024) param_reduce_kernel(const double *parts_
   }
 }
 
-// k-GPU backward: add the peers' partial [dWh | der] of this
-// part's own rows (received into `stage`, one [rows][ld] block per peer) to
-// the local partial, peers in ascending order (fixed order: deterministic).
-__global__ void __launch_bounds__(256) dist_combine_kernel(float *gfeat, int64_t ldgf, float *der, const float *stage,
-                                                           const float *stage_der, int npeers, int64_t rows,
-                                                           int64_t row0, int D, int H) {
+// k-GPU exchange (SURVEY §8(e), NEXT-1 halo): dst[di] = src[si] for i < cnt, rows of
+// row_bytes, si = sidx ? sidx[i] : i (gather into a send buffer), di = didx ? didx[i] : i
+// (scatter out of a receive buffer).  16-byte vectors when everything is 16-byte aligned.
+__global__ void __launch_bounds__(256) rows_move_kernel(const char *src, int64_t src_ld, const int32_t *sidx,
+                                                        char *dst, int64_t dst_ld, const int32_t *didx, int64_t cnt,
+                                                        int row_bytes, int vec16) {
+  const int per = vec16 ? row_bytes / 16 : row_bytes / 4;
+  const int64_t total = cnt * per;
+  for (int64_t t = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; t < total; t += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t i = t / per;
+    const int c = (int)(t % per);
+    const int64_t si = sidx ? sidx[i] : i, di = didx ? didx[i] : i;
+    if (vec16)
+      reinterpret_cast<uint4 *>(dst + di * dst_ld)[c] = reinterpret_cast<const uint4 *>(src + si * src_ld)[c];
+    else
+      reinterpret_cast<uint32_t *>(dst + di * dst_ld)[c] = reinterpret_cast<const uint32_t *>(src + si * src_ld)[c];
+  }
+}
+
+// k-GPU backward: add the peers' partial [dWh | der] of this part's own rows (received rows
+// `recv` [n][D] / `recv_der` [n][H]; pos[slot][r] = index of peer slot's partial of own row r,
+// -1 if that peer has no edge from r) to the local partial, peers in ascending order (fixed
+// order: deterministic).
+__global__ void __launch_bounds__(256) dist_combine_kernel(float *gfeat, int64_t ldgf, float *der, const float *recv,
+                                                           const float *recv_der, const int32_t *pos, int npeers,
+                                                           int64_t rows, int64_t row0, int D, int H) {
   const int64_t nv = rows * (D / 4);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < nv; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = i / (D / 4), c = 4 * (i % (D / 4));
     float4 *dst = reinterpret_cast<float4 *>(gfeat + (row0 + r) * ldgf + c);
     float4 acc = *dst;
     for (int q = 0; q < npeers; ++q) {
-      const float4 v = *reinterpret_cast<const float4 *>(stage + ((int64_t)q * rows + r) * ldgf + c);
+      const int32_t t = pos[(int64_t)q * rows + r];
+      if (t < 0) continue;
+      const float4 v = *reinterpret_cast<const float4 *>(recv + (int64_t)t * D + c);
       acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
     }
     *dst = acc;
   }
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < rows * H; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / H, h = i % H;
     float acc = der[row0 * H + i];
-    for (int q = 0; q < npeers; ++q) acc += stage_der[(int64_t)q * rows * H + i];
+    for (int q = 0; q < npeers; ++q) {
+      const int32_t t = pos[(int64_t)q * rows + r];
+      if (t >= 0) acc += recv_der[(int64_t)t * H + h];
+    }
     der[row0 * H + i] = acc;
   }
 }
@@ -1583,24 +1609,48 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
 // ---------------- k-GPU path ----------------
 namespace mega {
 namespace {
-struct DistWs { size_t fwd, bwd_base, stage, stage_der, bwd_total; };
+// workspace of the dist calls: fwd = mega_gat_fwd's (with the split-row slots) + halo send / receive
+// buffers of packed [Wh | er] rows; bwd = mega_gat_bwd's + packed partial [dWh | der] rows out / in
+struct DistWs { size_t fwd_base, f_sf, f_se, f_rf, f_re, fwd_total, bwd_base, b_sf, b_se, b_rf, b_re, bwd_total; };
 DistWs dist_ws(const mega_layout *L, int32_t part, const Shape &s) {
   const Part &P = L->parts[part];
   DevPart D = host_counts(P, L->n);
   int32_t nslots = P.n_d_slots;
+  int64_t nsend = (int64_t)P.hsend_idx.size(), nrecv = (int64_t)P.hrecv_idx.size();
   if (L->parts.size() > 1 && P.dl_items.empty() && P.dr_items.empty()) {
-    std::vector<int32_t> a, b, c;
+    std::vector<int32_t> a, b, c, d, e, f, g, h;
     dist_items(L, part, a, b, c, nslots);
+    halo_plan(L, part, d, e, f, g, h);
+    nsend = (int64_t)d.size();
+    nrecv = (int64_t)f.size();
   }
   D.n_fwd_slots = std::max(D.n_fwd_slots, nslots);
+  const size_t esz = 16 / s.epv, rf = (size_t)s.D * esz, re = (size_t)s.H * 4;
   DistWs w;
-  w.fwd = ws_fwd(D, s).total;
+  w.fwd_base = ws_fwd(D, s).total;
+  w.f_sf = w.fwd_base;
+  w.f_se = align256(w.f_sf + nsend * rf);
+  w.f_rf = align256(w.f_se + nsend * re);
+  w.f_re = align256(w.f_rf + nrecv * rf);
+  w.fwd_total = align256(w.f_re + nrecv * re);
   w.bwd_base = ws_bwd(D, s).total;
-  const size_t k1 = L->parts.size() - 1, rows = (size_t)(P.row_end - P.row_begin);
-  w.stage = w.bwd_base;
-  w.stage_der = align256(w.stage + k1 * rows * (size_t)s.D * 4);
-  w.bwd_total = align256(w.stage_der + k1 * rows * (size_t)s.H * 4);
+  w.b_sf = w.bwd_base;                                   // partials of the peers' rows this part references
+  w.b_se = align256(w.b_sf + nrecv * (size_t)s.D * 4);
+  w.b_rf = align256(w.b_se + nrecv * re);                // the peers' partials of this part's rows
+  w.b_re = align256(w.b_rf + nsend * (size_t)s.D * 4);
+  w.bwd_total = align256(w.b_re + nsend * re);
   return w;
+}
+mega_status move_rows(const void *src, int64_t src_ld, const int32_t *sidx, void *dst, int64_t dst_ld,
+                      const int32_t *didx, int64_t cnt, int row_bytes, cudaStream_t st, int dev) {
+  if (cnt <= 0) return MEGA_OK;
+  const bool v16 = row_bytes % 16 == 0 && src_ld % 16 == 0 && dst_ld % 16 == 0 && al16(src) && al16(dst);
+  const int64_t total = cnt * (v16 ? row_bytes / 16 : row_bytes / 4);
+  const int blocks = (int)std::min<int64_t>((total + 255) / 256, 8 * dev_info(dev).sms);
+  kern::rows_move_kernel<<<std::max(blocks, 1), 256, 0, st>>>(static_cast<const char *>(src), src_ld, sidx,
+                                                               static_cast<char *>(dst), dst_ld, didx, cnt, row_bytes,
+                                                               v16 ? 1 : 0);
+  return check_launch(st, "rows_move_kernel");
 }
 bool phase_flags(uint32_t flags, bool &snd, bool &rcv) {
   const uint32_t ph = flags & (MEGA_DIST_PHASE_SEND | MEGA_DIST_PHASE_RECV);
@@ -1629,7 +1679,7 @@ mega_status mega_gat_dist_workspace_bytes(const mega_layout *L, int32_t part, in
   mega_status rc = check_shape(heads, head_dim, dtype, s);
   if (rc != MEGA_OK) return rc;
   const DistWs w = dist_ws(L, part, s);
-  *fwd_ws = w.fwd;
+  *fwd_ws = w.fwd_total;
   *bwd_ws = w.bwd_total;
   return MEGA_OK;
 }
@@ -1657,7 +1707,7 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   if (!al16(feat) || !al16(out) || !al16(ctx) || !al16(ws)) return fail(MEGA_ERR_INVALID_ARGUMENT, "pointers must be 16-byte aligned");
   const Part &P = L->parts[part];
   const DistWs dw = dist_ws(L, part, s);
-  if (ws_bytes < dw.fwd) return fail(MEGA_ERR_OUT_OF_MEMORY, "fwd workspace too small (mega_gat_dist_workspace_bytes)");
+  if (ws_bytes < dw.fwd_total) return fail(MEGA_ERR_OUT_OF_MEMORY, "fwd workspace too small (mega_gat_dist_workspace_bytes)");
   bool snd, rcv;
   phase_flags(flags, snd, rcv);
   cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
@@ -1684,33 +1734,43 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
     b.L.fwd_splits = splits; b.L.n_fwd_splits = nsplits;
     return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(b, s, st, dev) : run_fwd<float>(b, s, st, dev);
   };
-  const int k = (int)L->parts.size(), p = part;
+  // NEXT-1 halo exchange: only the rows a peer's edges reference, packed [Wh] and [er] per peer
+  const int k = (int)L->parts.size();
+  const size_t rf = (size_t)s.D * esz, re = (size_t)s.H * 4;
+  char *sf = wb + dw.f_sf, *se = wb + dw.f_se, *rfb = wb + dw.f_rf, *reb = wb + dw.f_re;
   std::vector<CommMsg> sends, recvs;
   for (int q = 0; q < k; ++q) {
-    if (q == p) continue;
-    const int64_t q0 = L->bounds[q], qn = L->bounds[q + 1] - q0;
-    sends.push_back({q, 0, fb + b0 * ldf * esz, (size_t)(rows * ldf * esz)});
-    sends.push_back({q, 1, ctx + plane + b0 * s.H, (size_t)(rows * s.H * 4)});
-    recvs.push_back({q, 0, fb + q0 * ldf * esz, (size_t)(qn * ldf * esz)});
-    recvs.push_back({q, 1, ctx + plane + q0 * s.H, (size_t)(qn * s.H * 4)});
+    if (q == part) continue;
+    const int64_t s0 = P.hsend_off[q], sn = P.hsend_off[q + 1] - s0, r0 = P.hrecv_off[q], rn = P.hrecv_off[q + 1] - r0;
+    sends.push_back({q, 0, sf + s0 * rf, (size_t)sn * rf});
+    sends.push_back({q, 1, se + s0 * re, (size_t)sn * re});
+    recvs.push_back({q, 0, rfb + r0 * rf, (size_t)rn * rf});
+    recvs.push_back({q, 1, reb + r0 * re, (size_t)rn * re});
   }
+  const DevPart &DP = P.dev;
   if (snd) {
     if (!(flags & MEGA_FLAG_ELER_IN_CTX) && rows > 0) {   // el/er of the own rows (those we send)
       rc = launch_eler_any(dtype, fb + b0 * ldf * esz, ldf, rows, b0, attn_l, attn_r, heads, head_dim, ctx, ctx + plane, st);
       if (rc != MEGA_OK) return rc;
     }
-    // [Wh | er] of the own rows to every peer on the comm stream, the peers' rows back ...
+    // pack the own rows the peers need, send them on the comm stream, receive the peers' rows ...
+    if ((rc = move_rows(fb, ldf * esz, DP.hsend_idx, sf, rf, nullptr, DP.n_hsend, (int)rf, st, dev)) != MEGA_OK) return rc;
+    if ((rc = move_rows(ctx + plane, re, DP.hsend_idx, se, re, nullptr, DP.n_hsend, (int)re, st, dev)) != MEGA_OK) return rc;
     if ((rc = comm_exchange(comm, sends, recvs, st, cs, true, false)) != MEGA_OK) return rc;
     // ... while block (p, p) (sources this rank owns) runs on the compute stream
-    if ((rc = pass(P.dev.dl_items, P.dev.n_dl_items, nullptr, 0)) != MEGA_OK) return rc;
+    if ((rc = pass(DP.dl_items, DP.n_dl_items, nullptr, 0)) != MEGA_OK) return rc;
   }
   if (rcv) {
     if ((rc = comm_exchange(comm, sends, recvs, st, cs, false, true)) != MEGA_OK) return rc;
-    cudaError_t ce = cudaStreamWaitEvent(st, comm_done_event(comm), 0);
+    // scatter the received rows into the global [Wh | er] arrays (comm stream), then continue
+    if ((rc = move_rows(rfb, rf, nullptr, fb, ldf * esz, DP.hrecv_idx, DP.n_hrecv, (int)rf, cs, dev)) != MEGA_OK) return rc;
+    if ((rc = move_rows(reb, re, nullptr, ctx + plane, re, DP.hrecv_idx, DP.n_hrecv, (int)re, cs, dev)) != MEGA_OK) return rc;
+    cudaError_t ce = cudaEventRecord(comm_done_event(comm), cs);
+    if (ce == cudaSuccess) ce = cudaStreamWaitEvent(st, comm_done_event(comm), 0);
     if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("wait comm: ") + cudaGetErrorString(ce));
     // remote blocks, then the fixed-order merge of the rows split across passes / segments (KB7)
-    if ((rc = pass(P.dev.dr_items, P.dev.n_dr_items, nullptr, 0)) != MEGA_OK) return rc;
-    if ((rc = pass(nullptr, 0, P.dev.d_splits, P.dev.n_d_splits)) != MEGA_OK) return rc;
+    if ((rc = pass(DP.dr_items, DP.n_dr_items, nullptr, 0)) != MEGA_OK) return rc;
+    if ((rc = pass(nullptr, 0, DP.d_splits, DP.n_d_splits)) != MEGA_OK) return rc;
   }
   return MEGA_OK;
 }
@@ -1770,7 +1830,6 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
-  float *stage = reinterpret_cast<float *>(wb + dw.stage), *stage_der = reinterpret_cast<float *>(wb + dw.stage_der);
   cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
   // source-phase launches over a range of CSC items [i0, i1) and splits [s0, s1)
   auto src_range = [&](int32_t i0, int32_t i1, int32_t s0, int32_t s1, bool dlt) {
@@ -1780,24 +1839,27 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
     return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt)
                               : run_bwd<float>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt);
   };
-  const int k = (int)L->parts.size(), p = part;
+  // NEXT-1 halo: this rank's partials of the peers' rows its edges reference go back to their owners
+  // (the forward's receive lists), the peers' partials of our rows arrive in send-list order
+  const int k = (int)L->parts.size();
+  const size_t rf = (size_t)s.D * 4, re = (size_t)s.H * 4;
+  char *sf = wb + dw.b_sf, *se = wb + dw.b_se, *rfb = wb + dw.b_rf, *reb = wb + dw.b_re;
   std::vector<CommMsg> sends, recvs;
-  int slot = 0;
   for (int q = 0; q < k; ++q) {
-    if (q == p) continue;
-    const int64_t q0 = L->bounds[q], qn = L->bounds[q + 1] - q0;
-    // this rank's partial [dWh | der] of q's rows -> q; q's partial of our rows -> stage slot
-    sends.push_back({q, 2, grad_feat + q0 * ldgf, (size_t)(qn * ldgf * 4)});
-    sends.push_back({q, 3, ctx + 4 * plane + q0 * s.H, (size_t)(qn * s.H * 4)});
-    recvs.push_back({q, 2, stage + (int64_t)slot * rows * ldgf, (size_t)(rows * ldgf * 4)});
-    recvs.push_back({q, 3, stage_der + (int64_t)slot * rows * s.H, (size_t)(rows * s.H * 4)});
-    ++slot;
+    if (q == part) continue;
+    const int64_t s0 = P.hrecv_off[q], sn = P.hrecv_off[q + 1] - s0, r0 = P.hsend_off[q], rn = P.hsend_off[q + 1] - r0;
+    sends.push_back({q, 2, sf + s0 * rf, (size_t)sn * rf});
+    sends.push_back({q, 3, se + s0 * re, (size_t)sn * re});
+    recvs.push_back({q, 2, rfb + r0 * rf, (size_t)rn * rf});
+    recvs.push_back({q, 3, reb + r0 * re, (size_t)rn * re});
   }
   const DevPart &D = P.dev;
   if (snd) {
     // Dlt, then the sources other ranks own (their partials travel while ours are computed)
     if ((rc = src_range(0, D.bwd_own0, 0, D.bsplit_own0, true)) != MEGA_OK) return rc;
     if ((rc = src_range(D.bwd_own1, D.n_bwd_items, D.bsplit_own1, D.n_bwd_splits, false)) != MEGA_OK) return rc;
+    if ((rc = move_rows(grad_feat, ldgf * 4, D.hrecv_idx, sf, rf, nullptr, D.n_hrecv, (int)rf, st, dev)) != MEGA_OK) return rc;
+    if ((rc = move_rows(ctx + 4 * plane, re, D.hrecv_idx, se, re, nullptr, D.n_hrecv, (int)re, st, dev)) != MEGA_OK) return rc;
     if ((rc = comm_exchange(comm, sends, recvs, st, cs, true, false)) != MEGA_OK) return rc;
     if ((rc = src_range(D.bwd_own0, D.bwd_own1, D.bsplit_own0, D.bsplit_own1, false)) != MEGA_OK) return rc;
   }
@@ -1808,8 +1870,9 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
     if (k > 1 && rows > 0) {
       const int64_t nv = rows * (s.D / 4);
       const int blocks = (int)std::min<int64_t>((nv + 255) / 256, 4 * dev_info(dev).sms);
-      kern::dist_combine_kernel<<<std::max(blocks, 1), 256, 0, st>>>(grad_feat, ldgf, ctx + 4 * plane, stage, stage_der,
-                                                                     k - 1, rows, b0, s.D, s.H);
+      kern::dist_combine_kernel<<<std::max(blocks, 1), 256, 0, st>>>(
+          grad_feat, ldgf, ctx + 4 * plane, reinterpret_cast<const float *>(rfb), reinterpret_cast<const float *>(reb),
+          D.hpos, k - 1, rows, b0, s.D, s.H);
       if ((rc = check_launch(st, "dist_combine_kernel")) != MEGA_OK) return rc;
     }
     rc = dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, MEGA_BWD_PHASE_DST, st, dev)

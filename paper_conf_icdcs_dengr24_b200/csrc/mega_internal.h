@@ -48,6 +48,11 @@ struct DevPart {
   // backward: items / splits of this part's own sources (rows [row_begin, row_end)) are the
   // contiguous ranges [bwd_own0, bwd_own1) of bwd_items and [bsplit_own0, bsplit_own1) of bwd_splits
   int32_t bwd_own0 = 0, bwd_own1 = 0, bsplit_own0 = 0, bsplit_own1 = 0;
+  // NEXT-1 halo exchange: send_idx lists (peer by peer, ascending) the own rows some peer's edges
+  // reference, recv_idx the peers' rows this part's edges reference; pos [k-1][rows] maps an own row
+  // to the index of that peer's partial of it in the receive buffer (-1: the peer does not reference it)
+  const int32_t *hsend_idx = nullptr, *hrecv_idx = nullptr, *hpos = nullptr;
+  int64_t n_hsend = 0, n_hrecv = 0;
 };
 
 struct Part {
@@ -55,6 +60,7 @@ struct Part {
   // k > 1 dist items (derived from indptr/src/bounds at bind time; host copies for the view)
   std::vector<int32_t> dl_items, dr_items, d_splits;
   int32_t n_d_slots = 0;
+  std::vector<int32_t> hsend_idx, hsend_off, hrecv_idx, hrecv_off, hpos;   // halo plan (k > 1)
   std::vector<int32_t> indptr, src, eid, cindptr, cdst, cpos, csr2csc;
   std::vector<int32_t> fwd_items, fwd_splits, bwd_items, bwd_splits;
   int32_t n_fwd_slots = 0, n_bwd_slots = 0;
@@ -82,10 +88,14 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-constexpr int kImageArrays = 17;
+constexpr int kImageArrays = 20;
 // dist items of part p (k > 1): see DevPart; S = the layout's segment size
 void dist_items(const mega_layout *L, int part, std::vector<int32_t> &local, std::vector<int32_t> &remote,
                 std::vector<int32_t> &splits, int32_t &nslots);
+// NEXT-1 halo plan of part p (k > 1): rows each peer needs from p (send, grouped by peer q
+// ascending, offsets [k+1]), rows p needs from each peer (recv), and p's pos map (see DevPart)
+void halo_plan(const mega_layout *L, int part, std::vector<int32_t> &send_idx, std::vector<int32_t> &send_off,
+               std::vector<int32_t> &recv_idx, std::vector<int32_t> &recv_off, std::vector<int32_t> &pos);
 // comm.cpp: one exchange of (peer, pointer, bytes) messages (see mega_comm)
 struct CommMsg { int peer; int tag; const void *ptr; size_t bytes; };
 }  // namespace mega

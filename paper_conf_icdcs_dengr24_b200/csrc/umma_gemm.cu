@@ -55,6 +55,7 @@ struct Args {
   const float *al, *ar;
   int H, F;
   int64_t ctx_row0;
+  int ntiles;       // fwd / dX: column tiles (grid.x = row tiles * ntiles)
 };
 
 // ------------------------------------------------------------------ PTX helpers
@@ -84,6 +85,13 @@ __device__ __forceinline__ void tma_load_2d(uint32_t dst, const CUtensorMap *map
       "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(dst),
       "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(bar)
       : "memory");
+}
+// shared -> global tensor store (bulk group); the source must stay valid until the read completes
+__device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t src, int32_t x, int32_t y) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%1, %2}], [%3];" ::"l"(
+                   reinterpret_cast<uint64_t>(map)),
+               "r"(x), "r"(y), "r"(src)
+               : "memory");
 }
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
@@ -139,7 +147,8 @@ template <int BN> struct Tiles {
 // when B is MN-major).  FH: fwd only, min(head_dim, 32) (heads per 32-column chunk).
 template <int MODE, int BN, int FH>
 __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constant__ CUtensorMap tmA,
-                                                            const __grid_constant__ CUtensorMap tmB, const Args g) {
+                                                            const __grid_constant__ CUtensorMap tmB,
+                                                            const __grid_constant__ CUtensorMap tmO, const Args g) {
   using TL = Tiles<BN>;
   constexpr int STAGES = TL::STAGES;
   constexpr bool A_MN = MODE == DW, B_MN = MODE != DX;
@@ -150,8 +159,12 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
   float *s_al = reinterpret_cast<float *>(smem + STAGES * TL::STAGE + 256);
   float *s_ar = s_al + BN;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t m0 = (int64_t)blockIdx.x * BM;
-  const int n0 = blockIdx.y * BN;
+  // fwd / dX: one linear grid with the column tile fastest, so the CTAs that share a row tile of A
+  // (X, dWh) run together and the second column tile reads it from L2; dW: (m, n, split) grid
+  const int64_t mtile = MODE == DW ? (int64_t)blockIdx.x : (int64_t)blockIdx.x / g.ntiles;
+  const int ntile = MODE == DW ? (int)blockIdx.y : (int)(blockIdx.x % g.ntiles);
+  const int64_t m0 = mtile * BM;
+  const int n0 = ntile * BN;
   const int64_t kb0 = (int64_t)blockIdx.z * g.kb_split;
   const int64_t kb1 = g.kb_total < kb0 + g.kb_split ? g.kb_total : kb0 + g.kb_split;
   const int nkb = kb1 > kb0 ? (int)(kb1 - kb0) : 0;
@@ -168,6 +181,7 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
     if (lane == 0) {
       prefetch_tmap(&tmA);
       prefetch_tmap(&tmB);
+      if (MODE != DW) prefetch_tmap(&tmO);
       for (int s = 0; s < STAGES; ++s) {
         mbar_init(full0 + 8 * s, 1);
         mbar_init(empty0 + 8 * s, 1);
@@ -252,8 +266,11 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
         *reinterpret_cast<uint4 *>(dst + c0 + 4 * q) = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
     }
   } else {
-    __nv_bfloat16 *orow = static_cast<__nv_bfloat16 *>(g.out) + grow * g.ldo + n0;
+    // bf16 tile -> shared memory (the operand ring is free once the accumulator is complete),
+    // laid out as BN/64 TMA boxes of [128 rows][128 B] with the 128-byte swizzle (conflict-free
+    // row-per-thread writes), then TMA bulk stores (rows past M / columns past Nc are clipped)
     const bool live = grow < g.M;
+    const uint32_t obase = smem_u32(smem);
     float el_acc = 0.f, er_acc = 0.f;
 #pragma unroll 1
     for (int c0 = 0; c0 < BN; c0 += 32) {
@@ -262,11 +279,13 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
       uint32_t p[16];
 #pragma unroll
       for (int q = 0; q < 16; ++q) p[q] = bf2(__uint_as_float(r[2 * q]), __uint_as_float(r[2 * q + 1]));
-      if (live) {
+      const uint32_t box = obase + (uint32_t)(c0 / 64) * (BM * 128) + (uint32_t)row * 128;
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-          if (MODE == FWD || n0 + c0 + 8 * q < g.Nc)
-            *reinterpret_cast<uint4 *>(orow + c0 + 8 * q) = make_uint4(p[4 * q], p[4 * q + 1], p[4 * q + 2], p[4 * q + 3]);
+      for (int q = 0; q < 4; ++q) {
+        const uint32_t u = (uint32_t)((c0 % 64) / 8 + q);
+        asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(box + ((u ^ (uint32_t)(row & 7)) << 4)),
+                     "r"(p[4 * q]), "r"(p[4 * q + 1]), "r"(p[4 * q + 2]), "r"(p[4 * q + 3])
+                     : "memory");
       }
       if constexpr (MODE == FWD) {
         // el/er from the STORED (bf16-rounded) Wh, head by head (FH values per head segment)
@@ -294,6 +313,15 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
           }
         }
       }
+    }
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");   // st.shared -> visible to the TMA engine
+    __syncthreads();
+    if (threadIdx.x == 0) {
+#pragma unroll
+      for (int j = 0; j < BN / 64; ++j)
+        if (n0 + 64 * j < g.Nc) tma_store_2d(&tmO, obase + (uint32_t)j * (BM * 128), n0 + 64 * j, (int32_t)m0);
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");   // smem may be released after this
     }
   }
   tc_fence_before();
@@ -363,7 +391,8 @@ int sm_count() {
 }
 
 template <int MODE, int BN, int FH>
-mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const Args &g, dim3 grid, cudaStream_t st) {
+mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap &o, const Args &g, dim3 grid,
+                   cudaStream_t st) {
   auto k = umma_gemm_kernel<MODE, BN, FH>;
   const size_t smem = Tiles<BN>::SMEM;
   static bool attr = false;  // per instantiation
@@ -372,7 +401,7 @@ mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const Args &g, di
     if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma smem attribute: ") + cudaGetErrorString(e));
     attr = true;
   }
-  k<<<grid, THREADS, smem, st>>>(a, b, g);
+  k<<<grid, THREADS, smem, st>>>(a, b, o, g);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma_gemm_kernel: ") + cudaGetErrorString(e));
   return MEGA_OK;
@@ -391,34 +420,36 @@ mega_status umma_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_di
   const int BN = std::min(D, 256);
   if (D % 64 || BN % head_dim || head_dim % 8)
     return fail(MEGA_ERR_UNSUPPORTED, "tcgen05 projection: D must be a multiple of 64 and head_dim divide min(D, 256)");
-  CUtensorMap ta, tb;
+  CUtensorMap ta, tb, to;
   mega_status rc;
   if ((rc = tmap_2d(&ta, x, (uint64_t)in_dim, (uint64_t)rows, ldx, 64, BM)) != MEGA_OK) return rc;
   if ((rc = tmap_2d(&tb, w, (uint64_t)D, (uint64_t)in_dim, D, 64, 64)) != MEGA_OK) return rc;
+  if ((rc = tmap_2d(&to, feat, (uint64_t)D, (uint64_t)rows, ldf, 64, BM)) != MEGA_OK) return rc;
   Args g{};
   g.M = rows; g.Nc = D; g.kb_total = (in_dim + BK - 1) / BK; g.kb_split = g.kb_total;
   g.out = feat; g.ldo = ldf; g.el = el; g.er = er; g.al = al; g.ar = ar; g.H = heads; g.F = head_dim;
   g.ctx_row0 = ctx_row0;
-  const dim3 grid((unsigned)((rows + BM - 1) / BM), (unsigned)(D / BN), 1);
+  g.ntiles = D / BN;
+  const dim3 grid((unsigned)(((rows + BM - 1) / BM) * g.ntiles), 1, 1);
   const int fh = std::min(head_dim, 32);
   if (BN == 256) {
-    if (fh == 32) return launch<FWD, 256, 32>(ta, tb, g, grid, st);
-    if (fh == 16) return launch<FWD, 256, 16>(ta, tb, g, grid, st);
-    return launch<FWD, 256, 8>(ta, tb, g, grid, st);
+    if (fh == 32) return launch<FWD, 256, 32>(ta, tb, to, g, grid, st);
+    if (fh == 16) return launch<FWD, 256, 16>(ta, tb, to, g, grid, st);
+    return launch<FWD, 256, 8>(ta, tb, to, g, grid, st);
   }
   if (BN == 128) {
-    if (fh == 32) return launch<FWD, 128, 32>(ta, tb, g, grid, st);
-    if (fh == 16) return launch<FWD, 128, 16>(ta, tb, g, grid, st);
-    return launch<FWD, 128, 8>(ta, tb, g, grid, st);
+    if (fh == 32) return launch<FWD, 128, 32>(ta, tb, to, g, grid, st);
+    if (fh == 16) return launch<FWD, 128, 16>(ta, tb, to, g, grid, st);
+    return launch<FWD, 128, 8>(ta, tb, to, g, grid, st);
   }
   if (BN == 192) {
-    if (fh == 32) return launch<FWD, 192, 32>(ta, tb, g, grid, st);
-    if (fh == 16) return launch<FWD, 192, 16>(ta, tb, g, grid, st);
-    return launch<FWD, 192, 8>(ta, tb, g, grid, st);
+    if (fh == 32) return launch<FWD, 192, 32>(ta, tb, to, g, grid, st);
+    if (fh == 16) return launch<FWD, 192, 16>(ta, tb, to, g, grid, st);
+    return launch<FWD, 192, 8>(ta, tb, to, g, grid, st);
   }
-  if (fh == 32) return launch<FWD, 64, 32>(ta, tb, g, grid, st);
-  if (fh == 16) return launch<FWD, 64, 16>(ta, tb, g, grid, st);
-  return launch<FWD, 64, 8>(ta, tb, g, grid, st);
+  if (fh == 32) return launch<FWD, 64, 32>(ta, tb, to, g, grid, st);
+  if (fh == 16) return launch<FWD, 64, 16>(ta, tb, to, g, grid, st);
+  return launch<FWD, 64, 8>(ta, tb, to, g, grid, st);
 }
 
 // dX[rows][in_dim] = dWh W^T (bf16 out).  K = D (multiple of 64).  Columns are written in
@@ -428,16 +459,18 @@ mega_status umma_project_dx(const void *gf, int64_t ldgf, int64_t rows, int in_d
                             int64_t ldgx, cudaStream_t st) {
   if (D % 64) return fail(MEGA_ERR_UNSUPPORTED, "tcgen05 dX: D % 64 required");
   const int BN = in_dim >= 256 ? 256 : (in_dim >= 128 ? 128 : 64);
-  CUtensorMap ta, tb;
+  CUtensorMap ta, tb, to;
   mega_status rc;
   if ((rc = tmap_2d(&ta, gf, (uint64_t)D, (uint64_t)rows, ldgf, 64, BM)) != MEGA_OK) return rc;
   if ((rc = tmap_2d(&tb, w, (uint64_t)D, (uint64_t)in_dim, D, 64, BN)) != MEGA_OK) return rc;
+  if ((rc = tmap_2d(&to, gx, (uint64_t)((in_dim + 7) / 8 * 8), (uint64_t)rows, ldgx, 64, BM)) != MEGA_OK) return rc;
   Args g{};
   g.M = rows; g.Nc = (in_dim + 7) / 8 * 8; g.kb_total = D / BK; g.kb_split = g.kb_total; g.out = gx; g.ldo = ldgx;
-  const dim3 grid((unsigned)((rows + BM - 1) / BM), (unsigned)((in_dim + BN - 1) / BN), 1);
-  if (BN == 256) return launch<DX, 256, 32>(ta, tb, g, grid, st);
-  if (BN == 128) return launch<DX, 128, 32>(ta, tb, g, grid, st);
-  return launch<DX, 64, 32>(ta, tb, g, grid, st);
+  g.ntiles = (in_dim + BN - 1) / BN;
+  const dim3 grid((unsigned)(((rows + BM - 1) / BM) * g.ntiles), 1, 1);
+  if (BN == 256) return launch<DX, 256, 32>(ta, tb, to, g, grid, st);
+  if (BN == 128) return launch<DX, 128, 32>(ta, tb, to, g, grid, st);
+  return launch<DX, 64, 32>(ta, tb, to, g, grid, st);
 }
 
 // workspace of umma_project_dw: split partials
@@ -471,10 +504,10 @@ mega_status umma_project_dw(const void *x, int64_t ldx, const void *gf, int64_t 
   g.M = mpad; g.Nc = D; g.kb_total = (rows + BK - 1) / BK; g.kb_split = (g.kb_total + splits - 1) / splits;
   g.out = ws; g.mpad = mpad;
   const dim3 grid((unsigned)(mpad / BM), (unsigned)(D / BN), (unsigned)splits);
-  if (BN == 256) rc = launch<DW, 256, 32>(ta, tb, g, grid, st);
-  else if (BN == 128) rc = launch<DW, 128, 32>(ta, tb, g, grid, st);
-  else if (BN == 192) rc = launch<DW, 192, 32>(ta, tb, g, grid, st);
-  else rc = launch<DW, 64, 32>(ta, tb, g, grid, st);
+  if (BN == 256) rc = launch<DW, 256, 32>(ta, tb, ta, g, grid, st);
+  else if (BN == 128) rc = launch<DW, 128, 32>(ta, tb, ta, g, grid, st);
+  else if (BN == 192) rc = launch<DW, 192, 32>(ta, tb, ta, g, grid, st);
+  else rc = launch<DW, 64, 32>(ta, tb, ta, g, grid, st);
   if (rc != MEGA_OK) return rc;
   const int64_t n4 = (int64_t)in_dim * D / 4;
   const int blocks = (int)std::min<int64_t>((n4 + 255) / 256, 4 * sm_count());

@@ -114,10 +114,15 @@ class DistGATLayer:
                                                      comm_stream=self.cs))
         return L.out
 
-    def backward(self, grad_out_local, timed=None):
+    def backward(self, grad_out_local, timed=None, split=False):
+        """split (k = 1): the source and destination phases as two calls, for per-phase timing
+        (the same work as the single call)."""
         L = self.L
         t = timed or (lambda name, fn: fn())
-        if self.k == 1:   # one call: lets LP_ONLY keep the partial in the bf16 operand
+        if self.k == 1 and split:
+            t("gat_bwd_src", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_SRC))
+            t("gat_bwd_dst", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_DST))
+        elif self.k == 1:   # one call: lets LP_ONLY keep the partial in the bf16 operand
             t("gat_bwd", lambda: L.attend_backward(grad_out_local, 0))
         else:
             flags = M.MEGA_BWD_LP_ONLY if (L.lp_only and L.grad_feat_lp is not None) else 0

@@ -65,7 +65,9 @@ class mega_layout_dist_view(_c.Structure):
     _fields_ = [("struct_size", _c.c_uint32)] + [(k, _c.c_int64) for k in (
         "num_local_items", "num_remote_items", "num_splits", "num_slots", "bwd_own_items_begin", "bwd_own_items_end",
         "bwd_own_splits_begin", "bwd_own_splits_end")] + [(k, _c.POINTER(_c.c_int32)) for k in (
-        "local_items", "remote_items", "splits")]
+        "local_items", "remote_items", "splits")] + [(k, _c.c_int64) for k in (
+        "num_send", "num_recv", "full_recv_rows")] + [(k, _c.POINTER(_c.c_int32)) for k in (
+        "send_idx", "send_off", "recv_idx", "recv_off")]
 
 
 class mega_layout_view(_c.Structure):
@@ -318,10 +320,16 @@ def mega_layout_dist_view_get(layout: Layout, part: int = 0) -> dict:
     v = mega_layout_dist_view()
     _check(lib().mega_layout_dist_view_get(layout.handle, part, _c.byref(v)))
     d = {k: getattr(v, k) for k, _ in mega_layout_dist_view._fields_[1:9]}
+    d.update({k: getattr(v, k) for k in ("num_send", "num_recv", "full_recv_rows")})
     for k, w, n in (("local_items", 4, v.num_local_items), ("remote_items", 4, v.num_remote_items),
                     ("splits", 3, v.num_splits)):
         ptr = getattr(v, k)
         d[k] = (np.ctypeslib.as_array(ptr, shape=(n * w,)).copy() if n > 0 else np.zeros(0, np.int32)).reshape(-1, w)
+    k1 = layout.view(part, arrays=False)["num_parts"] + 1
+    for k, n in (("send_idx", v.num_send), ("recv_idx", v.num_recv), ("send_off", k1 if k1 > 2 else 0),
+                 ("recv_off", k1 if k1 > 2 else 0)):
+        ptr = getattr(v, k)
+        d[k] = np.ctypeslib.as_array(ptr, shape=(n,)).copy() if n > 0 and ptr else np.zeros(0, np.int32)
     return d
 
 

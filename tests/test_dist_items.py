@@ -118,3 +118,27 @@ def test_single_part_has_no_dist_items():
     ip, ix = synth.random_multigraph(2, 50, 300)
     d = M.mega_layout_dist_view_get(M.mega_preprocess(ip, ix), 0)
     assert d["num_local_items"] == d["num_remote_items"] == d["num_splits"] == 0
+
+
+@pytest.mark.parametrize("k", [2, 4])
+def test_halo_plan(k):
+    """NEXT-1: part p receives from q exactly the rows of q its edges reference, and the
+    list p sends to q is the list q receives from p (same order: the packed buffers line up)."""
+    cfg = synth.scaled(synth.CONFIGS["products"], 4000, 60000)
+    ip, ix, _ = synth.make_graph(cfg)
+    lay = M.mega_preprocess(ip, ix, num_parts=k)
+    b = lay.view(0)["bounds"]
+    views = [lay.view(p) for p in range(k)]
+    dv = [M.mega_layout_dist_view_get(lay, p) for p in range(k)]
+    for p in range(k):
+        ref = np.unique(views[p]["src"])
+        for q in range(k):
+            r = dv[p]["recv_idx"][dv[p]["recv_off"][q]:dv[p]["recv_off"][q + 1]]
+            if q == p:
+                assert len(r) == 0
+                continue
+            assert np.array_equal(r, ref[(ref >= b[q]) & (ref < b[q + 1])])
+            s_qp = dv[q]["send_idx"][dv[q]["send_off"][p]:dv[q]["send_off"][p + 1]]
+            assert np.array_equal(s_qp, r)
+        assert dv[p]["num_recv"] == dv[p]["recv_off"][-1] <= dv[p]["full_recv_rows"]
+        assert dv[p]["full_recv_rows"] == cfg.n - (b[p + 1] - b[p])
