@@ -45,7 +45,8 @@ def parse():
     ap.add_argument("--impl", default="mega", choices=["mega", "reference"])
     ap.add_argument("--config", default="products")
     ap.add_argument("--dtype", default="bf16", choices=["bf16", "fp32"])
-    ap.add_argument("--order", default="traversal")
+    ap.add_argument("--order", default="traversal",
+                    help="traversal (MEGA), identity, degree, random, community (ablations, SURVEY 8(d)-d5)")
     ap.add_argument("--window", type=int, default=0, help="traversal window omega (0 = auto)")
     ap.add_argument("--seg-edges", type=int, default=0, help="work-item segment size S (0 = auto)")
     ap.add_argument("--block-rows", type=int, default=-1,
@@ -220,11 +221,21 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=
     indptr, indices, gstats = synth.make_graph(cfg)
     t_gen = time.time() - t0
     from paper_conf_icdcs_dengr24_b200 import mega as M
+    relabel = None
+    if order == "community":   # ablation upper bound: nodes sorted by generator community
+        comm = synth.communities(cfg)
+        relabel = np.lexsort((np.arange(cfg.n), comm))
+        ip_in, ix_in = synth.relabel(indptr, indices, relabel)
+        order, block_rows = "identity", 0
+    else:
+        ip_in, ix_in = indptr, indices
     t0 = time.time()
-    layout = M.mega_preprocess(indptr, indices, order=order, num_parts=world, window=window, seg_edges=seg_edges,
+    layout = M.mega_preprocess(ip_in, ix_in, order=order, num_parts=world, window=window, seg_edges=seg_edges,
                                block_rows=block_rows)
     t_pre = time.time() - t0
     perm = layout.view(0)["perm"].astype(np.int64)
+    if relabel is not None:
+        perm = relabel[perm]     # back to the generator's node ids
     layers = []
     in_dim = cfg.f_in
     for li in range(cfg.layers):

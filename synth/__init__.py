@@ -146,6 +146,36 @@ def make_graph(cfg: GraphConfig):
     return indptr, indices, {"duplicates": int(st[0]), "self_loops": int(st[1])}
 
 
+def communities(cfg: GraphConfig) -> np.ndarray:
+    """Community id of every node of make_graph(cfg) (the generator's own assignment,
+    comm[v] = draw(seed ^ 0x2222..., v) % C; used only for the community-sorted
+    upper-bound ablation order of bench.py)."""
+    if cfg.batch:
+        raise ValueError("batch workloads have no community structure")
+    M64 = np.uint64(0xFFFFFFFFFFFFFFFF)
+    with np.errstate(over="ignore"):
+        z = (np.uint64(cfg.seed ^ 0x2222222222222222) +
+             (np.arange(cfg.n, dtype=np.uint64) + np.uint64(1)) * np.uint64(0x9E3779B97F4A7C15)) & M64
+        z = (z ^ (z >> np.uint64(30))) * np.uint64(0xBF58476D1CE4E5B9)
+        z = (z ^ (z >> np.uint64(27))) * np.uint64(0x94D049BB133111EB)
+        z = z ^ (z >> np.uint64(31))
+    return (z % np.uint64(cfg.communities)).astype(np.int32)
+
+
+def relabel(indptr, indices, order):
+    """The same graph with node order[r] renamed r (rows permuted, sources renamed)."""
+    indptr = np.asarray(indptr, np.int64)
+    order = np.asarray(order, np.int64)
+    n = len(indptr) - 1
+    new_of = np.empty(n, np.int64)
+    new_of[order] = np.arange(n)
+    deg = np.diff(indptr)[order]
+    ip2 = np.zeros(n + 1, np.int64)
+    np.cumsum(deg, out=ip2[1:])
+    pos = np.repeat(indptr[order] - ip2[:-1], deg) + np.arange(ip2[-1])
+    return ip2, new_of[np.asarray(indices)[pos]].astype(np.int32)
+
+
 def normal(seed: int, shape, scale: float = 1.0) -> np.ndarray:
     lib = _load()
     out = np.empty(int(np.prod(shape)), dtype=np.float32)

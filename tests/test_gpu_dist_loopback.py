@@ -55,8 +55,11 @@ def run_dist(layout, Wh_old, a_l, a_r, g_old, dtype, dev="cuda"):
             M.mega_gat_fwd_dist(layout, p, comms[p], r["feat"], al, ar, H, F, r["out"], r["ctx"], r["wsf"],
                                 flags=phase, comm_stream=r["cs"])
     torch.cuda.synchronize()
-    for r in R:   # every rank now holds every row, bit for bit
-        assert torch.equal(r["feat"], Wh_new)
+    er_owned = torch.cat([r["ctx"][1][r["b0"]:r["b1"]] for r in R])   # er of every row, from its owner
+    for p, r in enumerate(R):   # every rank now holds, bit for bit, every row its edges reference (NEXT-1 halo)
+        need = torch.tensor(np.unique(layout.view(p)["src"]).astype(np.int64), device=dev)
+        assert torch.equal(r["feat"][need], Wh_new[need])
+        assert torch.equal(r["ctx"][1][need], er_owned[need])
     for phase in (M.MEGA_DIST_PHASE_SEND, M.MEGA_DIST_PHASE_RECV):
         for p, r in enumerate(R):
             M.mega_gat_bwd_dist(layout, p, comms[p], r["feat"], al, ar, H, F, r["out"], g_new[r["b0"]:r["b1"]],
