@@ -820,20 +820,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
     }
     cp_async_commit();
   };
-  // each warp claims the next CH sources of the CSC order from the work counter, so the warps stay
-  // within a narrow window of the order and the g rows they gather share L2 (see gat_fwd_pipe_kernel)
-  constexpr int CH = 4;
-  int cbase = 0, cpos = CH;
-  auto next_item = [&]() -> int64_t {
-    if (cpos == CH) {
-      int c = 0;
-      if (lane == 0) c = atomicAdd(a.sched, CH);
-      cbase = __shfl_sync(0xffffffffu, c, 0);
-      cpos = 0;
-    }
-    return (int64_t)cbase + cpos++;
-  };
-  for (int64_t it = next_item(); it < a.L.n_bwd_items; it = next_item()) {
+  for (int64_t it = (int64_t)blockIdx.x * WPB + w; it < a.L.n_bwd_items; it += stride) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
     float whf[V][EPV], acc[V][EPV], derv[V], dacc = 0.f;
@@ -1493,7 +1480,6 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
             cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nblk, kr, TPB, smem);
             const int grid = (int)std::min<int64_t>((a.L.n_bwd_items + WPB - 1) / WPB,
                                                     (int64_t)dev_info(dev).sms * std::max(nblk, 1));
-            cudaMemsetAsync(a.sched, 0, sizeof(int), st);   // the ring kernel's work counter
             kr<<<std::max(grid, 1), TPB, smem, st>>>(a);
             ring = true;
           }

@@ -332,6 +332,211 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
   }
 }
 
+
+// ---------------- persistent, warp-specialised form (fwd and dX) ----------------
+// One CTA per SM loops over output tiles (tile t: row tile t / ntiles, column tile t % ntiles, so
+// consecutive tiles share their A rows through L2).  Warp 0 (one lane) streams A/B k-blocks through
+// a STAGES-deep TMA ring across tile boundaries; warp 1 (one lane) issues tcgen05.mma into one of
+// TWO TMEM accumulators; warps 2-5 drain the other accumulator at the same time: tcgen05.ld ->
+// bf16 -> swizzled shared-memory box -> TMA store (two 64-column boxes in flight), el/er on the way.
+// So loads, MMAs and the epilogue of consecutive tiles overlap; barriers: full/empty per ring slot,
+// tmem_full/tmem_empty per accumulator.
+template <int BN> struct PTiles {
+  static constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
+  static constexpr int OUT_BOX = BM * 128;                      // one 64-column bf16 box, 16 KB
+  static constexpr int STAGES = (200 * 1024 - 2 * OUT_BOX) / STAGE > 8 ? 8 : (200 * 1024 - 2 * OUT_BOX) / STAGE;
+  static constexpr int ACC_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int TMEM_COLS = 2 * ACC_COLS;
+  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + 2 * OUT_BOX + 512 + 2 * 1024 * 4;
+};
+constexpr int PTHREADS = 192;
+
+template <int MODE, int BN, int FH>
+__global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid_constant__ CUtensorMap tmA,
+                                                                    const __grid_constant__ CUtensorMap tmB,
+                                                                    const __grid_constant__ CUtensorMap tmO,
+                                                                    const Args g) {
+  using TL = PTiles<BN>;
+  constexpr int STAGES = TL::STAGES;
+  static_assert(MODE == FWD || MODE == DX, "persistent kernel: fwd and dX");
+  constexpr bool B_MN = MODE == FWD;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
+  uint8_t *outb = smem + STAGES * TL::STAGE;                         // 2 output boxes
+  uint64_t *bars = reinterpret_cast<uint64_t *>(outb + 2 * TL::OUT_BOX);
+  // bars: full[S], empty[S], tfull[2], tempty[2]
+  uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 4);
+  float *s_al = reinterpret_cast<float *>(outb + 2 * TL::OUT_BOX + 512);
+  float *s_ar = s_al + 1024;
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
+  const uint32_t tfull0 = smem_u32(bars + 2 * STAGES), tempty0 = smem_u32(bars + 2 * STAGES + 2);
+  const int64_t mtiles = (g.M + BM - 1) / BM, ntile_total = mtiles * g.ntiles;
+  const int nkb = (int)g.kb_total;
+
+  if (MODE == FWD)
+    for (int c = threadIdx.x; c < g.Nc; c += PTHREADS) { s_al[c] = g.al[c]; s_ar[c] = g.ar[c]; }
+  if (warp == 0 && lane == 0) {
+    prefetch_tmap(&tmA);
+    prefetch_tmap(&tmB);
+    prefetch_tmap(&tmO);
+    for (int s2 = 0; s2 < STAGES; ++s2) {
+      mbar_init(full0 + 8 * s2, 1);
+      mbar_init(empty0 + 8 * s2, 1);
+    }
+    for (int a2 = 0; a2 < 2; ++a2) {
+      mbar_init(tfull0 + 8 * a2, 1);
+      mbar_init(tempty0 + 8 * a2, 4);       // one arrive per epilogue warp
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+  }
+  if (warp == 1) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tslot)),
+                 "r"((uint32_t)TL::TMEM_COLS)
+                 : "memory");
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;" ::: "memory");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem = *tslot;
+
+  if (warp == 0) {
+    if (lane == 0) {   // ---- TMA producer: k-blocks of every tile of this CTA, through the ring ----
+      int64_t kc = 0;
+      for (int64_t t = blockIdx.x; t < ntile_total; t += gridDim.x) {
+        const int32_t m0 = (int32_t)((t / g.ntiles) * BM), n0 = (int32_t)((t % g.ntiles) * BN);
+        for (int i = 0; i < nkb; ++i, ++kc) {
+          const int s2 = (int)(kc % STAGES);
+          mbar_wait(empty0 + 8 * s2, (uint32_t)((kc / STAGES) & 1) ^ 1u);
+          const uint32_t full = full0 + 8 * s2;
+          mbar_expect_tx(full, TL::STAGE);
+          const uint32_t sa = smem_u32(smem + s2 * TL::STAGE), sb = sa + TL::A_BYTES;
+          const int32_t k = i * BK;
+          tma_load_2d(sa, &tmA, k, m0, full);
+          if constexpr (B_MN) {
+#pragma unroll
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * 8192, &tmB, n0 + 64 * j, k, full);
+          } else {
+            tma_load_2d(sb, &tmB, k, n0, full);
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {   // ---- MMA issuer ----
+      constexpr uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((B_MN ? 1u : 0u) << 16) |
+                                 ((uint32_t)(BN >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+      int64_t kc = 0, it = 0;
+      for (int64_t t = blockIdx.x; t < ntile_total; t += gridDim.x, ++it) {
+        const int acc = (int)(it & 1);
+        mbar_wait(tempty0 + 8 * acc, (uint32_t)((it >> 1) & 1) ^ 1u);   // the epilogue drained it
+        tc_fence_after();
+        const uint32_t td = tmem + (uint32_t)(acc * TL::ACC_COLS);
+        for (int i = 0; i < nkb; ++i, ++kc) {
+          const int s2 = (int)(kc % STAGES);
+          mbar_wait(full0 + 8 * s2, (uint32_t)((kc / STAGES) & 1));
+          tc_fence_after();
+          const uint32_t sa = smem_u32(smem + s2 * TL::STAGE), sb = sa + TL::A_BYTES;
+#pragma unroll
+          for (int kk = 0; kk < BK / 16; ++kk) {
+            const uint64_t da = sdesc(sa + kk * 32, 16, 1024);
+            const uint64_t db = B_MN ? sdesc(sb + kk * 2048, 8192, 1024) : sdesc(sb + kk * 32, 16, 1024);
+            umma_f16(td, da, db, idesc, (i | kk) ? 1u : 0u);
+          }
+          umma_commit(empty0 + 8 * s2);
+        }
+        umma_commit(tfull0 + 8 * acc);
+      }
+    }
+  } else {
+    // ---- epilogue warps 2..5: TMEM lanes 32 (warp % 4) .. +31 = tile rows ----
+    const int ew = warp & 3, row = ew * 32 + lane, et = threadIdx.x - 64;   // et: 0..127
+    const uint32_t obase = smem_u32(outb);
+    int64_t it = 0, chunk = 0;
+    for (int64_t t = blockIdx.x; t < ntile_total; t += gridDim.x, ++it) {
+      const int64_t m0 = (t / g.ntiles) * BM;
+      const int n0 = (int)((t % g.ntiles) * BN);
+      const int acc = (int)(it & 1);
+      mbar_wait(tfull0 + 8 * acc, (uint32_t)((it >> 1) & 1));
+      tc_fence_after();
+      const uint32_t taddr = tmem + (uint32_t)(acc * TL::ACC_COLS) + ((uint32_t)(ew * 32) << 16);
+      const int64_t grow = m0 + row;
+      const bool live = grow < g.M;
+      float el_acc = 0.f, er_acc = 0.f;
+#pragma unroll 1
+      for (int c64 = 0; c64 < BN; c64 += 64, ++chunk) {
+        const int b = (int)(chunk & 1);
+        // the TMA store that last read box b must be done before it is rewritten
+        if (et == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        const uint32_t box = obase + (uint32_t)b * TL::OUT_BOX + (uint32_t)row * 128;
+#pragma unroll
+        for (int h32 = 0; h32 < 2; ++h32) {
+          const int c0 = c64 + 32 * h32;
+          uint32_t r[32];
+          tmem_ld32(taddr + c0, r);
+          uint32_t p[16];
+#pragma unroll
+          for (int q = 0; q < 16; ++q) p[q] = bf2(__uint_as_float(r[2 * q]), __uint_as_float(r[2 * q + 1]));
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            const uint32_t u = (uint32_t)(4 * h32 + q);
+            asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(box + ((u ^ (uint32_t)(row & 7)) << 4)),
+                         "r"(p[4 * q]), "r"(p[4 * q + 1]), "r"(p[4 * q + 2]), "r"(p[4 * q + 3])
+                         : "memory");
+          }
+          if constexpr (MODE == FWD) {   // el/er from the stored (bf16-rounded) Wh, head by head
+#pragma unroll
+            for (int sgm = 0; sgm < 32 / FH; ++sgm) {
+#pragma unroll
+              for (int q = 0; q < FH; q += 2) {
+                const uint32_t w2 = p[(sgm * FH + q) / 2];
+                const float x0 = __uint_as_float(w2 << 16), x1 = __uint_as_float(w2 & 0xffff0000u);
+                const int c = n0 + c0 + sgm * FH + q;
+                el_acc = fmaf(s_al[c], x0, el_acc);
+                el_acc = fmaf(s_al[c + 1], x1, el_acc);
+                er_acc = fmaf(s_ar[c], x0, er_acc);
+                er_acc = fmaf(s_ar[c + 1], x1, er_acc);
+              }
+              const int cend = c0 + (sgm + 1) * FH;
+              if (cend % g.F == 0) {
+                const int h = (n0 + cend) / g.F - 1;
+                if (live) {
+                  g.el[(g.ctx_row0 + grow) * g.H + h] = el_acc;
+                  g.er[(g.ctx_row0 + grow) * g.H + h] = er_acc;
+                }
+                el_acc = 0.f;
+                er_acc = 0.f;
+              }
+            }
+          }
+        }
+        if (c64 + 64 >= BN) {   // this thread's TMEM reads of the tile are done: release the accumulator
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(tempty0 + 8 * acc) : "memory");
+        }
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+        asm volatile("bar.sync 1, 128;" ::: "memory");
+        if (et == 0) {
+          if (n0 + c64 < g.Nc) tma_store_2d(&tmO, obase + (uint32_t)b * TL::OUT_BOX, n0 + c64, (int32_t)m0);
+          asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+        }
+      }
+    }
+    if (et == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+  }
+  __syncwarp();
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"((uint32_t)TL::TMEM_COLS)
+                 : "memory");
+  }
+}
+
 // dW: fixed-order sum of the split partials (deterministic), fp32
 __global__ void __launch_bounds__(256) dw_reduce_kernel(const float *parts, int splits, int64_t mpad, int K, int D,
                                                         float *out) {
@@ -407,6 +612,25 @@ mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap
   return MEGA_OK;
 }
 
+template <int MODE, int BN, int FH>
+mega_status launch_persistent(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap &o, const Args &g,
+                              cudaStream_t st) {
+  auto k = umma_gemm_persistent<MODE, BN, FH>;
+  const size_t smem = PTiles<BN>::SMEM;
+  static bool attr = false;  // per instantiation
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma smem attribute: ") + cudaGetErrorString(e));
+    attr = true;
+  }
+  const int64_t tiles = ((g.M + BM - 1) / BM) * g.ntiles;
+  const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, sm_count()));
+  k<<<grid, PTHREADS, smem, st>>>(a, b, o, g);
+  cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma_gemm_persistent: ") + cudaGetErrorString(e));
+  return MEGA_OK;
+}
+
 }  // namespace umma
 
 using namespace umma;
@@ -433,23 +657,23 @@ mega_status umma_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_di
   const dim3 grid((unsigned)(((rows + BM - 1) / BM) * g.ntiles), 1, 1);
   const int fh = std::min(head_dim, 32);
   if (BN == 256) {
-    if (fh == 32) return launch<FWD, 256, 32>(ta, tb, to, g, grid, st);
-    if (fh == 16) return launch<FWD, 256, 16>(ta, tb, to, g, grid, st);
-    return launch<FWD, 256, 8>(ta, tb, to, g, grid, st);
+    if (fh == 32) return launch_persistent<FWD, 256, 32>(ta, tb, to, g, st);
+    if (fh == 16) return launch_persistent<FWD, 256, 16>(ta, tb, to, g, st);
+    return launch_persistent<FWD, 256, 8>(ta, tb, to, g, st);
   }
   if (BN == 128) {
-    if (fh == 32) return launch<FWD, 128, 32>(ta, tb, to, g, grid, st);
-    if (fh == 16) return launch<FWD, 128, 16>(ta, tb, to, g, grid, st);
-    return launch<FWD, 128, 8>(ta, tb, to, g, grid, st);
+    if (fh == 32) return launch_persistent<FWD, 128, 32>(ta, tb, to, g, st);
+    if (fh == 16) return launch_persistent<FWD, 128, 16>(ta, tb, to, g, st);
+    return launch_persistent<FWD, 128, 8>(ta, tb, to, g, st);
   }
   if (BN == 192) {
-    if (fh == 32) return launch<FWD, 192, 32>(ta, tb, to, g, grid, st);
-    if (fh == 16) return launch<FWD, 192, 16>(ta, tb, to, g, grid, st);
-    return launch<FWD, 192, 8>(ta, tb, to, g, grid, st);
+    if (fh == 32) return launch_persistent<FWD, 192, 32>(ta, tb, to, g, st);
+    if (fh == 16) return launch_persistent<FWD, 192, 16>(ta, tb, to, g, st);
+    return launch_persistent<FWD, 192, 8>(ta, tb, to, g, st);
   }
-  if (fh == 32) return launch<FWD, 64, 32>(ta, tb, to, g, grid, st);
-  if (fh == 16) return launch<FWD, 64, 16>(ta, tb, to, g, grid, st);
-  return launch<FWD, 64, 8>(ta, tb, to, g, grid, st);
+  if (fh == 32) return launch_persistent<FWD, 64, 32>(ta, tb, to, g, st);
+  if (fh == 16) return launch_persistent<FWD, 64, 16>(ta, tb, to, g, st);
+  return launch_persistent<FWD, 64, 8>(ta, tb, to, g, st);
 }
 
 // dX[rows][in_dim] = dWh W^T (bf16 out).  K = D (multiple of 64).  Columns are written in
@@ -468,9 +692,9 @@ mega_status umma_project_dx(const void *gf, int64_t ldgf, int64_t rows, int in_d
   g.M = rows; g.Nc = (in_dim + 7) / 8 * 8; g.kb_total = D / BK; g.kb_split = g.kb_total; g.out = gx; g.ldo = ldgx;
   g.ntiles = (in_dim + BN - 1) / BN;
   const dim3 grid((unsigned)(((rows + BM - 1) / BM) * g.ntiles), 1, 1);
-  if (BN == 256) return launch<DX, 256, 32>(ta, tb, to, g, grid, st);
-  if (BN == 128) return launch<DX, 128, 32>(ta, tb, to, g, grid, st);
-  return launch<DX, 64, 32>(ta, tb, to, g, grid, st);
+  if (BN == 256) return launch_persistent<DX, 256, 32>(ta, tb, to, g, st);
+  if (BN == 128) return launch_persistent<DX, 128, 32>(ta, tb, to, g, st);
+  return launch_persistent<DX, 64, 32>(ta, tb, to, g, st);
 }
 
 // workspace of umma_project_dw: split partials
