@@ -226,47 +226,26 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
   const T *feat = static_cast<const T *>(a.feat);
   const T *featl = feat + gl * EPV;
-  const int64_t n_items = a.L.n_fwd_items;
+  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
+  const int64_t it0 = ((int64_t)blockIdx.x * WPB + w) * GPW + grp, n_items = a.L.n_fwd_items;
+  if (it0 >= n_items) return;
   auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
     const T *rp = featl + (jj & idm) * ldf;
     const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
     for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
-  // descriptor batch k: the group claims the next G items of the layout order from the work
-  // counter (items [cl, cl + G)), so all groups stay within a narrow window of the MEGA order and
-  // the rows they gather stay L2-resident together (a static grid-stride split drifts apart with
-  // the degree skew); results do not depend on which group takes an item
-  int cl[2];
+  // descriptor batch k: items it0 + (kG + l) stride, l < G, into s_desc[k & 1].  Static striding keeps
+  // the groups in a window of ~gridDim * WPB * GPW consecutive rows of the MEGA order (measured: dynamic
+  // claims of G consecutive items per group widen that window G-fold and cost 40% on products)
   auto stage_desc = [&](int k) {
-    int c = 0;
-    if (gl == 0) c = atomicAdd(a.sched, G);
-    c = __shfl_sync(gmask, c, rb);
-    cl[k & 1] = c;
-    const int64_t itq = (int64_t)c + gl;
+    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
     if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][rb + gl], a.L.fwd_items + itq);
-    cp_async_commit();
-  };
-  // chunk (itm, bse): source ids (tail lanes repeat the last edge) and, for the first chunk of an item, el
-  auto stage_src = [&](int b, int4 itm, int bse) {
-    if (itm.z > itm.y) cp_async_small<4>(&s_src[b][w][rb + gl], a.L.src + min(bse + gl, itm.z - 1));
-    else s_src[b][w][rb + gl] = 0;
-    if (bse == itm.y && gl == 0) cp_async_h<HT>(&s_el[b][w][grp][0], a.el + (a.L.row_begin + itm.x) * H);
-    cp_async_commit();
-  };
-  // er of the staged chunk's sources, and their rows into L2
-  auto stage_er = [&](int b, int4 itm, int bse) {
-    const uint32_t jj = (uint32_t)s_src[b][w][rb + gl];
-    cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
     cp_async_commit();
   };
   // prologue: descriptor batches 0 and 1, chunk 0 staged
   stage_desc(0);
   stage_desc(1);
-  if (cl[0] >= n_items) {
-    cp_async_wait<0>();
-    return;
-  }
   cp_async_wait<1>();
   __syncwarp(gmask);
   int q = 0;
@@ -287,7 +266,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
     bool has_next = true;
     if (nbase >= item.z) {
       nq = q + 1;
-      if ((int64_t)cl[(nq / G) & 1] + nq % G >= n_items) {
+      if (it0 + (int64_t)nq * stride >= n_items) {
         has_next = false;
       } else {
         if (nq % G == 0) {  // entering descriptor batch nq/G: make sure it landed, refill the other buffer
@@ -1354,18 +1333,17 @@ mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
   return MEGA_OK;
 }
 
-struct WsFwd { size_t m, l, acc, sched, total; };
+struct WsFwd { size_t m, l, acc, total; };
 WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   WsFwd w;
   size_t slots = (size_t)std::max(1, D.n_fwd_slots);
   w.m = 0;
   w.l = align256(w.m + slots * s.H * 4);
   w.acc = align256(w.l + slots * s.H * 4);
-  w.sched = align256(w.acc + slots * s.D * 4);
-  w.total = w.sched + 256;
+  w.total = align256(w.acc + slots * s.D * 4);
   return w;
 }
-struct WsBwd { size_t dz, bacc, bder, dal, dar, sched, total; };
+struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
 WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   WsBwd w;
   size_t slots = (size_t)std::max(1, D.n_bwd_slots);
@@ -1374,8 +1352,7 @@ WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   w.bder = align256(w.bacc + slots * s.D * 4);
   w.dal = align256(w.bder + slots * s.H * 4);
   w.dar = align256(w.dal + (size_t)MAX_GRID * s.D * 8);
-  w.sched = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
-  w.total = w.sched + 256;
+  w.total = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
   return w;
 }
 DevPart host_counts(const Part &P, int64_t n) {  // sizes without binding
@@ -1434,12 +1411,8 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
         };
         // chunk-pipelined kernel for groups of >= 8 lanes (products 3 layers: 25.5 vs 29.3 ms/step for the
         // register-batch kernel, which stays for narrow rows: static shared memory of the pipe kernel)
-        if constexpr (G >= 8) {
-          cudaMemsetAsync(a.sched, 0, sizeof(int), st);   // the pipe kernel's work counter
-          launch(gat_fwd_pipe_kernel<T, G, V, HT>);
-        } else {
-          launch(gat_fwd_kernel<T, G, V, HT, 0>);
-        }
+        if constexpr (G >= 8) launch(gat_fwd_pipe_kernel<T, G, V, HT>);
+        else launch(gat_fwd_kernel<T, G, V, HT, 0>);
       });
       if (rc != MEGA_OK) return;
     }
@@ -1565,7 +1538,6 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.sched = reinterpret_cast<int *>(wb + w.sched);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
@@ -1612,7 +1584,6 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
   a.ws_dal = reinterpret_cast<double *>(wb + w.dal);
   a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
-  a.sched = reinterpret_cast<int *>(wb + w.sched);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
@@ -1744,7 +1715,6 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.sched = reinterpret_cast<int *>(wb + w.sched);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   auto pass = [&](const int4 *items, int32_t nitems, const int32_t *splits, int32_t nsplits) {
@@ -1844,7 +1814,6 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.ws_bder = reinterpret_cast<float *>(wb + w.bder);
   a.ws_dal = reinterpret_cast<double *>(wb + w.dal);
   a.ws_dar = reinterpret_cast<double *>(wb + w.dar);
-  a.sched = reinterpret_cast<int *>(wb + w.sched);
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;

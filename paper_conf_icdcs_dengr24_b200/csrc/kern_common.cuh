@@ -288,7 +288,6 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
-  int *sched;   // work counter (zeroed before each launch): groups claim the next items in layout order
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
   int pol_mode; // MEGA_L2_POLICY
 };
@@ -315,7 +314,6 @@ struct BwdArgs {
   float *gal, *gar;
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
-  int *sched;   // work counter of the source pass (zeroed before each launch)
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int pol_mode; // MEGA_L2_POLICY
 };

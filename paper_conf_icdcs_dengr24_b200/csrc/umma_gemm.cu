@@ -341,32 +341,36 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
 // bf16 -> swizzled shared-memory box -> TMA store (two 64-column boxes in flight), el/er on the way.
 // So loads, MMAs and the epilogue of consecutive tiles overlap; barriers: full/empty per ring slot,
 // tmem_full/tmem_empty per accumulator.
-template <int BN> struct PTiles {
+// EPI epilogue warpgroups (1 or 2): warpgroup e drains columns [e BN/EPI, (e+1) BN/EPI) of the
+// accumulator (TMEM lanes are tied to warp % 4, so two warpgroups split the columns, not the rows).
+template <int BN, int EPI> struct PTiles {
   static constexpr int A_BYTES = BM * BK * 2, B_BYTES = BN * BK * 2, STAGE = A_BYTES + B_BYTES;
   static constexpr int OUT_BOX = BM * 128;                      // one 64-column bf16 box, 16 KB
-  static constexpr int STAGES = (200 * 1024 - 2 * OUT_BOX) / STAGE > 8 ? 8 : (200 * 1024 - 2 * OUT_BOX) / STAGE;
+  static constexpr int OUT = 2 * EPI * OUT_BOX;                 // two boxes in flight per warpgroup
+  static constexpr int STAGES = (216 * 1024 - OUT) / STAGE > 8 ? 8 : (216 * 1024 - OUT) / STAGE;
   static constexpr int ACC_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr int TMEM_COLS = 2 * ACC_COLS;
-  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + 2 * OUT_BOX + 512 + 2 * 1024 * 4;
+  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + OUT + 512 + 2 * 1024 * 4;
+  static constexpr int THREADS = 64 + 128 * EPI;
 };
-constexpr int PTHREADS = 192;
 
-template <int MODE, int BN, int FH>
-__global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid_constant__ CUtensorMap tmA,
-                                                                    const __grid_constant__ CUtensorMap tmB,
-                                                                    const __grid_constant__ CUtensorMap tmO,
-                                                                    const Args g) {
-  using TL = PTiles<BN>;
+template <int MODE, int BN, int FH, int EPI>
+__global__ void __launch_bounds__(PTiles<BN, EPI>::THREADS, 1)
+    umma_gemm_persistent(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                         const __grid_constant__ CUtensorMap tmO, const Args g) {
+  using TL = PTiles<BN, EPI>;
+  constexpr int PTHREADS = TL::THREADS, CW = BN / EPI;    // columns per epilogue warpgroup
+  static_assert(CW % 64 == 0 || EPI == 1, "a warpgroup's columns are whole 64-column boxes");
   constexpr int STAGES = TL::STAGES;
   static_assert(MODE == FWD || MODE == DX, "persistent kernel: fwd and dX");
   constexpr bool B_MN = MODE == FWD;
   extern __shared__ uint8_t smem_raw[];
   uint8_t *smem = reinterpret_cast<uint8_t *>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~(uintptr_t)1023);
-  uint8_t *outb = smem + STAGES * TL::STAGE;                         // 2 output boxes
-  uint64_t *bars = reinterpret_cast<uint64_t *>(outb + 2 * TL::OUT_BOX);
+  uint8_t *outb = smem + STAGES * TL::STAGE;                         // 2 output boxes per warpgroup
+  uint64_t *bars = reinterpret_cast<uint64_t *>(outb + TL::OUT);
   // bars: full[S], empty[S], tfull[2], tempty[2]
   uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 4);
-  float *s_al = reinterpret_cast<float *>(outb + 2 * TL::OUT_BOX + 512);
+  float *s_al = reinterpret_cast<float *>(outb + TL::OUT + 512);
   float *s_ar = s_al + 1024;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
@@ -386,7 +390,7 @@ __global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid
     }
     for (int a2 = 0; a2 < 2; ++a2) {
       mbar_init(tfull0 + 8 * a2, 1);
-      mbar_init(tempty0 + 8 * a2, 4);       // one arrive per epilogue warp
+      mbar_init(tempty0 + 8 * a2, 4 * EPI);       // one arrive per epilogue warp
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -451,9 +455,11 @@ __global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid
       }
     }
   } else {
-    // ---- epilogue warps 2..5: TMEM lanes 32 (warp % 4) .. +31 = tile rows ----
-    const int ew = warp & 3, row = ew * 32 + lane, et = threadIdx.x - 64;   // et: 0..127
-    const uint32_t obase = smem_u32(outb);
+    // ---- epilogue warps 2..: TMEM lanes 32 (warp % 4) .. +31 = tile rows; warpgroup ewg takes
+    // columns [ewg CW, (ewg+1) CW) of each tile ----
+    const int ew = warp & 3, ewg = (warp - 2) / 4, row = ew * 32 + lane, et = threadIdx.x - 64 - 128 * ewg;
+    const uint32_t obase = smem_u32(outb) + (uint32_t)(ewg * 2 * TL::OUT_BOX);
+    const int bar_id = 1 + ewg;
     int64_t it = 0, chunk = 0;
     for (int64_t t = blockIdx.x; t < ntile_total; t += gridDim.x, ++it) {
       const int64_t m0 = (t / g.ntiles) * BM;
@@ -466,11 +472,11 @@ __global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid
       const bool live = grow < g.M;
       float el_acc = 0.f, er_acc = 0.f;
 #pragma unroll 1
-      for (int c64 = 0; c64 < BN; c64 += 64, ++chunk) {
+      for (int c64 = ewg * CW; c64 < (ewg + 1) * CW; c64 += 64, ++chunk) {
         const int b = (int)(chunk & 1);
         // the TMA store that last read box b must be done before it is rewritten
         if (et == 0) asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
-        asm volatile("bar.sync 1, 128;" ::: "memory");
+        asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
         const uint32_t box = obase + (uint32_t)b * TL::OUT_BOX + (uint32_t)row * 128;
 #pragma unroll
         for (int h32 = 0; h32 < 2; ++h32) {
@@ -513,13 +519,13 @@ __global__ void __launch_bounds__(PTHREADS, 1) umma_gemm_persistent(const __grid
             }
           }
         }
-        if (c64 + 64 >= BN) {   // this thread's TMEM reads of the tile are done: release the accumulator
+        if (c64 + 64 >= (ewg + 1) * CW) {   // this thread's TMEM reads of the tile are done: release
           tc_fence_before();
           __syncwarp();
           if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(tempty0 + 8 * acc) : "memory");
         }
         asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
-        asm volatile("bar.sync 1, 128;" ::: "memory");
+        asm volatile("bar.sync %0, 128;" ::"r"(bar_id) : "memory");
         if (et == 0) {
           if (n0 + c64 < g.Nc) tma_store_2d(&tmO, obase + (uint32_t)b * TL::OUT_BOX, n0 + c64, (int32_t)m0);
           asm volatile("cp.async.bulk.commit_group;" ::: "memory");
@@ -612,11 +618,11 @@ mega_status launch(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap
   return MEGA_OK;
 }
 
-template <int MODE, int BN, int FH>
-mega_status launch_persistent(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap &o, const Args &g,
-                              cudaStream_t st) {
-  auto k = umma_gemm_persistent<MODE, BN, FH>;
-  const size_t smem = PTiles<BN>::SMEM;
+template <int MODE, int BN, int FH, int EPI>
+mega_status launch_persistent_e(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap &o, const Args &g,
+                                cudaStream_t st) {
+  auto k = umma_gemm_persistent<MODE, BN, FH, EPI>;
+  const size_t smem = PTiles<BN, EPI>::SMEM;
   static bool attr = false;  // per instantiation
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -625,10 +631,19 @@ mega_status launch_persistent(const CUtensorMap &a, const CUtensorMap &b, const 
   }
   const int64_t tiles = ((g.M + BM - 1) / BM) * g.ntiles;
   const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(tiles, sm_count()));
-  k<<<grid, PTHREADS, smem, st>>>(a, b, o, g);
+  k<<<grid, PTiles<BN, EPI>::THREADS, smem, st>>>(a, b, o, g);
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("umma_gemm_persistent: ") + cudaGetErrorString(e));
   return MEGA_OK;
+}
+// two epilogue warpgroups when each half of the tile is whole 64-column boxes holding whole heads
+template <int MODE, int BN, int FH>
+mega_status launch_persistent(const CUtensorMap &a, const CUtensorMap &b, const CUtensorMap &o, const Args &g,
+                              cudaStream_t st) {
+  if constexpr (BN % 128 == 0) {
+    if (MODE == DX || (BN / 2) % g.F == 0) return launch_persistent_e<MODE, BN, FH, 2>(a, b, o, g, st);
+  }
+  return launch_persistent_e<MODE, BN, FH, 1>(a, b, o, g, st);
 }
 
 }  // namespace umma
