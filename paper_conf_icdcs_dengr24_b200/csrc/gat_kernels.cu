@@ -243,6 +243,19 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
     if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][rb + gl], a.L.fwd_items + itq);
     cp_async_commit();
   };
+  // chunk (itm, bse): source ids (tail lanes repeat the last edge) and, for the first chunk of an item, el
+  auto stage_src = [&](int b, int4 itm, int bse) {
+    if (itm.z > itm.y) cp_async_small<4>(&s_src[b][w][rb + gl], a.L.src + min(bse + gl, itm.z - 1));
+    else s_src[b][w][rb + gl] = 0;
+    if (bse == itm.y && gl == 0) cp_async_h<HT>(&s_el[b][w][grp][0], a.el + (a.L.row_begin + itm.x) * H);
+    cp_async_commit();
+  };
+  // er of the staged chunk's sources
+  auto stage_er = [&](int b, int4 itm, int bse) {
+    const uint32_t jj = (uint32_t)s_src[b][w][rb + gl];
+    cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
+    cp_async_commit();
+  };
   // prologue: descriptor batches 0 and 1, chunk 0 staged
   stage_desc(0);
   stage_desc(1);
