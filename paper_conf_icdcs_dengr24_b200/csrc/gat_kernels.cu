@@ -1520,6 +1520,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
                          uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws, size_t ws_bytes,
                          mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gat_fwd");
   int dev = 0;
   mega_status rc = check_part(L, part, dev);
   if (rc != MEGA_OK) return rc;
@@ -1562,6 +1563,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
                          float *grad_feat, int64_t ldgf, void *grad_feat_lp, int64_t ldlp, float *grad_attn_l,
                          float *grad_attn_r, void *ws, size_t ws_bytes, mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gat_bwd");
   int dev = 0;
   mega_status rc = check_part(L, part, dev);
   if (rc != MEGA_OK) return rc;
@@ -1691,6 +1693,7 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
                               float negative_slope, uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws,
                               size_t ws_bytes, mega_stream_t stream, mega_stream_t comm_stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gat_fwd_dist");
   int dev = 0;
   mega_status rc = check_part(L, part, dev);
   if (rc != MEGA_OK) return rc;
@@ -1784,6 +1787,7 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
                               int64_t ldlp, float *grad_attn_l, float *grad_attn_r, void *ws, size_t ws_bytes,
                               mega_stream_t stream, mega_stream_t comm_stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gat_bwd_dist");
   int dev = 0;
   mega_status rc = check_part(L, part, dev);
   if (rc != MEGA_OK) return rc;

@@ -269,6 +269,7 @@ mega_status mega_gt_workspace_bytes(const mega_layout *L, int32_t part, int head
 mega_status mega_gt_fwd(const mega_layout *L, int32_t part, const float *q, const float *k, const float *v, int64_t ld,
                         int heads, int head_dim, float *out, int64_t ldo, float *lse, mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gt_fwd");
   int sms = 0;
   mega_status rc = gt::check(L, part, heads, head_dim, sms);
   if (rc != MEGA_OK) return rc;
@@ -290,6 +291,7 @@ mega_status mega_gt_bwd(const mega_layout *L, int32_t part, const float *q, cons
                         const float *grad_out, int64_t ldg, float *grad_q, float *grad_k, float *grad_v, int64_t ldgr,
                         void *ws, size_t ws_bytes, mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_gt_bwd");
   int sms = 0;
   mega_status rc = gt::check(L, part, heads, head_dim, sms);
   if (rc != MEGA_OK) return rc;

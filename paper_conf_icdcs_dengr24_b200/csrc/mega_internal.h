@@ -5,11 +5,21 @@
 #include <vector>
 
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 #include <vector_types.h>
 
 #include "../../include/mega.h"
 
 namespace mega {
+
+// NVTX range around every C-ABI compute call (header-only NVTX3: a no-op unless a tool such as
+// Nsight Systems / ncu --nvtx is attached), so profiles show the library calls by name.
+struct NvtxRange {
+  explicit NvtxRange(const char *name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+  NvtxRange(const NvtxRange &) = delete;
+  NvtxRange &operator=(const NvtxRange &) = delete;
+};
 
 // Sets the thread-local error message and returns the status.
 mega_status fail(mega_status s, const std::string &msg);

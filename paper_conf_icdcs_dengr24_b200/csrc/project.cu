@@ -86,6 +86,7 @@ mega_status mega_project_fwd(const void *x, int64_t ldx, int64_t rows, int in_di
                              int head_dim, const float *attn_l, const float *attn_r, mega_dtype dtype, void *feat,
                              int64_t ldf, float *ctx, int64_t ctx_n, int64_t ctx_row0, mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_project_fwd");
   mega_status rc = check_proj(x, ldx, rows, in_dim, w, heads, head_dim, dtype);
   if (rc != MEGA_OK) return rc;
   const int D = heads * head_dim;
@@ -133,6 +134,7 @@ mega_status mega_project_bwd(const void *x, int64_t ldx, int64_t rows, int in_di
                              int head_dim, mega_dtype dtype, const void *grad_feat, int64_t ldgf, void *grad_x,
                              int64_t ldgx, float *grad_w, void *ws, size_t ws_bytes, mega_stream_t stream) {
   clear_error();
+  NvtxRange nvtx_("mega_project_bwd");
   mega_status rc = check_proj(x, ldx, rows, in_dim, w, heads, head_dim, dtype);
   if (rc != MEGA_OK) return rc;
   const int D = heads * head_dim;

@@ -101,24 +101,40 @@ class DistGATLayer:
         L = self.L
         self._pg = [L.grad_w, L.grad_attn_l, L.grad_attn_r]
 
-    def forward(self, timed=None):
-        """timed(name, fn): optional wrapper used by bench.py to time each call."""
+    def forward(self, timed=None, phase=0):
+        """timed(name, fn): optional wrapper used by bench.py to time each call.
+        phase: 0 (both halves), or MEGA_DIST_PHASE_SEND / _RECV for a driver that runs every
+        rank in one process (the LOCAL transport): SEND projects and posts, RECV finishes."""
         L = self.L
         t = timed or (lambda name, fn: fn())
-        t("project_fwd", L.project)
+        if phase != M.MEGA_DIST_PHASE_RECV:
+            t("project_fwd", L.project)
         if self.k == 1:
             t("gat_fwd", lambda: L.attend(True))
         else:   # exchange of [Wh | er] overlapped with block (p, p), remote blocks, merge
             t("gat_fwd", lambda: M.mega_gat_fwd_dist(L.layout, self.rank, self.comm, L.feat, L.attn_l, L.attn_r, L.H,
-                                                     L.F, L.out, L.ctx, L.ws_f, L.slope, M.MEGA_FLAG_ELER_IN_CTX,
-                                                     comm_stream=self.cs))
+                                                     L.F, L.out, L.ctx, L.ws_f, L.slope,
+                                                     M.MEGA_FLAG_ELER_IN_CTX | phase, comm_stream=self.cs))
         return L.out
 
-    def backward(self, grad_out_local, timed=None, split=False):
+    def backward(self, grad_out_local, timed=None, split=False, phase=0):
         """split (k = 1): the source and destination phases as two calls, for per-phase timing
-        (the same work as the single call)."""
+        (the same work as the single call).  phase: as in forward (k > 1; the RECV half runs the
+        projection backward and the parameter all-reduce)."""
         L = self.L
         t = timed or (lambda name, fn: fn())
+        if self.k > 1 and phase:
+            flags = M.MEGA_BWD_LP_ONLY if (L.lp_only and L.grad_feat_lp is not None) else 0
+            t("gat_bwd", lambda: M.mega_gat_bwd_dist(L.layout, self.rank, self.comm, L.feat, L.attn_l, L.attn_r, L.H,
+                                                     L.F, L.out, grad_out_local, L.ctx, L.grad_feat, L.grad_attn_l,
+                                                     L.grad_attn_r, L.ws_b, L.grad_feat_lp, L.slope, flags | phase,
+                                                     comm_stream=self.cs))
+            if phase == M.MEGA_DIST_PHASE_SEND:
+                return None
+            t("project_bwd", L.project_backward)
+            if _world(self.group) > 1:
+                t("allreduce_params", self._allreduce_params)
+            return L.grad_x
         if self.k == 1 and split:
             t("gat_bwd_src", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_SRC))
             t("gat_bwd_dst", lambda: L.attend_backward(grad_out_local, M.MEGA_BWD_PHASE_DST))

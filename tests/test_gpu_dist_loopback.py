@@ -131,3 +131,51 @@ def test_nccl_comm_single_rank(cuda_device):
     inv[perm] = np.arange(n)
     ref = coracle.gat_forward(ip, ix, Wh, a_l, a_r)
     hz.assert_fp32_close(out.cpu().numpy()[inv], ref["out"].reshape(n, -1), "out")
+
+
+@pytest.mark.parametrize("k", [2, 3])
+def test_dist_whole_layer_bf16(cuda_device, k):
+    """dist.DistGATLayer (what bench.py runs on k GPUs) end to end on one GPU through the LOCAL
+    transport: tcgen05 projection of the own rows, halo exchange + split forward, split backward,
+    projection backward; the summed parameter partials stand in for the all-reduce."""
+    from oracle import gat as og
+    from paper_conf_icdcs_dengr24_b200.dist import DistGATLayer
+    cfg = synth.scaled(synth.CONFIGS["products"], 4000, 80000)
+    ip, ix, _ = synth.make_graph(cfg)
+    inp = synth.make_layer_inputs(cfg)
+    x, w, g = synth.bf16_round(inp["x"]), synth.bf16_round(inp["w"]), synth.bf16_round(inp["grad_out"])
+    H, F, D, n = cfg.heads, cfg.head_dim, cfg.dim, cfg.n
+    lay = M.mega_preprocess(ip, ix, num_parts=k)
+    perm = lay.view(0)["perm"].astype(np.int64)
+    bounds = lay.view(0)["bounds"]
+    comms = M.mega_comm_init_local(k)
+    layers = []
+    for p in range(k):
+        lay.bind(p)
+        b0, b1 = int(bounds[p]), int(bounds[p + 1])
+        xt = torch.tensor(x[perm][b0:b1], device="cuda").bfloat16().contiguous()
+        layers.append(DistGATLayer(lay, p, xt, torch.tensor(w, device="cuda").bfloat16(),
+                                   torch.tensor(inp["a_l"], device="cuda"), torch.tensor(inp["a_r"], device="cuda"),
+                                   H, F, in_dim=inp["in_dim"], want_grad_x=True, lp_only=True, comm=comms[p]))
+    gn = torch.tensor(g[perm], device="cuda").bfloat16()
+    for phase in (M.MEGA_DIST_PHASE_SEND, M.MEGA_DIST_PHASE_RECV):
+        for Ld in layers:
+            Ld.forward(phase=phase)
+    for phase in (M.MEGA_DIST_PHASE_SEND, M.MEGA_DIST_PHASE_RECV):
+        for p, Ld in enumerate(layers):
+            Ld.backward(gn[int(bounds[p]):int(bounds[p + 1])], phase=phase)
+    torch.cuda.synchronize()
+    inv = np.empty(n, np.int64)
+    inv[perm] = np.arange(n)
+    Wh = synth.bf16_round(og.project_forward(x, w).astype(np.float32)).astype(np.float64).reshape(n, H, F)
+    f = coracle.gat_forward(ip, ix, Wh, inp["a_l"], inp["a_r"])
+    b = coracle.gat_backward(ip, ix, Wh, inp["a_l"], inp["a_r"], g.reshape(n, H, F), fwd=f)
+    pb = og.project_backward(x, w, b["grad_feat"].reshape(n, D))
+    out = torch.cat([Ld.L.out for Ld in layers]).float().cpu().numpy()[inv]
+    gx = torch.cat([Ld.L.grad_x for Ld in layers]).float().cpu().numpy()[inv]
+    hz.assert_bf16_close(out, f["out"].reshape(n, D), "out")
+    hz.assert_bf16_close(gx, pb["grad_x"], "grad_x")
+    for name, ref in (("grad_w", pb["grad_w"]), ("grad_attn_l", b["grad_attn_l"].reshape(-1)),
+                      ("grad_attn_r", b["grad_attn_r"].reshape(-1))):
+        got = sum(getattr(Ld.L, name) for Ld in layers).cpu().numpy()
+        hz.assert_bf16_close(got, ref, name)
