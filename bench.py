@@ -222,9 +222,10 @@ def build_workload(cfg_name, dtype, order, rank=0, world=1, window=0, seg_edges=
     t_gen = time.time() - t0
     from paper_conf_icdcs_dengr24_b200 import mega as M
     relabel = None
-    if order == "community":   # ablation upper bound: nodes sorted by generator community
-        comm = synth.communities(cfg)
-        relabel = np.lexsort((np.arange(cfg.n), comm))
+    if order in ("community", "comdeg"):   # ablation upper bound: nodes sorted by generator
+        comm = synth.communities(cfg)         # community (comdeg: and by descending in-degree inside it)
+        keys = (np.arange(cfg.n), comm) if order == "community" else (np.arange(cfg.n), -np.diff(indptr), comm)
+        relabel = np.lexsort(keys)
         ip_in, ix_in = synth.relabel(indptr, indices, relabel)
         order, block_rows = "identity", 0
     else:
