@@ -564,6 +564,31 @@ def run_mega(args):
                 "kernels": kernels}
     if kd.get("traffic"):
         roofline["traffic_frac"] = kd["traffic_frac"]
+    # ---- L2 fraction when the gathered table fits in L2: the forward's requested
+    # gather rate (E rows of D*s bytes / its time) against a bare gather of the SAME index stream
+    # (mega_calib_gather over the layout's CSR sources, same table) timed here ----
+    row_bytes = cfg.dim * sb
+    if world == 1 and cfg.n * row_bytes <= l2_bytes and row_bytes in (512, 1024, 2048) and "gat_fwd" in calls:
+        from paper_conf_icdcs_dengr24_b200 import mega as M
+        idx = torch.tensor(wl["layout"].view(0)["src"], dtype=torch.int32, device=dev)
+        table = model.layers[0].L.feat
+        sink = torch.empty(1 << 16, dtype=torch.float32, device=dev)
+        M.mega_calib_gather(table, row_bytes, idx, sink)
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(5):
+            a_, b_ = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a_.record()
+            M.mega_calib_gather(table, row_bytes, idx, sink)
+            b_.record()
+            torch.cuda.synchronize()
+            ts.append(a_.elapsed_time(b_))
+        calib_gbs = idx.numel() * row_bytes / (float(np.median(ts)) * 1e-3) / 1e9
+        fwd_gbs = model.part_edges * row_bytes / (calls["gat_fwd"] * 1e-3) / 1e9
+        roofline["l2"] = {"bound": "l2 gather", "fwd_requested_gbs": fwd_gbs, "calib_gbs": calib_gbs,
+                          "frac": fwd_gbs / calib_gbs, "table_bytes": cfg.n * row_bytes,
+                          "note": "fwd gathered-row bytes (E * D * s, no reuse counted) per second over a bare "
+                                  "gather of the same CSR source stream from the same table (mega_calib_gather)"}
     if ncu:
         roofline["gemm"] = {g: {**ncu[g], "ms_per_call": calls.get("project_fwd" if g == "proj_fwd" else "project_bwd")}
                             for g in ("proj_fwd", "proj_bwd") if g in ncu}

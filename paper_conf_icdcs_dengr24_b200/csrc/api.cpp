@@ -141,7 +141,8 @@ size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
                                       P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
                                       make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size(),
-                                      dl.size(), dr.size(), ds.size(), hs.size(), hr.size(), hp.size()};
+                                      dl.size(), dr.size(), ds.size(), hs.size(), hr.size(), hp.size(),
+                                      P.indptr.size() - 1};
   size_t off = 0;
   for (int i = 0; i < kImageArrays; ++i) {
     offs[i] = off;
@@ -346,10 +347,17 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
     dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
     halo_plan(L, part, P.hsend_idx, P.hsend_off, P.hrecv_idx, P.hrecv_off, P.hpos);
   }
+  // destination-pass row order: descending in-degree (stable), i.e. longest-work-first, so the
+  // static grid stride hands every warp a similar amount of work (the pass gathers nothing)
+  std::vector<int32_t> dorder(P.indptr.size() - 1);
+  for (size_t r = 0; r < dorder.size(); ++r) dorder[r] = (int32_t)r;
+  std::stable_sort(dorder.begin(), dorder.end(), [&](int32_t x, int32_t y) {
+    return P.indptr[x + 1] - P.indptr[x] > P.indptr[y + 1] - P.indptr[y];
+  });
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
       &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos,
-      &P.dl_items, &P.dr_items, &P.d_splits, &P.hsend_idx, &P.hrecv_idx, &P.hpos};
+      &P.dl_items, &P.dr_items, &P.d_splits, &P.hsend_idx, &P.hrecv_idx, &P.hpos, &dorder};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
     if (arrs[i]->empty()) continue;
@@ -397,6 +405,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.hsend_idx = reinterpret_cast<const int32_t *>(base + offs[17]);
   D.hrecv_idx = reinterpret_cast<const int32_t *>(base + offs[18]);
   D.hpos = reinterpret_cast<const int32_t *>(base + offs[19]);
+  D.dorder = dorder.empty() ? nullptr : reinterpret_cast<const int32_t *>(base + offs[20]);
   D.n_hsend = (int64_t)P.hsend_idx.size();
   D.n_hrecv = (int64_t)P.hrecv_idx.size();
   {  // own-source ranges of the CSC work (items and splits are sorted by source id)

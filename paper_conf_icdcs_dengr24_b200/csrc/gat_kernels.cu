@@ -1032,12 +1032,18 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     if (e0 + gl < e1) cp_async_h<HT>(&s_dz[b][w][rb + gl][0], a.dz + (int64_t)(e0 + gl) * H);
     cp_async_commit();
   };
-  int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  // rows are taken in the layout's balanced order (dorder: descending in-degree, so each stride
+  // round holds rows of similar work and no warp is left with the long ones at the end); this pass
+  // gathers nothing, so the order costs no locality
+  const int32_t *ord = a.L.dorder;
+  auto row_at = [&](int64_t q) -> int64_t { return ord ? (int64_t)ord[q] : q; };
+  int64_t pos = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
   int ce0 = 0, ce1 = 0, ne0 = 0, ne1 = 0, buf = 0;
-  if (r < a.L.rows) { ce0 = a.L.indptr[r]; ce1 = a.L.indptr[r + 1]; }
+  if (pos < a.L.rows) { const int64_t r0 = row_at(pos); ce0 = a.L.indptr[r0]; ce1 = a.L.indptr[r0 + 1]; }
   stage_dz(0, ce0, ce1);
-  if (r + stride < a.L.rows) { ne0 = a.L.indptr[r + stride]; ne1 = a.L.indptr[r + stride + 1]; }
-  for (; r < a.L.rows; r += stride) {
+  if (pos + stride < a.L.rows) { const int64_t r1 = row_at(pos + stride); ne0 = a.L.indptr[r1]; ne1 = a.L.indptr[r1 + 1]; }
+  for (; pos < a.L.rows; pos += stride) {
+    const int64_t r = row_at(pos);
     const int64_t grow = a.L.row_begin + r;
     // row-local operands first: they do not depend on del, so their latency
     // overlaps the dz gather below
@@ -1054,10 +1060,14 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     float derr[HT];
     load_h<HT>(a.der + grow * H, H, derr);
     const int e0 = ce0, e1 = ce1;
-    if (r + stride < a.L.rows) stage_dz(buf ^ 1, ne0, ne1);
+    if (pos + stride < a.L.rows) stage_dz(buf ^ 1, ne0, ne1);
     else cp_async_commit();
     ce0 = ne0; ce1 = ne1;
-    if (r + 2 * stride < a.L.rows) { ne0 = a.L.indptr[r + 2 * stride]; ne1 = a.L.indptr[r + 2 * stride + 1]; }
+    if (pos + 2 * stride < a.L.rows) {
+      const int64_t r2 = row_at(pos + 2 * stride);
+      ne0 = a.L.indptr[r2];
+      ne1 = a.L.indptr[r2 + 1];
+    }
     cp_async_wait<1>();  // this row's staged dz
     float dp[HT];
 #pragma unroll

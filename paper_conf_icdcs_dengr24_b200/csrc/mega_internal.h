@@ -39,6 +39,7 @@ struct DevPart {
   const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
   const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
   const int32_t *cpos = nullptr;      // [E_p] CSR position of each CSC edge (dz is stored in CSR order)
+  const int32_t *dorder = nullptr;   // [rows] local rows by descending in-degree (destination pass order)
   const int4 *ftiles = nullptr;      // (e_begin, e_end, slot, 0): runs of whole CSR rows / one split segment
   const int4 *btiles = nullptr;      // the same over the CSC (sources)
   int32_t n_ftiles = 0, n_btiles = 0;
@@ -98,7 +99,7 @@ namespace mega {
 // preprocess.cpp
 mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, mega_layout *L);
 // image layout shared by device_bytes / bind
-constexpr int kImageArrays = 20;
+constexpr int kImageArrays = 21;
 // dist items of part p (k > 1): see DevPart; S = the layout's segment size
 void dist_items(const mega_layout *L, int part, std::vector<int32_t> &local, std::vector<int32_t> &remote,
                 std::vector<int32_t> &splits, int32_t &nslots);

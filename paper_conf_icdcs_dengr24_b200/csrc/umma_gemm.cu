@@ -129,6 +129,15 @@ __device__ __forceinline__ void tmem_ld32(uint32_t taddr, uint32_t (&r)[32]) {
       : "r"(taddr));
   asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
 }
+// packed fp32x2 FMA (sm_100 FFMA2): d{0,1} += a{0,1} * c{0,1}
+__device__ __forceinline__ void ffma2(float &d0, float &d1, float a0, float a1, float c0, float c1) {
+  unsigned long long D, A, C;
+  asm("mov.b64 %0, {%1, %2};" : "=l"(A) : "f"(a0), "f"(a1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(C) : "f"(c0), "f"(c1));
+  asm("mov.b64 %0, {%1, %2};" : "=l"(D) : "f"(d0), "f"(d1));
+  asm("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(D) : "l"(A), "l"(C));
+  asm("mov.b64 {%0, %1}, %2;" : "=f"(d0), "=f"(d1) : "l"(D));
+}
 __device__ __forceinline__ uint32_t bf2(float a, float b) {
   __nv_bfloat162 t = __floats2bfloat162_rn(a, b);
   return *reinterpret_cast<uint32_t *>(&t);
@@ -470,7 +479,7 @@ __global__ void __launch_bounds__(PTiles<BN, EPI>::THREADS, 1)
       const uint32_t taddr = tmem + (uint32_t)(acc * TL::ACC_COLS) + ((uint32_t)(ew * 32) << 16);
       const int64_t grow = m0 + row;
       const bool live = grow < g.M;
-      float el_acc = 0.f, er_acc = 0.f;
+      float el0 = 0.f, el1 = 0.f, er0 = 0.f, er1 = 0.f;   // even / odd column partial sums (FFMA2)
 #pragma unroll 1
       for (int c64 = ewg * CW; c64 < (ewg + 1) * CW; c64 += 64, ++chunk) {
         const int b = (int)(chunk & 1);
@@ -497,24 +506,26 @@ __global__ void __launch_bounds__(PTiles<BN, EPI>::THREADS, 1)
 #pragma unroll
             for (int sgm = 0; sgm < 32 / FH; ++sgm) {
 #pragma unroll
-              for (int q = 0; q < FH; q += 2) {
-                const uint32_t w2 = p[(sgm * FH + q) / 2];
-                const float x0 = __uint_as_float(w2 << 16), x1 = __uint_as_float(w2 & 0xffff0000u);
+              for (int q = 0; q < FH; q += 4) {   // 4 columns: one 16-byte broadcast load of a_l and a_r each
+                const uint32_t wa = p[(sgm * FH + q) / 2], wb = p[(sgm * FH + q) / 2 + 1];
+                const float x0 = __uint_as_float(wa << 16), x1 = __uint_as_float(wa & 0xffff0000u);
+                const float x2 = __uint_as_float(wb << 16), x3 = __uint_as_float(wb & 0xffff0000u);
                 const int c = n0 + c0 + sgm * FH + q;
-                el_acc = fmaf(s_al[c], x0, el_acc);
-                el_acc = fmaf(s_al[c + 1], x1, el_acc);
-                er_acc = fmaf(s_ar[c], x0, er_acc);
-                er_acc = fmaf(s_ar[c + 1], x1, er_acc);
+                const float4 al4 = *reinterpret_cast<const float4 *>(s_al + c);
+                const float4 ar4 = *reinterpret_cast<const float4 *>(s_ar + c);
+                ffma2(el0, el1, x0, x1, al4.x, al4.y);
+                ffma2(el0, el1, x2, x3, al4.z, al4.w);
+                ffma2(er0, er1, x0, x1, ar4.x, ar4.y);
+                ffma2(er0, er1, x2, x3, ar4.z, ar4.w);
               }
               const int cend = c0 + (sgm + 1) * FH;
               if (cend % g.F == 0) {
                 const int h = (n0 + cend) / g.F - 1;
                 if (live) {
-                  g.el[(g.ctx_row0 + grow) * g.H + h] = el_acc;
-                  g.er[(g.ctx_row0 + grow) * g.H + h] = er_acc;
+                  g.el[(g.ctx_row0 + grow) * g.H + h] = el0 + el1;
+                  g.er[(g.ctx_row0 + grow) * g.H + h] = er0 + er1;
                 }
-                el_acc = 0.f;
-                er_acc = 0.f;
+                el0 = el1 = er0 = er1 = 0.f;
               }
             }
           }

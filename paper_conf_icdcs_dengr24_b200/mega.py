@@ -120,6 +120,7 @@ def lib():
                                       P, I64, P, P, _c.c_size_t, P, P]),
             "mega_gat_bwd_dist": (S, [P, _c.c_int32, P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32,
                                       P, I64, P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P, P]),
+            "mega_calib_gather": (S, [P, I64, _c.c_int, P, I64, P, I64, P]),
             "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P]),
             "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, P]),
             "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P, I64, P, P, P, I64,
@@ -311,6 +312,12 @@ def mega_project_bwd(x, w, heads, head_dim, grad_feat, grad_w, grad_x=None, in_d
                                   dt, _ptr(grad_feat), grad_feat.stride(0), _ptr(grad_x),
                                   grad_x.stride(0) if grad_x is not None else 0, _ptr(grad_w), _ptr(ws),
                                   0 if ws is None else ws.numel() * ws.element_size(), _stream(stream)))
+
+
+def mega_calib_gather(table, row_bytes, idx, sink, stream=None):
+    """Measurement helper: gather rows idx of `table` (device, [rows][row_bytes])."""
+    _check(lib().mega_calib_gather(_ptr(table), table.numel() * table.element_size() // row_bytes, row_bytes,
+                                   _ptr(idx), idx.numel(), _ptr(sink), sink.numel(), _stream(stream)))
 
 
 # ---------------- k GPUs (include/mega.h "k GPUs: destination partitions") ----------------
