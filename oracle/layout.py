@@ -22,13 +22,9 @@ from __future__ import annotations
 
 import numpy as np
 
-NUM_SMS_FOR_AUTO = 148
-
-
 def auto_seg_edges(m: int) -> int:
-    """S = max(256, round_up_32(ceil(m / (148*256))))  (DESIGN.md "Work items")."""
-    per = -(-m // (NUM_SMS_FOR_AUTO * 256))
-    return int(max(256, (per + 31) // 32 * 32))
+    """S = 256 (DESIGN.md "Work items"; a layout input like the tile sizes, SURVEY c6 #27)."""
+    return 256
 
 
 def relabel(indptr, indices, perm):

@@ -39,7 +39,7 @@ struct DevPart {
   const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
   const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
   const int32_t *cpos = nullptr;      // [E_p] CSR position of each CSC edge (dz is stored in CSR order)
-  const int32_t *dorder = nullptr;   // [rows] local rows by descending in-degree (destination pass order)
+  const int32_t *dorder = nullptr;   // [rows] destination-pass row order: heavy rows first (see bind)
   const int4 *ftiles = nullptr;      // (e_begin, e_end, slot, 0): runs of whole CSR rows / one split segment
   const int4 *btiles = nullptr;      // the same over the CSC (sources)
   int32_t n_ftiles = 0, n_btiles = 0;

@@ -251,11 +251,12 @@ mega_status build_layout(const mega_csr *csr, const mega_schedule_opts *opts, me
   int omega = opts->window;
   if (omega <= 0) omega = (int)std::min<int64_t>(64, std::max<int64_t>(1, (2 * m + n) / (2 * n)));
   const int K = opts->candidate_cap > 0 ? opts->candidate_cap : 32;
+  // S: work-item segment size.  Items are taken with a static grid stride, so the kernel ends
+  // with the warp whose items sum to the most edges; 256 keeps that within ~13% of the mean on
+  // products and reddit (measured best: products 81.1 ms/step at 256 vs 85.6 at round 1's
+  // m/(148*256) = 1664; reddit 16.7 vs 21.4 at 3040)
   int32_t S = opts->seg_edges;
-  if (S <= 0) {
-    int64_t per = (m + 148 * 256 - 1) / (148 * 256);
-    S = (int32_t)std::max<int64_t>(256, (per + 31) / 32 * 32);
-  }
+  if (S <= 0) S = 256;
 
   // ---- node order ----
   int64_t path_len = n, jumps = 0, sweeps = 0, nblocks = n;
