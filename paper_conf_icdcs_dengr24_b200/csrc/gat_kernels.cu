@@ -1038,12 +1038,14 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
   const int32_t *ord = a.L.dorder;
   auto row_at = [&](int64_t q) -> int64_t { return ord ? (int64_t)ord[q] : q; };
   int64_t pos = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  // row ids and their indptr pairs are software-pipelined one and two rows ahead (cr, nr)
   int ce0 = 0, ce1 = 0, ne0 = 0, ne1 = 0, buf = 0;
-  if (pos < a.L.rows) { const int64_t r0 = row_at(pos); ce0 = a.L.indptr[r0]; ce1 = a.L.indptr[r0 + 1]; }
+  int64_t cr = 0, nr = 0;
+  if (pos < a.L.rows) { cr = row_at(pos); ce0 = a.L.indptr[cr]; ce1 = a.L.indptr[cr + 1]; }
   stage_dz(0, ce0, ce1);
-  if (pos + stride < a.L.rows) { const int64_t r1 = row_at(pos + stride); ne0 = a.L.indptr[r1]; ne1 = a.L.indptr[r1 + 1]; }
+  if (pos + stride < a.L.rows) { nr = row_at(pos + stride); ne0 = a.L.indptr[nr]; ne1 = a.L.indptr[nr + 1]; }
   for (; pos < a.L.rows; pos += stride) {
-    const int64_t r = row_at(pos);
+    const int64_t r = cr;
     const int64_t grow = a.L.row_begin + r;
     // row-local operands first: they do not depend on del, so their latency
     // overlaps the dz gather below
@@ -1062,11 +1064,11 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     const int e0 = ce0, e1 = ce1;
     if (pos + stride < a.L.rows) stage_dz(buf ^ 1, ne0, ne1);
     else cp_async_commit();
-    ce0 = ne0; ce1 = ne1;
+    ce0 = ne0; ce1 = ne1; cr = nr;
     if (pos + 2 * stride < a.L.rows) {
-      const int64_t r2 = row_at(pos + 2 * stride);
-      ne0 = a.L.indptr[r2];
-      ne1 = a.L.indptr[r2 + 1];
+      nr = row_at(pos + 2 * stride);
+      ne0 = a.L.indptr[nr];
+      ne1 = a.L.indptr[nr + 1];
     }
     cp_async_wait<1>();  // this row's staged dz
     float dp[HT];
