@@ -347,16 +347,18 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
     dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
     halo_plan(L, part, P.hsend_idx, P.hsend_off, P.hrecv_idx, P.hrecv_off, P.hpos);
   }
-  // destination-pass row order: the heavy rows (in-degree > 2x the part's mean) first, longest
-  // first, then every other row in layout order.  The pass gathers nothing, but it streams each
-  // row's dz slice; the heavy rows are what unbalances the static grid stride (a reddit hub row
-  // carries ~40% of a warp's share), and leaving the other ~93% in order keeps the streams
-  // sequential (measured: a full degree sort cost products 18% on this pass, saved reddit 36%).
+  // destination-pass row order.  The pass gathers nothing but streams each row's dz slice (16 B
+  // per edge and head group) and its row operands.  When rows are long (mean in-degree >= 64) the
+  // heavy rows (> 2x the mean) unbalance the static grid stride (a reddit hub carries ~40% of a
+  // warp's share): they go first, longest first, the rest in layout order (reddit 1.40 -> 0.91
+  // ms/step).  With short rows (products, mean 25) any reordering cost more than it balanced
+  // (6.8 -> 7.8 ms/step measured), so the layout order is kept (no order array).
   std::vector<int32_t> dorder;
   {
-    const int64_t rows = (int64_t)P.indptr.size() - 1;
+    int64_t rows = (int64_t)P.indptr.size() - 1;
     const double mean = rows > 0 ? (double)P.indptr[rows] / (double)rows : 0.0;
     std::vector<int32_t> heavy;
+    if (mean < 64.0) rows = 0;   // short rows: keep the layout order
     dorder.reserve(rows);
     for (int64_t r = 0; r < rows; ++r)
       if (P.indptr[r + 1] - P.indptr[r] > 2.0 * mean) heavy.push_back((int32_t)r);

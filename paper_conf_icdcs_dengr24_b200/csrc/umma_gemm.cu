@@ -93,6 +93,12 @@ __device__ __forceinline__ void tma_store_2d(const CUtensorMap *map, uint32_t sr
                "r"(x), "r"(y), "r"(src)
                : "memory");
 }
+// TMA prefetch of a 2-D box into L2 (no shared memory, no completion tracking)
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap *map, int32_t x, int32_t y) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(reinterpret_cast<uint64_t>(map)),
+               "r"(x), "r"(y)
+               : "memory");
+}
 __device__ __forceinline__ void prefetch_tmap(const CUtensorMap *map) {
   asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
 }
@@ -359,7 +365,7 @@ template <int BN, int EPI> struct PTiles {
   static constexpr int STAGES = (216 * 1024 - OUT) / STAGE > 8 ? 8 : (216 * 1024 - OUT) / STAGE;
   static constexpr int ACC_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr int TMEM_COLS = 2 * ACC_COLS;
-  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + OUT + 512 + 2 * 1024 * 4;
+  static constexpr size_t SMEM = 1024 + (size_t)STAGES * STAGE + OUT + 512;   // + 8 KB static (a_l, a_r)
   static constexpr int THREADS = 64 + 128 * EPI;
 };
 
@@ -379,8 +385,8 @@ __global__ void __launch_bounds__(PTiles<BN, EPI>::THREADS, 1)
   uint64_t *bars = reinterpret_cast<uint64_t *>(outb + TL::OUT);
   // bars: full[S], empty[S], tfull[2], tempty[2]
   uint32_t *tslot = reinterpret_cast<uint32_t *>(bars + 2 * STAGES + 4);
-  float *s_al = reinterpret_cast<float *>(outb + TL::OUT + 512);
-  float *s_ar = s_al + 1024;
+  __shared__ __align__(16) float s_alr[2][1024];   // a_l, a_r (static: the compiler knows they are shared)
+  float *s_al = s_alr[0], *s_ar = s_alr[1];
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t full0 = smem_u32(bars), empty0 = smem_u32(bars + STAGES);
   const uint32_t tfull0 = smem_u32(bars + 2 * STAGES), tempty0 = smem_u32(bars + 2 * STAGES + 2);
@@ -417,10 +423,22 @@ __global__ void __launch_bounds__(PTiles<BN, EPI>::THREADS, 1)
 
   if (warp == 0) {
     if (lane == 0) {   // ---- TMA producer: k-blocks of every tile of this CTA, through the ring ----
+      // The A operand (X / dWh rows) streams from HBM: its k-blocks are also prefetched into L2
+      // PF k-blocks ahead (across tile boundaries), so a ring slot waits on an L2 hit, not on DRAM
+      // latency (the ring is only STAGES deep; B is small and L2-resident anyway).
+      constexpr int PF = 6;
+      int64_t pt = blockIdx.x;
+      int pi = 0;
+      for (int q = 0; q < PF; ++q) {   // warm-up: the first PF k-blocks
+        if (pt < ntile_total) tma_prefetch_2d(&tmA, pi * BK, (int32_t)((pt / g.ntiles) * BM));
+        if (++pi == nkb) { pi = 0; pt += gridDim.x; }
+      }
       int64_t kc = 0;
       for (int64_t t = blockIdx.x; t < ntile_total; t += gridDim.x) {
         const int32_t m0 = (int32_t)((t / g.ntiles) * BM), n0 = (int32_t)((t % g.ntiles) * BN);
         for (int i = 0; i < nkb; ++i, ++kc) {
+          if (pt < ntile_total) tma_prefetch_2d(&tmA, pi * BK, (int32_t)((pt / g.ntiles) * BM));
+          if (++pi == nkb) { pi = 0; pt += gridDim.x; }
           const int s2 = (int)(kc % STAGES);
           mbar_wait(empty0 + 8 * s2, (uint32_t)((kc / STAGES) & 1) ^ 1u);
           const uint32_t full = full0 + 8 * s2;
