@@ -153,7 +153,8 @@ def design_bytes(kernel, rows, N, E, H, D, sb):
 
 # kernel-name prefixes (ncu launch list) of each launch group
 GROUPS = {"KB2": ("gat_fwd",), "KB3+KB4": ("dlt_kernel", "gat_bwd_src"), "KB5": ("gat_bwd_dst", "param_reduce"),
-          "proj_fwd": ("umma_gemm_kernel<0",), "proj_bwd": ("umma_gemm_kernel<1", "umma_gemm_kernel<2", "dw_reduce")}
+          "proj_fwd": ("umma_gemm_persistent<0",),
+          "proj_bwd": ("umma_gemm_persistent<1", "umma_gemm_kernel<2", "dw_reduce")}
 
 
 def ncu_launch_summary(path):

@@ -221,6 +221,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
   const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
+  const uint64_t pol_st = a.st_hint ? policy_first() : policy_normal();
   const float *sp_v[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
@@ -382,7 +383,7 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
           float y[EPV];
 #pragma unroll
           for (int k = 0; k < EPV; ++k) y[k] = acc[v][k] * inv;
-          st16(orow + v * G * EPV, pack(y, T()));
+          st16_pol(orow + v * G * EPV, pack(y, T()), pol_st);
         }
         for (int h = gl; h < H; h += G) {
           const float Lh = sel<HT>(lt, h);
@@ -785,6 +786,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
   const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
   const int hot_cls = a.hot_cls;
   const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
+  const uint64_t pol_st = a.st_hint ? policy_first() : policy_normal();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
@@ -820,7 +822,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       const T *rp = feat + j * a.ldf + gl * EPV;
 #pragma unroll
       for (int v = 0; v < V; ++v) {
-        unpack(ldg16(rp + v * G * EPV), whf[v], T());
+        unpack(ldg16_pol(rp + v * G * EPV, pol_st), whf[v], T());
         derv[v] = 0.f;
 #pragma unroll
         for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
@@ -917,7 +919,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       if (valid) {
         float *dzp = a.dz + (int64_t)cp_c * H;  // CSR order
         if constexpr (HT == 4) {
-          reinterpret_cast<float4 *>(dzp)[0] = make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]);
+          st16f_pol(dzp, make_float4(s_z[w][lane][0], s_z[w][lane][1], s_z[w][lane][2], s_z[w][lane][3]), pol_st);
         } else {
           for (int h = 0; h < H; ++h) dzp[h] = s_z[w][lane][h];
         }
@@ -950,7 +952,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
           y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          st16f_pol(orow + v * G * EPV + k, make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]), pol_st);
         }
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
@@ -1297,6 +1299,14 @@ int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
 
 // L2 policy of gathered rows (ablation knob MEGA_L2_POLICY): 0 = hot rows evict_last, the rest
 // evict_first (default); 1 = all evict_normal; 2 = hot evict_last, rest evict_normal
+int st_hint_mode() {   // MEGA_ST_HINT=0 turns the evict_first hints on streamed results off (ablation)
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_ST_HINT");
+    v = e ? std::atoi(e) : 1;
+  }
+  return v;
+}
 int l2_policy_mode() {
   static int v = -1;
   if (v < 0) {
@@ -1566,6 +1576,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.st_hint = st_hint_mode();
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1616,6 +1627,7 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.st_hint = st_hint_mode();
   cudaStream_t st = (cudaStream_t)stream;
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }
@@ -1745,6 +1757,7 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.st_hint = st_hint_mode();
   auto pass = [&](const int4 *items, int32_t nitems, const int32_t *splits, int32_t nsplits) {
     kern::FwdArgs b = a;
     b.L.fwd_items = items; b.L.n_fwd_items = nitems;
@@ -1848,6 +1861,7 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
+  a.st_hint = st_hint_mode();
   cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
   // source-phase launches over a range of CSC items [i0, i1) and splits [s0, s1)
   auto src_range = [&](int32_t i0, int32_t i1, int32_t s0, int32_t s1, bool dlt) {

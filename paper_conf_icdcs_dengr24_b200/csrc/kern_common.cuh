@@ -57,6 +57,16 @@ __device__ __forceinline__ int ld_stream(const int32_t *p, uint64_t pol) {
   return v;
 }
 __device__ __forceinline__ void st16(void *p, uint4 v) { *reinterpret_cast<uint4 *>(p) = v; }
+// streaming 16-byte stores with an L2 policy (evict_first: results written once must not push the
+// gathered rows out of L2)
+__device__ __forceinline__ void st16_pol(void *p, uint4 v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void st16f_pol(void *p, float4 v, uint64_t pol) {
+  st16_pol(p, make_uint4(__float_as_uint(v.x), __float_as_uint(v.y), __float_as_uint(v.z), __float_as_uint(v.w)), pol);
+}
 
 __device__ __forceinline__ void unpack(const uint4 &r, float (&x)[4], float) {
   x[0] = __uint_as_float(r.x); x[1] = __uint_as_float(r.y);
@@ -289,6 +299,7 @@ struct FwdArgs {
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
+  int st_hint;  // 1: streamed results (out rows) stored with L2 evict_first (MEGA_ST_HINT)
   int pol_mode; // MEGA_L2_POLICY
 };
 
@@ -315,6 +326,7 @@ struct BwdArgs {
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
+  int st_hint;  // 1: streamed results (dWh, dz, der) and the source's own Wh row use L2 evict_first
   int pol_mode; // MEGA_L2_POLICY
 };
 
