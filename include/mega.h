@@ -373,32 +373,36 @@ mega_status mega_gat_bwd_dist(const mega_layout *layout, int32_t part, mega_comm
 /* NEXT-3: Graph Transformer edge attention, the paper's
  * headline model (Table I; DESIGN.md R-gt), over the same layout:
  *   s_e = Q_i.K_j / sqrt(head_dim) per head, alpha = softmax over In(i),
- *   out_i = sum_e alpha_e V_j.   fp32 only in this first cut.
- *   q, k, v   device fp32 [num_nodes][ld] (new order; heads concatenated)
- *   out       device fp32 [rows_p][ldo] (written; 0 for rows without in-edges)
+ *   out_i = sum_e alpha_e V_j.
+ *   dtype  MEGA_F32: q/k/v/out fp32 (first cut: one warp per row and head);
+ *          MEGA_BF16: q/k/v/out bf16 with fp32 accumulation (row-vector kernels
+ *          over the layout's work items, split rows merged in fixed order;
+ *          heads 1/2/4/8, head_dim a multiple of 8 with head_dim/8 a power of two,
+ *          heads*head_dim/8 in {8, 16, 32, 64, 128}).
+ *   q, k, v   device [num_nodes][ld] (new order; heads concatenated)
+ *   out       device [rows_p][ldo] (written; 0 for rows without in-edges)
  *   lse       device fp32 [rows_p][heads] (written; -inf without in-edges)
- * Supported: heads <= 8, head_dim <= 128.  Errors: INVALID_ARGUMENT,
- * UNSUPPORTED, STATE (part not bound here), CUDA. */
-mega_status mega_gt_fwd(const mega_layout *layout, int32_t part, const float *q, const float *k, const float *v,
-                        int64_t ld, int heads, int head_dim, float *out, int64_t ldo, float *lse,
-                        mega_stream_t stream);
-
-/* Workspace (bytes, device) of mega_gt_bwd: (alpha, ds) per edge and head. */
-mega_status mega_gt_workspace_bytes(const mega_layout *layout, int32_t part, int heads, size_t *bwd_ws);
+ *   ws        device workspace >= mega_gt_workspace_bytes (unused by MEGA_F32 fwd).
+ * Errors: INVALID_ARGUMENT, UNSUPPORTED, STATE (part not bound here), CUDA. */
+mega_status mega_gt_workspace_bytes(const mega_layout *layout, int32_t part, int heads, int head_dim,
+                                    mega_dtype dtype, size_t *ws_bytes);
+mega_status mega_gt_fwd(const mega_layout *layout, int32_t part, const void *q, const void *k, const void *v,
+                        int64_t ld, int heads, int head_dim, mega_dtype dtype, void *out, int64_t ldo, float *lse,
+                        void *ws, size_t ws_bytes, mega_stream_t stream);
 
 /* Backward of mega_gt_fwd, no atomics: destination pass over the CSR
- * (dQ_i = sum ds_e K_j / sqrt(F), ds_e = alpha_e (g_i.V_j - g_i.out_i)),
- * then source pass over the CSC (dK_j = sum ds_e Q_i / sqrt(F),
- * dV_j = sum alpha_e g_i).
- *   grad_out  device fp32 [rows_p][ldg]
+ * (dQ_i = sum ds_e K_j / sqrt(F), ds_e = alpha_e (g_i.V_j - g_i.out_i), with
+ * out the stored forward output), then source pass over the CSC
+ * (dK_j = sum ds_e Q_i / sqrt(F), dV_j = sum alpha_e g_i).
+ *   grad_out  device [rows_p][ldg] (dtype)
  *   grad_q    device fp32 [rows_p][ldgr] (written, this part's rows)
  *   grad_k/v  device fp32 [num_nodes][ldgr] (written; this part's partial
  *             when k > 1 — the caller sums over parts)
  * Errors as mega_gt_fwd, plus OUT_OF_MEMORY (workspace too small). */
-mega_status mega_gt_bwd(const mega_layout *layout, int32_t part, const float *q, const float *k, const float *v,
-                        int64_t ld, int heads, int head_dim, const float *out, int64_t ldo, const float *lse,
-                        const float *grad_out, int64_t ldg, float *grad_q, float *grad_k, float *grad_v,
-                        int64_t ldgr, void *ws, size_t ws_bytes, mega_stream_t stream);
+mega_status mega_gt_bwd(const mega_layout *layout, int32_t part, const void *q, const void *k, const void *v,
+                        int64_t ld, int heads, int head_dim, mega_dtype dtype, const void *out, int64_t ldo,
+                        const float *lse, const void *grad_out, int64_t ldg, float *grad_q, float *grad_k,
+                        float *grad_v, int64_t ldgr, void *ws, size_t ws_bytes, mega_stream_t stream);
 
 /* Measurement helper (SURVEY §8(d)-d2 calibration; not part of the GAT path):
  * gathers the rows idx[0..n) of a device table [rows][row_bytes] (row_bytes in

@@ -249,33 +249,56 @@ int grid_for(int64_t warps, int sms) {
   } while (0)
 
 }  // namespace gt
+// gt_bf16.cu
+size_t gtb_workspace_bytes(const Part &P, int H, int D);
+mega_status gtb_run(const mega_layout *L, int32_t part, bool bwd, const void *q, const void *k, const void *v,
+                    int64_t ld, int heads, int head_dim, void *out, int64_t ldo, float *lse, const void *grad_out,
+                    int64_t ldg, float *gq, float *gk, float *gv, int64_t ldgr, void *ws, size_t ws_bytes,
+                    cudaStream_t st, int sms);
 }  // namespace mega
 
 using namespace mega;
 
 extern "C" {
 
-mega_status mega_gt_workspace_bytes(const mega_layout *L, int32_t part, int heads, size_t *bwd_ws) {
+mega_status mega_gt_workspace_bytes(const mega_layout *L, int32_t part, int heads, int head_dim, mega_dtype dtype,
+                                    size_t *ws_bytes) {
   clear_error();
-  if (!L || !bwd_ws) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  if (!L || !ws_bytes) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
   if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
-  if (heads < 1 || heads > 8) return fail(MEGA_ERR_UNSUPPORTED, "heads in [1, 8]");
+  if (heads < 1 || heads > 8 || head_dim < 1) return fail(MEGA_ERR_UNSUPPORTED, "heads in [1, 8]");
+  if (dtype != MEGA_F32 && dtype != MEGA_BF16) return fail(MEGA_ERR_INVALID_ARGUMENT, "bad dtype");
   const Part &P = L->parts[part];
+  if (dtype == MEGA_BF16) {
+    *ws_bytes = gtb_workspace_bytes(P, heads, heads * head_dim);
+    return MEGA_OK;
+  }
   const size_t e = std::max<size_t>({(size_t)1, P.src.size(), (size_t)P.dev.edges});
-  *bwd_ws = 2 * ((e * heads * 4 + 255) / 256 * 256);
+  *ws_bytes = 2 * ((e * heads * 4 + 255) / 256 * 256);
   return MEGA_OK;
 }
 
-mega_status mega_gt_fwd(const mega_layout *L, int32_t part, const float *q, const float *k, const float *v, int64_t ld,
-                        int heads, int head_dim, float *out, int64_t ldo, float *lse, mega_stream_t stream) {
+mega_status mega_gt_fwd(const mega_layout *L, int32_t part, const void *q_, const void *k_, const void *v_, int64_t ld,
+                        int heads, int head_dim, mega_dtype dtype, void *out_, int64_t ldo, float *lse, void *ws,
+                        size_t ws_bytes, mega_stream_t stream) {
   clear_error();
   NvtxRange nvtx_("mega_gt_fwd");
   int sms = 0;
   mega_status rc = gt::check(L, part, heads, head_dim, sms);
   if (rc != MEGA_OK) return rc;
-  if (!q || !k || !v || !out || !lse) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  if (!q_ || !k_ || !v_ || !out_ || !lse) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
   const int64_t D = (int64_t)heads * head_dim;
   if (ld < D || ldo < D) return fail(MEGA_ERR_INVALID_ARGUMENT, "ld/ldo must be >= heads*head_dim");
+  if (dtype == MEGA_BF16) {
+    if (heads & (heads - 1)) return fail(MEGA_ERR_UNSUPPORTED, "bf16 GT: heads must be 1, 2, 4 or 8");
+    if (!ws || ld % 8 || ldo % 8) return fail(MEGA_ERR_INVALID_ARGUMENT, "bf16 GT: workspace, 16-byte rows");
+    return gtb_run(L, part, false, q_, k_, v_, ld, heads, head_dim, out_, ldo, lse, nullptr, 0, nullptr, nullptr,
+                   nullptr, 0, ws, ws_bytes, (cudaStream_t)stream, sms);
+  }
+  if (dtype != MEGA_F32) return fail(MEGA_ERR_INVALID_ARGUMENT, "bad dtype");
+  const float *q = static_cast<const float *>(q_), *k = static_cast<const float *>(k_),
+              *v = static_cast<const float *>(v_);
+  float *out = static_cast<float *>(out_);
   gt::Args a{};
   a.L = L->parts[part].dev;
   a.q = q; a.k = k; a.v = v; a.ld = ld;
@@ -286,21 +309,32 @@ mega_status mega_gt_fwd(const mega_layout *L, int32_t part, const float *q, cons
   return MEGA_OK;
 }
 
-mega_status mega_gt_bwd(const mega_layout *L, int32_t part, const float *q, const float *k, const float *v, int64_t ld,
-                        int heads, int head_dim, const float *out, int64_t ldo, const float *lse,
-                        const float *grad_out, int64_t ldg, float *grad_q, float *grad_k, float *grad_v, int64_t ldgr,
+mega_status mega_gt_bwd(const mega_layout *L, int32_t part, const void *q_, const void *k_, const void *v_, int64_t ld,
+                        int heads, int head_dim, mega_dtype dtype, const void *out_, int64_t ldo, const float *lse,
+                        const void *grad_out_, int64_t ldg, float *grad_q, float *grad_k, float *grad_v, int64_t ldgr,
                         void *ws, size_t ws_bytes, mega_stream_t stream) {
   clear_error();
   NvtxRange nvtx_("mega_gt_bwd");
   int sms = 0;
   mega_status rc = gt::check(L, part, heads, head_dim, sms);
   if (rc != MEGA_OK) return rc;
-  if (!q || !k || !v || !out || !lse || !grad_out || !grad_q || !grad_k || !grad_v || !ws)
+  if (!q_ || !k_ || !v_ || !out_ || !lse || !grad_out_ || !grad_q || !grad_k || !grad_v || !ws)
     return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
   const int64_t D = (int64_t)heads * head_dim;
   if (ld < D || ldo < D || ldg < D || ldgr < D) return fail(MEGA_ERR_INVALID_ARGUMENT, "leading dims must be >= D");
+  if (dtype == MEGA_BF16) {
+    if (heads & (heads - 1)) return fail(MEGA_ERR_UNSUPPORTED, "bf16 GT: heads must be 1, 2, 4 or 8");
+    if (ld % 8 || ldo % 8 || ldg % 8 || ldgr % 4) return fail(MEGA_ERR_INVALID_ARGUMENT, "bf16 GT: 16-byte rows");
+    return gtb_run(L, part, true, q_, k_, v_, ld, heads, head_dim, const_cast<void *>(out_), ldo,
+                   const_cast<float *>(lse), grad_out_, ldg, grad_q, grad_k, grad_v, ldgr, ws, ws_bytes,
+                   (cudaStream_t)stream, sms);
+  }
+  if (dtype != MEGA_F32) return fail(MEGA_ERR_INVALID_ARGUMENT, "bad dtype");
+  const float *q = static_cast<const float *>(q_), *k = static_cast<const float *>(k_),
+              *v = static_cast<const float *>(v_), *out = static_cast<const float *>(out_),
+              *grad_out = static_cast<const float *>(grad_out_);
   size_t need = 0;
-  mega_gt_workspace_bytes(L, part, heads, &need);
+  mega_gt_workspace_bytes(L, part, heads, head_dim, MEGA_F32, &need);
   if (ws_bytes < need) return fail(MEGA_ERR_OUT_OF_MEMORY, "GT bwd workspace too small");
   gt::Args a{};
   a.L = L->parts[part].dev;

@@ -276,9 +276,11 @@ __global__ void __launch_bounds__(THREADS) umma_gemm_kernel(const __grid_constan
       else
 #pragma unroll
         for (int q = 0; q < 32; ++q) r[q] = 0u;
+      if (grow < g.M) {   // slab mode: M = mpad (every row); direct mode: M = in_dim rows of grad_w
 #pragma unroll
-      for (int q = 0; q < 8; ++q)
-        *reinterpret_cast<uint4 *>(dst + c0 + 4 * q) = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+        for (int q = 0; q < 8; ++q)
+          *reinterpret_cast<uint4 *>(dst + c0 + 4 * q) = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+      }
     }
   } else {
     // bf16 tile -> shared memory (the operand ring is free once the accumulator is complete),
@@ -748,10 +750,13 @@ void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, s
   const int64_t kbt = (rows + BK - 1) / BK;
   int64_t s = (2 * (int64_t)sm_count() + mt * nt - 1) / (mt * nt);
   s = std::max<int64_t>(1, std::min<int64_t>(s, kbt));
+  // short reductions (the paper's batches of small graphs: ~1-6K rows) run unsplit, writing grad_w
+  // directly: one launch instead of a split GEMM plus its reduction, which is what such steps pay for
+  if (kbt <= 128) s = 1;
   const int64_t per = (kbt + s - 1) / s;
   splits = (int)((kbt + per - 1) / per);   // every split non-empty
   mpad = mt * BM;
-  bytes = (size_t)splits * (size_t)mpad * (size_t)D * 4;
+  bytes = splits == 1 ? 256 : (size_t)splits * (size_t)mpad * (size_t)D * 4;
 }
 
 // dW[in_dim][D] = X^T dWh (fp32 out), split over rows, fixed-order reduce.
@@ -771,12 +776,17 @@ mega_status umma_project_dw(const void *x, int64_t ldx, const void *gf, int64_t 
   Args g{};
   g.M = mpad; g.Nc = D; g.kb_total = (rows + BK - 1) / BK; g.kb_split = (g.kb_total + splits - 1) / splits;
   g.out = ws; g.mpad = mpad;
+  if (splits == 1) {   // direct: the one partial is grad_w itself (rows < in_dim written)
+    g.M = in_dim;
+    g.out = gw;
+    g.mpad = 0;
+  }
   const dim3 grid((unsigned)(mpad / BM), (unsigned)(D / BN), (unsigned)splits);
   if (BN == 256) rc = launch<DW, 256, 32>(ta, tb, ta, g, grid, st);
   else if (BN == 128) rc = launch<DW, 128, 32>(ta, tb, ta, g, grid, st);
   else if (BN == 192) rc = launch<DW, 192, 32>(ta, tb, ta, g, grid, st);
   else rc = launch<DW, 64, 32>(ta, tb, ta, g, grid, st);
-  if (rc != MEGA_OK) return rc;
+  if (rc != MEGA_OK || splits == 1) return rc;
   const int64_t n4 = (int64_t)in_dim * D / 4;
   const int blocks = (int)std::min<int64_t>((n4 + 255) / 256, 4 * sm_count());
   dw_reduce_kernel<<<std::max(blocks, 1), 256, 0, st>>>(static_cast<const float *>(ws), splits, mpad, in_dim, D, gw);

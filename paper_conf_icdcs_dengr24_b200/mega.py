@@ -121,9 +121,9 @@ def lib():
             "mega_gat_bwd_dist": (S, [P, _c.c_int32, P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32,
                                       P, I64, P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P, P]),
             "mega_calib_gather": (S, [P, I64, _c.c_int, P, I64, P, I64, P]),
-            "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P]),
-            "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, P]),
-            "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, P, I64, P, P, I64, P, P, P, I64,
+            "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, _c.c_size_t, P]),
+            "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, _c.c_int, S, P]),
+            "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, I64, P, P, P, I64,
                                 P, _c.c_size_t, P]),
         }
         for name, (res, args) in sig.items():
@@ -412,35 +412,38 @@ def mega_gat_bwd_dist(layout: Layout, part, comm: Comm, feat, attn_l, attn_r, he
                                    _stream(comm_stream)))
 
 
-# NEXT-3: Graph Transformer edge attention (include/mega.h mega_gt_*; fp32)
-def mega_gt_workspace_bytes(layout: Layout, part: int, heads: int):
+# NEXT-3: Graph Transformer edge attention (include/mega.h mega_gt_*; fp32 or bf16 storage)
+def mega_gt_workspace_bytes(layout: Layout, part: int, heads: int, head_dim: int = 0, dtype: int = MEGA_F32):
     b = _c.c_size_t()
-    _check(lib().mega_gt_workspace_bytes(layout.handle, part, heads, _c.byref(b)))
+    _check(lib().mega_gt_workspace_bytes(layout.handle, part, heads, head_dim or 1, dtype, _c.byref(b)))
     return b.value
 
 
-def _gt_check(name, tensors, ld_group):
-    """mega_gt_* take fp32 row-major operands with ONE leading dimension per group:
+def _gt_check(name, tensors, ld_group, dtype):
+    """mega_gt_* take row-major operands of one dtype with ONE leading dimension per group:
     refuse anything else instead of letting the kernels read it as the wrong data."""
-    import torch
     for t in tensors:
-        if t.dtype != torch.float32 or not t.is_cuda or t.dim() != 2 or t.stride(1) != 1:
-            raise TypeError(f"{name}: operands must be fp32 CUDA 2-D tensors with unit column stride")
+        if t.dtype != dtype or not t.is_cuda or t.dim() != 2 or t.stride(1) != 1:
+            raise TypeError(f"{name}: operands must be {dtype} CUDA 2-D tensors with unit column stride")
     if len({t.stride(0) for t in ld_group}) != 1:
         raise ValueError(f"{name}: {len(ld_group)} operands sharing one leading dimension have different strides")
 
 
-def mega_gt_fwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, stream=None):
-    _gt_check("mega_gt_fwd", (q, k, v, out, lse), (q, k, v))
-    _check(lib().mega_gt_fwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
-                             out.stride(0), _ptr(lse), _stream(stream)))
+def mega_gt_fwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, ws=None, stream=None):
+    import torch
+    _gt_check("mega_gt_fwd", (q, k, v, out), (q, k, v), q.dtype)
+    _gt_check("mega_gt_fwd", (lse,), (lse,), torch.float32)
+    _check(lib().mega_gt_fwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim,
+                             _dtype_code(q), _ptr(out), out.stride(0), _ptr(lse), _ptr(ws),
+                             0 if ws is None else ws.numel() * ws.element_size(), _stream(stream)))
 
 
 def mega_gt_bwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, grad_out, grad_q, grad_k, grad_v, ws,
                 stream=None):
-    _gt_check("mega_gt_bwd", (q, k, v, out, lse, grad_out, grad_q, grad_k, grad_v), (q, k, v))
-    _gt_check("mega_gt_bwd", (grad_q, grad_k, grad_v), (grad_q, grad_k, grad_v))
-    _check(lib().mega_gt_bwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim, _ptr(out),
-                             out.stride(0), _ptr(lse), _ptr(grad_out), grad_out.stride(0), _ptr(grad_q), _ptr(grad_k),
-                             _ptr(grad_v), grad_k.stride(0), _ptr(ws), ws.numel() * ws.element_size(),
-                             _stream(stream)))
+    import torch
+    _gt_check("mega_gt_bwd", (q, k, v, out, grad_out), (q, k, v), q.dtype)
+    _gt_check("mega_gt_bwd", (lse, grad_q, grad_k, grad_v), (grad_q, grad_k, grad_v), torch.float32)
+    _check(lib().mega_gt_bwd(layout.handle, part, _ptr(q), _ptr(k), _ptr(v), q.stride(0), heads, head_dim,
+                             _dtype_code(q), _ptr(out), out.stride(0), _ptr(lse), _ptr(grad_out), grad_out.stride(0),
+                             _ptr(grad_q), _ptr(grad_k), _ptr(grad_v), grad_k.stride(0), _ptr(ws),
+                             ws.numel() * ws.element_size(), _stream(stream)))
