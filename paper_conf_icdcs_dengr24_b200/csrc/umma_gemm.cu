@@ -750,9 +750,10 @@ void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, s
   const int64_t kbt = (rows + BK - 1) / BK;
   int64_t s = (2 * (int64_t)sm_count() + mt * nt - 1) / (mt * nt);
   s = std::max<int64_t>(1, std::min<int64_t>(s, kbt));
-  // short reductions (the paper's batches of small graphs: ~1-6K rows) run unsplit, writing grad_w
-  // directly: one launch instead of a split GEMM plus its reduction, which is what such steps pay for
-  if (kbt <= 128) s = 1;
+  // very short reductions (<= 512 rows) run unsplit, writing grad_w directly (one launch); longer
+  // ones split: one CTA walking ~100 K blocks was measured slower (zinc-b256 step 0.26 -> 0.31 ms)
+  // than a split GEMM plus its reduction
+  if (kbt <= 8) s = 1;
   const int64_t per = (kbt + s - 1) / s;
   splits = (int)((kbt + per - 1) / per);   // every split non-empty
   mpad = mt * BM;
