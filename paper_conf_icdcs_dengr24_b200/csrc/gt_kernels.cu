@@ -211,11 +211,11 @@ __global__ void __launch_bounds__(kWarps * 32) gt_bwd_src_kernel(Args a) {
   }
 }
 
-mega_status check(const mega_layout *L, int32_t part, int heads, int head_dim, int &sms) {
+mega_status check(const mega_layout *L, int32_t part, int heads, int head_dim, int &sms, bool bf16 = false) {
   if (!L) return fail(MEGA_ERR_INVALID_ARGUMENT, "null layout");
   if (part < 0 || part >= (int32_t)L->parts.size()) return fail(MEGA_ERR_INVALID_ARGUMENT, "part out of range");
-  if (heads < 1 || heads > 8 || head_dim < 1 || head_dim > kMaxF)
-    return fail(MEGA_ERR_UNSUPPORTED, "GT kernels: heads in [1, 8], head_dim in [1, 128]");
+  if (heads < 1 || heads > 8 || head_dim < 1 || (!bf16 && head_dim > kMaxF))
+    return fail(MEGA_ERR_UNSUPPORTED, "GT kernels: heads in [1, 8], head_dim in [1, 128] (fp32)");
   int dev = 0, major = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(e));
@@ -284,7 +284,7 @@ mega_status mega_gt_fwd(const mega_layout *L, int32_t part, const void *q_, cons
   clear_error();
   NvtxRange nvtx_("mega_gt_fwd");
   int sms = 0;
-  mega_status rc = gt::check(L, part, heads, head_dim, sms);
+  mega_status rc = gt::check(L, part, heads, head_dim, sms, dtype == MEGA_BF16);
   if (rc != MEGA_OK) return rc;
   if (!q_ || !k_ || !v_ || !out_ || !lse) return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
   const int64_t D = (int64_t)heads * head_dim;
@@ -316,7 +316,7 @@ mega_status mega_gt_bwd(const mega_layout *L, int32_t part, const void *q_, cons
   clear_error();
   NvtxRange nvtx_("mega_gt_bwd");
   int sms = 0;
-  mega_status rc = gt::check(L, part, heads, head_dim, sms);
+  mega_status rc = gt::check(L, part, heads, head_dim, sms, dtype == MEGA_BF16);
   if (rc != MEGA_OK) return rc;
   if (!q_ || !k_ || !v_ || !out_ || !lse || !grad_out_ || !grad_q || !grad_k || !grad_v || !ws)
     return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
