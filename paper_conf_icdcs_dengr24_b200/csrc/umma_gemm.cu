@@ -582,7 +582,15 @@ __global__ void __launch_bounds__(256) dw_reduce_kernel(const float *parts, int 
     const int64_t e = 4 * i;
     const int64_t k = e / D, d = e % D;
     float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
-    for (int z = 0; z < splits; ++z) {
+    int z = 0;
+    for (; z + 8 <= splits; z += 8) {   // 8 independent loads in flight, then the fixed-order adds
+      float4 v[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) v[u] = *reinterpret_cast<const float4 *>(parts + ((int64_t)(z + u) * mpad + k) * D + d);
+#pragma unroll
+      for (int u = 0; u < 8; ++u) { s.x += v[u].x; s.y += v[u].y; s.z += v[u].z; s.w += v[u].w; }
+    }
+    for (; z < splits; ++z) {
       const float4 v = *reinterpret_cast<const float4 *>(parts + ((int64_t)z * mpad + k) * D + d);
       s.x += v.x; s.y += v.y; s.z += v.z; s.w += v.w;
     }
@@ -754,7 +762,7 @@ void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, s
   // ones split: one CTA walking ~100 K blocks was measured slower (zinc-b256 step 0.26 -> 0.31 ms)
   // than a split GEMM plus its reduction
   if (kbt <= 8) s = 1;
-  const int64_t per = (kbt + s - 1) / s;
+  const int64_t per = std::max<int64_t>(kbt <= 8 ? kbt : 4, (kbt + s - 1) / s);   // >= 4 K blocks per split
   splits = (int)((kbt + per - 1) / per);   // every split non-empty
   mpad = mt * BM;
   bytes = splits == 1 ? 256 : (size_t)splits * (size_t)mpad * (size_t)D * 4;
