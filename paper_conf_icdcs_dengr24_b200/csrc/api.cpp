@@ -4,6 +4,7 @@
 #include <algorithm>
 #include <cstdio>
 #include <functional>
+#include <cstdlib>
 #include <cstring>
 #include <new>
 
@@ -21,36 +22,28 @@ void clear_error() { g_last_error.clear(); }
 static const size_t kAlign = 256;
 static size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 
-// Device image of one part: 9 int32 arrays at 256-byte aligned offsets.
-// Device image: the view arrays, plus two derived per-edge arrays the
-// edge-streaming kernels read (erow: CSR edge -> local row; csrc: CSC edge ->
-// source), 4 bytes per edge each.
-std::vector<int32_t> make_tiles(const std::vector<int32_t> &items) {
-  std::vector<int32_t> t;
-  int32_t b = 0, e = 0;
-  bool open = false;
-  auto close = [&] {
-    if (open) t.insert(t.end(), {b, e, -1, 0});
-    open = false;
-  };
-  for (size_t k = 0; k + 3 < items.size(); k += 4) {
-    const int32_t e0 = items[k + 1], e1 = items[k + 2], slot = items[k + 3];
-    if (e1 == e0) continue;
-    if (slot >= 0) {
-      t.insert(t.end(), {e0, e1, slot, 0});
-      continue;
-    }
-    if (open && e == e0 && (e1 - b) <= kTileEdges) {
-      e = e1;
-    } else {
-      close();
-      b = e0;
-      e = e1;
-      open = true;
+// Device image of one part: kImageArrays int32 arrays at 256-byte aligned offsets (the view
+// arrays, the chunk schedules, the k-GPU item lists and halo plan, the destination-pass order).
+std::vector<int32_t> make_chunks(const std::vector<int32_t> &items, int q, int cap) {
+  std::vector<int32_t> c;
+  const int64_t n = (int64_t)items.size() / 4;
+  c.reserve(n / 4 + 2);
+  c.push_back(0);
+  int64_t cost = 0, cnt = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    cost += (int64_t)items[4 * i + 2] - items[4 * i + 1] + kChunkItemCost;
+    if (++cnt >= cap || cost >= q) {
+      c.push_back((int32_t)(i + 1));
+      cost = cnt = 0;
     }
   }
-  close();
-  return t;
+  if (c.back() != (int32_t)n) c.push_back((int32_t)n);
+  return c;
+}
+
+int chunk_quantum(bool fwd) {
+  const char *e = std::getenv(fwd ? "MEGA_SCHED_Q" : "MEGA_SCHED_QB");
+  return e ? std::max(0, std::atoi(e)) : (fwd ? kChunkEdgesFwd : kChunkEdgesBwd);
 }
 
 // Forward work split by source owner for the k-GPU path:
@@ -139,8 +132,10 @@ size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays
   }
   const size_t sizes[kImageArrays] = {P.indptr.size(), P.src.size(), P.cindptr.size(), P.cdst.size(),
                                       P.csr2csc.size(), P.fwd_items.size(), P.fwd_splits.size(),
-                                      P.bwd_items.size(), P.bwd_splits.size(), P.src.size(), P.cdst.size(),
-                                      make_tiles(P.fwd_items).size(), make_tiles(P.bwd_items).size(), P.cpos.size(),
+                                      P.bwd_items.size(), P.bwd_splits.size(),
+                                      make_chunks(P.fwd_items, chunk_quantum(true), kChunkCapFwd).size(),
+                                      make_chunks(P.bwd_items, chunk_quantum(false), kChunkCapBwd).size(), 0, 0,
+                                      P.cpos.size(),
                                       dl.size(), dr.size(), ds.size(), hs.size(), hr.size(), hp.size(),
                                       P.indptr.size() - 1};
   size_t off = 0;
@@ -337,12 +332,10 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
       pcdst[q] = (int32_t)(((uint32_t)degree_class(P.indptr[r + 1] - P.indptr[r]) << 26) | (uint32_t)r);
     }
   }
-  std::vector<int32_t> erow(P.src.size()), csrc(P.cdst.size());
-  for (size_t r = 0; r + 1 < P.indptr.size(); ++r)
-    for (int32_t q = P.indptr[r]; q < P.indptr[r + 1]; ++q) erow[q] = (int32_t)r;
-  for (int64_t v = 0; v < L->n; ++v)
-    for (int32_t q = P.cindptr[v]; q < P.cindptr[v + 1]; ++q) csrc[q] = (int32_t)v;
-  const std::vector<int32_t> ftiles = make_tiles(P.fwd_items), btiles = make_tiles(P.bwd_items);
+  // balanced chunks of work items (the kernels' schedule, see make_chunks)
+  const std::vector<int32_t> fchunks = make_chunks(P.fwd_items, chunk_quantum(true), kChunkCapFwd);
+  const std::vector<int32_t> bchunks = make_chunks(P.bwd_items, chunk_quantum(false), kChunkCapBwd);
+  const std::vector<int32_t> none;
   if (L->parts.size() > 1) {
     dist_items(L, part, P.dl_items, P.dr_items, P.d_splits, P.n_d_slots);
     halo_plan(L, part, P.hsend_idx, P.hsend_off, P.hrecv_idx, P.hrecv_off, P.hpos);
@@ -371,7 +364,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   }
   const std::vector<int32_t> *arrs[kImageArrays] = {
       &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
-      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &erow, &csrc, &ftiles, &btiles, &P.cpos,
+      &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &fchunks, &bchunks, &none, &none, &P.cpos,
       &P.dl_items, &P.dr_items, &P.d_splits, &P.hsend_idx, &P.hrecv_idx, &P.hpos, &dorder};
   char *base = static_cast<char *>(dev_buf);
   for (int i = 0; i < kImageArrays; ++i) {
@@ -392,13 +385,11 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.fwd_splits = reinterpret_cast<const int32_t *>(base + offs[6]);
   D.bwd_items = reinterpret_cast<const int4 *>(base + offs[7]);
   D.bwd_splits = reinterpret_cast<const int32_t *>(base + offs[8]);
-  D.erow = reinterpret_cast<const int32_t *>(base + offs[9]);
-  D.csrc = reinterpret_cast<const int32_t *>(base + offs[10]);
-  D.ftiles = reinterpret_cast<const int4 *>(base + offs[11]);
-  D.btiles = reinterpret_cast<const int4 *>(base + offs[12]);
+  D.fchunk = reinterpret_cast<const int32_t *>(base + offs[9]);
+  D.bchunk = reinterpret_cast<const int32_t *>(base + offs[10]);
   D.cpos = reinterpret_cast<const int32_t *>(base + offs[13]);
-  D.n_ftiles = (int32_t)(ftiles.size() / 4);
-  D.n_btiles = (int32_t)(btiles.size() / 4);
+  D.n_fchunks = (int32_t)fchunks.size() - 1;
+  D.n_bchunks = (int32_t)bchunks.size() - 1;
   D.n = L->n;
   D.rows = P.row_end - P.row_begin;
   D.row_begin = P.row_begin;

@@ -227,21 +227,38 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
   const T *feat = static_cast<const T *>(a.feat);
   const T *featl = feat + gl * EPV;
-  const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
-  const int64_t it0 = ((int64_t)blockIdx.x * WPB + w) * GPW + grp, n_items = a.L.n_fwd_items;
-  if (it0 >= n_items) return;
+  // the group's work: a sequence of chunks of the balanced schedule (DevPart::fchunk: items [b, b + n),
+  // n <= 8 <= G; without one, the k-GPU passes, one item per chunk), one descriptor batch per chunk.
+  // Chunks are claimed in layout order from a counter (a.ctr), three batches ahead of use, so the
+  // groups work on a window of about one round of chunks however unevenly the warps are scheduled;
+  // a.ctr == nullptr: static striding, chunk gid + k W for the group's batch k (MEGA_SCHED_DYN=0)
+  const int64_t W = (int64_t)gridDim.x * WPB * GPW, gid = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
+  const int32_t *fc = a.L.fchunk;
+  const int64_t n_ch = fc ? a.L.n_fchunks : a.L.n_fwd_items;
   auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
     const T *rp = featl + (jj & idm) * ldf;
     const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
     for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
   };
-  // descriptor batch k: items it0 + (kG + l) stride, l < G, into s_desc[k & 1].  Static striding keeps
-  // the groups in a window of ~gridDim * WPB * GPW consecutive rows of the MEGA order (measured: dynamic
-  // claims of G consecutive items per group widen that window G-fold and cost 40% on products)
-  auto stage_desc = [&](int k) {
-    const int64_t itq = it0 + ((int64_t)k * G + gl) * stride;
-    if (itq < n_items) cp_async_small<16>(&s_desc[k & 1][w][rb + gl], a.L.fwd_items + itq);
+  auto next_chunk = [&](int k) -> int64_t {
+    if (a.ctr) {
+      int c = 0;
+      if (gl == 0) c = atomicAdd(a.ctr, 1);
+      return __shfl_sync(gmask, c, rb);
+    }
+    return gid + (int64_t)k * W;
+  };
+  auto bounds = [&](int64_t c, int &b, int &n) {
+    b = 0;
+    n = 0;
+    if (c < n_ch) {
+      if (fc) { b = __ldg(fc + c); n = __ldg(fc + c + 1) - b; }
+      else { b = (int)c; n = 1; }
+    }
+  };
+  auto stage_desc = [&](int k, int b, int n) {
+    if (gl < n) cp_async_small<16>(&s_desc[k & 1][w][rb + gl], a.L.fwd_items + b + gl);
     cp_async_commit();
   };
   // chunk (itm, bse): source ids (tail lanes repeat the last edge) and, for the first chunk of an item, el
@@ -257,9 +274,19 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
     cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
     cp_async_commit();
   };
-  // prologue: descriptor batches 0 and 1, chunk 0 staged
-  stage_desc(0);
-  stage_desc(1);
+  // prologue: descriptor batches 0 and 1 staged, batch 2's bounds in registers, batch 3's chunk claimed
+  int kb = 0, cnt_cur, cnt_nxt, b2, n2;
+  int64_t c3;
+  {
+    int b0, b1;
+    bounds(next_chunk(0), b0, cnt_cur);
+    if (cnt_cur == 0) return;
+    bounds(next_chunk(1), b1, cnt_nxt);
+    stage_desc(0, b0, cnt_cur);
+    stage_desc(1, b1, cnt_nxt);
+    bounds(next_chunk(2), b2, n2);
+    c3 = next_chunk(3);
+  }
   cp_async_wait<1>();
   __syncwarp(gmask);
   int q = 0;
@@ -280,18 +307,23 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
     bool has_next = true;
     if (nbase >= item.z) {
       nq = q + 1;
-      if (it0 + (int64_t)nq * stride >= n_items) {
+      if (nq < cnt_cur) {
+        nitem = s_desc[kb & 1][w][rb + nq];
+        nbase = nitem.y;
+      } else if (cnt_nxt == 0) {
         has_next = false;
-      } else {
-        if (nq % G == 0) {  // entering descriptor batch nq/G: make sure it landed, refill the other buffer
-          cp_async_wait<0>();
-          __syncwarp(gmask);
-          nitem = s_desc[(nq / G) & 1][w][rb];
-          __syncwarp(gmask);
-          stage_desc(nq / G + 1);
-        } else {
-          nitem = s_desc[(nq / G) & 1][w][rb + (int)(nq % G)];
-        }
+      } else {  // entering descriptor batch kb + 1: make sure it landed, refill the finished buffer
+        cp_async_wait<0>();
+        __syncwarp(gmask);
+        nitem = s_desc[(kb + 1) & 1][w][rb];
+        __syncwarp(gmask);
+        ++kb;
+        nq = 0;
+        stage_desc(kb + 1, b2, n2);
+        cnt_cur = cnt_nxt;
+        cnt_nxt = n2;
+        bounds(c3, b2, n2);
+        c3 = next_chunk(kb + 3);
         nbase = nitem.y;
       }
     }
@@ -814,7 +846,32 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
     }
     cp_async_commit();
   };
-  for (int64_t it = (int64_t)blockIdx.x * WPB + w; it < a.L.n_bwd_items; it += stride) {
+  // work: chunks c = warp, warp + W, ... of the balanced schedule (DevPart::bchunk; without one,
+  // the k-GPU passes over their own item ranges, one item per chunk)
+  // chunks are claimed in layout order from a.ctr one chunk ahead of use (as in the forward);
+  // a.ctr == nullptr: static striding
+  const int32_t *bc = a.L.bchunk;
+  const int64_t n_bch = bc ? a.L.n_bchunks : a.L.n_bwd_items;
+  auto claim = [&](int64_t stat) -> int64_t {
+    if (!a.ctr) return stat;
+    int c = 0;
+    if (lane == 0) c = atomicAdd(a.ctr, 1);
+    return __shfl_sync(gmask, c, 0);
+  };
+  int64_t ch = claim((int64_t)blockIdx.x * WPB + w), it_end = 0;
+  int64_t ch_next = claim(ch + stride);
+  auto chunk_begin = [&]() -> int64_t {
+    if (ch >= n_bch) return -1;
+    it_end = bc ? __ldg(bc + ch + 1) : ch + 1;
+    return bc ? __ldg(bc + ch) : ch;
+  };
+  auto next_item = [&](int64_t it) -> int64_t {
+    if (++it < it_end) return it;
+    ch = ch_next;
+    ch_next = claim(ch + stride);
+    return chunk_begin();
+  };
+  for (int64_t it = chunk_begin(); it >= 0; it = next_item(it)) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
     float whf[V][EPV], acc[V][EPV], derv[V], dacc = 0.f;
@@ -1297,8 +1354,6 @@ int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
   return c;
 }
 
-// L2 policy of gathered rows (ablation knob MEGA_L2_POLICY): 0 = hot rows evict_last, the rest
-// evict_first (default); 1 = all evict_normal; 2 = hot evict_last, rest evict_normal
 int st_hint_mode() {   // MEGA_ST_HINT=0 turns the evict_first hints on streamed results off (ablation)
   static int v = -1;
   if (v < 0) {
@@ -1307,11 +1362,15 @@ int st_hint_mode() {   // MEGA_ST_HINT=0 turns the evict_first hints on streamed
   }
   return v;
 }
+// L2 policy of gathered rows (ablation knob MEGA_L2_POLICY): 0 = hot rows evict_last, the rest
+// evict_first (round 1's default); 1 = all evict_normal (default: evict_first lines get ~30 MB of
+// the L2, profiles/r02/l2/, and with the claimed schedule the pin on hot rows no longer pays);
+// 2 = hot evict_last, rest evict_normal
 int l2_policy_mode() {
   static int v = -1;
   if (v < 0) {
     const char *e = std::getenv("MEGA_L2_POLICY");
-    v = e ? std::atoi(e) : 0;
+    v = e ? std::atoi(e) : 1;
   }
   return v;
 }
@@ -1368,17 +1427,29 @@ mega_status check_part(const mega_layout *L, int32_t part, int &dev) {
   return MEGA_OK;
 }
 
-struct WsFwd { size_t m, l, acc, total; };
+// work-claim counters (one per claiming launch of a call), zeroed at the start of the call
+constexpr int kCtrs = 64;
+struct WsFwd { size_t m, l, acc, ctr, total; };
 WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   WsFwd w;
   size_t slots = (size_t)std::max(1, D.n_fwd_slots);
   w.m = 0;
   w.l = align256(w.m + slots * s.H * 4);
   w.acc = align256(w.l + slots * s.H * 4);
-  w.total = align256(w.acc + slots * s.D * 4);
+  w.ctr = align256(w.acc + slots * s.D * 4);
+  w.total = align256(w.ctr + kCtrs * 4);
   return w;
 }
-struct WsBwd { size_t dz, bacc, bder, dal, dar, total; };
+// MEGA_SCHED_DYN=0: static striding over the chunks instead of claiming them (ablation)
+bool sched_dynamic() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_SCHED_DYN");
+    v = e ? std::atoi(e) : 1;
+  }
+  return v != 0;
+}
+struct WsBwd { size_t dz, bacc, bder, dal, dar, ctr, total; };
 WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   WsBwd w;
   size_t slots = (size_t)std::max(1, D.n_bwd_slots);
@@ -1387,7 +1458,8 @@ WsBwd ws_bwd(const DevPart &D, const Shape &s) {
   w.bder = align256(w.bacc + slots * s.D * 4);
   w.dal = align256(w.bder + slots * s.H * 4);
   w.dar = align256(w.dal + (size_t)MAX_GRID * s.D * 8);
-  w.total = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
+  w.ctr = align256(w.dar + (size_t)MAX_GRID * s.D * 8);
+  w.total = align256(w.ctr + kCtrs * 4);
   return w;
 }
 DevPart host_counts(const Part &P, int64_t n) {  // sizes without binding
@@ -1577,6 +1649,12 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
+  a.ctr = nullptr;
+  if (sched_dynamic()) {
+    a.ctr = reinterpret_cast<int *>(wb + w.ctr);
+    cudaError_t ce = cudaMemsetAsync(a.ctr, 0, kCtrs * 4, st);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));
+  }
   return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(a, s, st, dev) : run_fwd<float>(a, s, st, dev);
 }
 
@@ -1629,6 +1707,13 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
   cudaStream_t st = (cudaStream_t)stream;
+  a.ctr = nullptr;
+  const uint32_t ph = flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST);
+  if (sched_dynamic() && (ph == 0 || (ph & MEGA_BWD_PHASE_SRC))) {
+    a.ctr = reinterpret_cast<int *>(wb + w.ctr);
+    cudaError_t ce = cudaMemsetAsync(a.ctr, 0, kCtrs * 4, st);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));
+  }
   return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(a, s, flags, st, dev) : run_bwd<float>(a, s, flags, st, dev);
 }
 
@@ -1758,9 +1843,13 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
-  auto pass = [&](const int4 *items, int32_t nitems, const int32_t *splits, int32_t nsplits) {
+  // counters: 0 = the local pass, 1 = the remote pass; zeroed by the SEND phase (the RECV phase may be
+  // a separate call)
+  int *ctrs = sched_dynamic() ? reinterpret_cast<int *>(wb + w.ctr) : nullptr;
+  auto pass = [&](const int4 *items, int32_t nitems, const int32_t *splits, int32_t nsplits, int ci) {
     kern::FwdArgs b = a;
-    b.L.fwd_items = items; b.L.n_fwd_items = nitems;
+    b.ctr = ctrs ? ctrs + ci : nullptr;
+    b.L.fwd_items = items; b.L.n_fwd_items = nitems; b.L.fchunk = nullptr;
     b.L.fwd_splits = splits; b.L.n_fwd_splits = nsplits;
     return dtype == MEGA_BF16 ? run_fwd<__nv_bfloat16>(b, s, st, dev) : run_fwd<float>(b, s, st, dev);
   };
@@ -1783,12 +1872,16 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
       rc = launch_eler_any(dtype, fb + b0 * ldf * esz, ldf, rows, b0, attn_l, attn_r, heads, head_dim, ctx, ctx + plane, st);
       if (rc != MEGA_OK) return rc;
     }
+    if (ctrs) {
+      cudaError_t ce = cudaMemsetAsync(ctrs, 0, kCtrs * 4, st);
+      if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));
+    }
     // pack the own rows the peers need, send them on the comm stream, receive the peers' rows ...
     if ((rc = move_rows(fb, ldf * esz, DP.hsend_idx, sf, rf, nullptr, DP.n_hsend, (int)rf, st, dev)) != MEGA_OK) return rc;
     if ((rc = move_rows(ctx + plane, re, DP.hsend_idx, se, re, nullptr, DP.n_hsend, (int)re, st, dev)) != MEGA_OK) return rc;
     if ((rc = comm_exchange(comm, sends, recvs, st, cs, true, false)) != MEGA_OK) return rc;
     // ... while block (p, p) (sources this rank owns) runs on the compute stream
-    if ((rc = pass(DP.dl_items, DP.n_dl_items, nullptr, 0)) != MEGA_OK) return rc;
+    if ((rc = pass(DP.dl_items, DP.n_dl_items, nullptr, 0, 0)) != MEGA_OK) return rc;
   }
   if (rcv) {
     if ((rc = comm_exchange(comm, sends, recvs, st, cs, false, true)) != MEGA_OK) return rc;
@@ -1799,8 +1892,8 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
     if (ce == cudaSuccess) ce = cudaStreamWaitEvent(st, comm_done_event(comm), 0);
     if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("wait comm: ") + cudaGetErrorString(ce));
     // remote blocks, then the fixed-order merge of the rows split across passes / segments (KB7)
-    if ((rc = pass(DP.dr_items, DP.n_dr_items, nullptr, 0)) != MEGA_OK) return rc;
-    if ((rc = pass(nullptr, 0, DP.d_splits, DP.n_d_splits)) != MEGA_OK) return rc;
+    if ((rc = pass(DP.dr_items, DP.n_dr_items, nullptr, 0, 1)) != MEGA_OK) return rc;
+    if ((rc = pass(nullptr, 0, DP.d_splits, DP.n_d_splits, 2)) != MEGA_OK) return rc;
   }
   return MEGA_OK;
 }
@@ -1862,11 +1955,16 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
+  a.ctr = nullptr;
   cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;
+  // counters 0..2: the three source-phase launches of the SEND phase (zeroed there)
+  int *ctrs = sched_dynamic() ? reinterpret_cast<int *>(wb + w.ctr) : nullptr;
+  int npass = 0;
   // source-phase launches over a range of CSC items [i0, i1) and splits [s0, s1)
   auto src_range = [&](int32_t i0, int32_t i1, int32_t s0, int32_t s1, bool dlt) {
     kern::BwdArgs b = a;
-    b.L.bwd_items = P.dev.bwd_items + i0; b.L.n_bwd_items = std::max(0, i1 - i0);
+    b.ctr = ctrs ? ctrs + npass++ : nullptr;
+    b.L.bwd_items = P.dev.bwd_items + i0; b.L.n_bwd_items = std::max(0, i1 - i0); b.L.bchunk = nullptr;
     b.L.bwd_splits = P.dev.bwd_splits + 3 * s0; b.L.n_bwd_splits = std::max(0, s1 - s0);
     return dtype == MEGA_BF16 ? run_bwd<__nv_bfloat16>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt)
                               : run_bwd<float>(b, s, MEGA_BWD_PHASE_SRC, st, dev, dlt);
@@ -1887,6 +1985,10 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   }
   const DevPart &D = P.dev;
   if (snd) {
+    if (ctrs) {
+      cudaError_t ce = cudaMemsetAsync(ctrs, 0, kCtrs * 4, st);
+      if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));
+    }
     // Dlt, then the sources other ranks own (their partials travel while ours are computed)
     if ((rc = src_range(0, D.bwd_own0, 0, D.bsplit_own0, true)) != MEGA_OK) return rc;
     if ((rc = src_range(D.bwd_own1, D.n_bwd_items, D.bsplit_own1, D.n_bwd_splits, false)) != MEGA_OK) return rc;

@@ -301,6 +301,7 @@ struct FwdArgs {
   int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
   int st_hint;  // 1: streamed results (out rows) stored with L2 evict_first (MEGA_ST_HINT)
   int pol_mode; // MEGA_L2_POLICY
+  int *ctr;     // zeroed work-claim counter (workspace), nullptr = static striding (MEGA_SCHED_DYN=0)
 };
 
 struct BwdArgs {
@@ -328,6 +329,7 @@ struct BwdArgs {
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int st_hint;  // 1: streamed results (dWh, dz, der) and the source's own Wh row use L2 evict_first
   int pol_mode; // MEGA_L2_POLICY
+  int *ctr;     // zeroed work-claim counter of the source pass (workspace), nullptr = static striding
 };
 
 }  // namespace kern

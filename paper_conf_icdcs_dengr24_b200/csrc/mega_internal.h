@@ -36,13 +36,14 @@ struct DevPart {
   const int32_t *fwd_splits = nullptr;
   const int4 *bwd_items = nullptr;
   const int32_t *bwd_splits = nullptr;
-  const int32_t *erow = nullptr;     // [E_p] local destination row of each CSR edge (device only)
-  const int32_t *csrc = nullptr;     // [E_p] source of each CSC edge (device only)
+  // balanced chunks of work items (make_chunks): chunk c = items [fchunk[c], fchunk[c+1]); a kernel's
+  // group g takes chunks g, g + W, g + 2W, ... (W groups), so all groups advance through the layout
+  // order at the same rate.  nullptr (the k-GPU passes over their own item lists): one item per chunk
+  const int32_t *fchunk = nullptr;   // [n_fchunks + 1]
+  const int32_t *bchunk = nullptr;   // [n_bchunks + 1]
   const int32_t *cpos = nullptr;      // [E_p] CSR position of each CSC edge (dz is stored in CSR order)
   const int32_t *dorder = nullptr;   // [rows] destination-pass row order: heavy rows first (see bind)
-  const int4 *ftiles = nullptr;      // (e_begin, e_end, slot, 0): runs of whole CSR rows / one split segment
-  const int4 *btiles = nullptr;      // the same over the CSC (sources)
-  int32_t n_ftiles = 0, n_btiles = 0;
+  int32_t n_fchunks = 0, n_bchunks = 0;
   int64_t n = 0, rows = 0, row_begin = 0, edges = 0;
   // src (CSR) and cdst (CSC) entries carry a degree class in bits [31:26] when
   // n < 2^26: class = floor(2 log2(deg)) of the row they name (out-degree of the
@@ -119,11 +120,15 @@ bool comm_is_local(const mega_comm *c);
 mega_status comm_exchange(mega_comm *c, const std::vector<CommMsg> &sends, const std::vector<CommMsg> &recvs,
                           cudaStream_t ready_on, cudaStream_t cs, bool phase_send, bool phase_recv);
 cudaEvent_t comm_done_event(mega_comm *c);
-// Edge tiles of the streaming kernels: consecutive unsplit work items are
-// merged while their edges stay contiguous and total <= kTileEdges; a split
-// segment (slot >= 0) is a tile of its own; rows without edges are skipped.
-constexpr int kTileEdges = 512;
-std::vector<int32_t> make_tiles(const std::vector<int32_t> &items);
+// Work schedule of the gathering kernels: consecutive work items (layout order) are grouped into
+// chunks of about q edge-equivalents (each item costs its edges + kChunkItemCost), at most cap
+// items (the forward stages one chunk's descriptors in one pass of its >= 8-lane groups).  With
+// W groups taking chunks g, g + W, ..., every group gets the same work per round, so the groups
+// stay within a few rounds of each other and the rows gathered concurrently stay in a narrow
+// window of the order (L2 reuse).  q = 0: one item per chunk (plain item striding).
+// MEGA_SCHED_Q / MEGA_SCHED_QB override q for the forward / source pass at bind time.
+constexpr int kChunkItemCost = 2, kChunkEdgesFwd = 256, kChunkEdgesBwd = 256, kChunkCapFwd = 8, kChunkCapBwd = 1 << 30;
+std::vector<int32_t> make_chunks(const std::vector<int32_t> &items, int q, int cap);
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]);
 // degree class: floor(2 log2 d) for d >= 1, clamped to 63; 0 for d = 0
 inline int degree_class(int64_t d) {
