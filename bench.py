@@ -138,16 +138,17 @@ def floor_bytes(kernel, rows, N, E, H, D, sb, R=None):
 def design_bytes(kernel, rows, N, E, H, D, sb):
     """The design's own compulsory bytes (LP_ONLY training path): what these
     kernels must move given the layout (16-byte work items, the cpos map, dz in CSR order,
-    the bf16 projection operand written instead of fp32 dWh)."""
+    the bf16 projection operand written instead of fp32 dWh; in bf16 the source pass's dWh
+    partial also lives in that operand, DESIGN.md R-lp)."""
     items = 16 * rows
+    pb = sb if sb == 2 else 4   # bytes of the dWh partial handed from the source to the destination pass
     if kernel == "KB2":   # idx, items, Wh, er (all sources once), el, out, lse
         return 4 * E + items + N * D * sb + N * H * 4 + rows * H * 4 + rows * D * sb + rows * H * 4
     if kernel == "KB3+KB4":   # g,out -> Dlt; cdst, cpos, items, Wh, er, g_i, el/lse/Dlt, dz, dWh, der
         return ((2 * rows * D * sb + rows * H * 4) + (8 * E + 16 * N + N * D * sb + N * H * 4 + rows * D * sb
-                                                       + 3 * rows * H * 4 + 4 * E * H + N * D * 4 + N * H * 4))
+                                                       + 3 * rows * H * 4 + 4 * E * H + N * D * pb + N * H * 4))
     if kernel == "KB5":   # indptr, dz, dWh partial, der, Wh, bf16 operand
-        pb = sb if sb == 2 else 4
-        return 4 * (rows + 1) + 4 * E * H + rows * D * 4 + rows * H * 4 + rows * D * sb + rows * D * pb
+        return 4 * (rows + 1) + 4 * E * H + rows * D * pb + rows * H * 4 + rows * D * sb + rows * D * pb
     raise KeyError(kernel)
 
 

@@ -364,11 +364,13 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
         s_p[w][lane][h] = p;
       }
     }
+    if (base != item.y) {   // acc is 0 in an item's first chunk
 #pragma unroll
-    for (int v = 0; v < V; ++v) {
-      const float f = sel<HT>(sc, ((v * G + gl) * EPV) / FF);
+      for (int v = 0; v < V; ++v) {
+        const float f = sel<HT>(sc, ((v * G + gl) * EPV) / FF);
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
+        for (int k = 0; k < EPV; ++k) acc[v][k] *= f;
+      }
     }
     // next chunk's ids have had the score phase to land: stage its er, prefetch its rows
     cp_async_wait<0>();
@@ -774,8 +776,10 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
           y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-          *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
+          if (!a.lp_partial)
+            *reinterpret_cast<float4 *>(orow + v * G * EPV + k) = make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]);
         }
+        if (a.lp_partial) st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()));
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
@@ -1009,8 +1013,9 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
           const float4 r4 = __ldg(reinterpret_cast<const float4 *>(arp + k));
           y[k] = fmaf(derv[v], r4.x, acc[v][k]); y[k + 1] = fmaf(derv[v], r4.y, acc[v][k + 1]);
           y[k + 2] = fmaf(derv[v], r4.z, acc[v][k + 2]); y[k + 3] = fmaf(derv[v], r4.w, acc[v][k + 3]);
-          st16f_pol(orow + v * G * EPV + k, make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]), pol_st);
+          if (!a.lp_partial) st16f_pol(orow + v * G * EPV + k, make_float4(y[k], y[k + 1], y[k + 2], y[k + 3]), pol_st);
         }
+        if (a.lp_partial) st16_pol(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + (v * G + gl) * EPV, pack(y, T()), pol_st);
         if (head_lead<G, LPH>(gl, v)) a.der[j * H + hv[v]] = derv[v];
       }
     } else {
@@ -1058,8 +1063,12 @@ __global__ void __launch_bounds__(TPB) gat_bwd_src_merge_kernel(const BwdArgs a)
       float *orow = a.gfeat + j * a.ldgf + col;
 #pragma unroll
       for (int k = 0; k < EPV; ++k) y[k] = fmaf(der, a.ar[col + k], y[k]);
+      if (a.lp_partial) {
+        st16(static_cast<T *>(a.gfeat_lp) + j * a.ldlp + col, pack(y, T()));
+      } else {
 #pragma unroll
-      for (int k = 0; k < EPV; ++k) orow[k] = y[k];
+        for (int k = 0; k < EPV; ++k) orow[k] = y[k];
+      }
     }
   }
 }
@@ -1111,12 +1120,16 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
     float *gr = a.gfeat + grow * a.ldgf + gl * EPV;
     const T *wr = feat + grow * a.ldf + gl * EPV;
     float4 part[V][EPV / 4];
-    uint4 whp[V];
+    uint4 whp[V], plp[V];
 #pragma unroll
     for (int v = 0; v < V; ++v) {
       whp[v] = ldg16(wr + v * G * EPV);
+      if (a.lp_partial) {   // the source pass left its partial in the bf16 operand (read back, in place)
+        plp[v] = *reinterpret_cast<const uint4 *>(static_cast<const T *>(a.gfeat_lp) + grow * a.ldlp + (v * G + gl) * EPV);
+      } else {
 #pragma unroll
-      for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
+        for (int k = 0; k < EPV / 4; ++k) part[v][k] = *reinterpret_cast<const float4 *>(gr + v * G * EPV + 4 * k);
+      }
     }
     float derr[HT];
     load_h<HT>(a.der + grow * H, H, derr);
@@ -1149,6 +1162,12 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
       const float d = sel<HT>(del, hv[v]), dr = sel<HT>(derr, hv[v]);
       float y[EPV], wh[EPV];
       unpack(whp[v], wh, T());
+      if (a.lp_partial) {   // unpacked only now: its load latency overlapped the dz gather
+        float x[EPV];
+        unpack(plp[v], x, T());
+#pragma unroll
+        for (int k = 0; k < EPV / 4; ++k) part[v][k] = make_float4(x[4 * k], x[4 * k + 1], x[4 * k + 2], x[4 * k + 3]);
+      }
 #pragma unroll
       for (int k = 0; k < EPV / 4; ++k) {
         y[4 * k] = fmaf(d, alv[v][4 * k], part[v][k].x);
@@ -1440,6 +1459,15 @@ WsFwd ws_fwd(const DevPart &D, const Shape &s) {
   w.total = align256(w.ctr + kCtrs * 4);
   return w;
 }
+// MEGA_LP_PARTIAL=0: keep the source pass's dWh partial in fp32 grad_feat in LP_ONLY mode (ablation)
+bool lp_partial_mode() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_LP_PARTIAL");
+    v = e ? std::atoi(e) : 1;
+  }
+  return v != 0;
+}
 // MEGA_SCHED_DYN=0: static striding over the chunks instead of claiming them (ablation)
 bool sched_dynamic() {
   static int v = -1;
@@ -1517,7 +1545,9 @@ mega_status run_fwd(const FwdArgs &a, const Shape &s, cudaStream_t st, int dev) 
           rc = check_launch(st, "gat_fwd_kernel");
         };
         // chunk-pipelined kernel for groups of >= 8 lanes (products 3 layers: 25.5 vs 29.3 ms/step for the
-        // register-batch kernel, which stays for narrow rows: static shared memory of the pipe kernel)
+        // register-batch kernel, which stays for narrow rows: static shared memory of the pipe kernel).
+        // A TMA-ring variant (rows in flight in shared memory, cp.async.bulk per row) measured 9.7 vs
+        // 6.8 ms per products layer: 113 vs 85 warp instructions per edge in an issue-bound kernel
         if constexpr (G >= 8) launch(gat_fwd_pipe_kernel<T, G, V, HT>);
         else launch(gat_fwd_kernel<T, G, V, HT, 0>);
       });
@@ -1703,6 +1733,10 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
+  // LP_ONLY in bf16 with both phases in this call: the source pass leaves dWh's partial in the bf16
+  // operand itself instead of fp32 grad_feat (DESIGN R-lp: 2.5 GB less written and read per products layer)
+  a.lp_partial = a.lp_only && dtype == MEGA_BF16 && !(flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) &&
+                 lp_partial_mode() ? 1 : 0;
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
@@ -1952,6 +1986,7 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.gal = grad_attn_l; a.gar = grad_attn_r;
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
+  a.lp_partial = 0;   // the exchange moves fp32 partials of grad_feat rows
   a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
   a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();

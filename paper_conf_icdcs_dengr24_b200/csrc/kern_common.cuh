@@ -90,9 +90,15 @@ __device__ __forceinline__ uint4 pack(const float (&x)[8], __nv_bfloat16) {
 }
 
 template <int G> __device__ __forceinline__ float gmax(float v, unsigned mask) {
+  if constexpr (G == 32) {   // whole warp: one CREDUX.MAX.F32 (sm_100a) instead of 5 shuffle + max steps
+    float r;
+    asm volatile("redux.sync.max.f32 %0, %1, 0xffffffff;" : "=f"(r) : "f"(v));
+    return r;
+  } else {
 #pragma unroll
-  for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(mask, v, o, G));
-  return v;
+    for (int o = G / 2; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(mask, v, o, G));
+    return v;
+  }
 }
 template <int G> __device__ __forceinline__ float gsum(float v, unsigned mask) {
 #pragma unroll
@@ -326,6 +332,7 @@ struct BwdArgs {
   float *gal, *gar;
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
+  int lp_partial;  // (bf16, lp_only) the source pass's partial rows live in gfeat_lp too (no fp32 gfeat)
   int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int st_hint;  // 1: streamed results (dWh, dz, der) and the source's own Wh row use L2 evict_first
   int pol_mode; // MEGA_L2_POLICY
