@@ -316,22 +316,6 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   int dev = 0;
   cudaError_t ce = cudaGetDevice(&dev);
   if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(ce));
-  // Device copies of src / cdst carry the degree class of the row they name in
-  // bits [31:26] (n < 2^26), the kernels' L2 hot/cold hint; host arrays stay plain.
-  const bool packed = L->n < (1LL << 26);
-  std::vector<int32_t> psrc, pcdst;
-  if (packed) {
-    psrc.resize(P.src.size());
-    pcdst.resize(P.cdst.size());
-    for (size_t q = 0; q < P.src.size(); ++q) {
-      const int32_t j = P.src[q];
-      psrc[q] = (int32_t)(((uint32_t)degree_class(P.cindptr[j + 1] - P.cindptr[j]) << 26) | (uint32_t)j);
-    }
-    for (size_t q = 0; q < P.cdst.size(); ++q) {
-      const int32_t r = P.cdst[q];
-      pcdst[q] = (int32_t)(((uint32_t)degree_class(P.indptr[r + 1] - P.indptr[r]) << 26) | (uint32_t)r);
-    }
-  }
   // balanced chunks of work items (the kernels' schedule, see make_chunks)
   const std::vector<int32_t> fchunks = make_chunks(P.fwd_items, chunk_quantum(true), kChunkCapFwd);
   const std::vector<int32_t> bchunks = make_chunks(P.bwd_items, chunk_quantum(false), kChunkCapBwd);
@@ -363,7 +347,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
       if (!(P.indptr[r + 1] - P.indptr[r] > 2.0 * mean)) dorder.push_back((int32_t)r);
   }
   const std::vector<int32_t> *arrs[kImageArrays] = {
-      &P.indptr, packed ? &psrc : &P.src, &P.cindptr, packed ? &pcdst : &P.cdst, &P.csr2csc, &P.fwd_items,
+      &P.indptr, &P.src, &P.cindptr, &P.cdst, &P.csr2csc, &P.fwd_items,
       &P.fwd_splits, &P.bwd_items, &P.bwd_splits, &fchunks, &bchunks, &none, &none, &P.cpos,
       &P.dl_items, &P.dr_items, &P.d_splits, &P.hsend_idx, &P.hrecv_idx, &P.hpos, &dorder};
   char *base = static_cast<char *>(dev_buf);
@@ -400,7 +384,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
   D.n_bwd_items = (int32_t)(P.bwd_items.size() / 4);
   D.n_bwd_splits = (int32_t)(P.bwd_splits.size() / 3);
   D.n_bwd_slots = P.n_bwd_slots;
-  D.id_mask = packed ? ((1u << 26) - 1u) : 0x7fffffffu;
+  D.id_mask = 0x7fffffffu;
   D.dl_items = reinterpret_cast<const int4 *>(base + offs[14]);
   D.dr_items = reinterpret_cast<const int4 *>(base + offs[15]);
   D.d_splits = reinterpret_cast<const int32_t *>(base + offs[16]);
@@ -425,7 +409,7 @@ mega_status mega_layout_bind_device(mega_layout *L, int32_t part, void *dev_buf,
     D.bsplit_own0 = first_ge(P.bwd_splits, 3, (int32_t)P.row_begin);
     D.bsplit_own1 = first_ge(P.bwd_splits, 3, (int32_t)P.row_end);
   }
-  // pageable-memory copies return once staged, so the packed temporaries may go
+  // pageable-memory copies return once staged, so the temporaries may go
   return MEGA_OK;
 }
 

@@ -59,10 +59,10 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
   __shared__ int s_j[WPB][32];  // packed source id (class bits + id)
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, rb = grp * G;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
+  const int rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
+  const uint64_t pol_cold = policy_first();
   const float *sp_v[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) sp_v[v] = &s_p[w][rb][((v * G + gl) * EPV) / FF];
@@ -71,9 +71,8 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, VAR>::MINB) gat_fwd_kernel(cons
   // element offsets fit in 32 bits (checked on the host: n * ldf < 2^32)
   auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
     const T *rp = featl + (jj & idm) * ldf;
-    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
-    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
+    for (int v = 0; v < V; ++v) r[v] = ldg16(rp + v * G * EPV);
   };
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
     const int4 item = a.L.fwd_items[it];
@@ -217,10 +216,9 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   __shared__ __align__(16) float s_el[2][WPB][GPW][HT];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, rb = grp * G;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
+  const int rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldf = (uint32_t)a.ldf;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode);
   const uint64_t pol_st = a.st_hint ? policy_first() : policy_normal();
   const float *sp_v[V];
 #pragma unroll
@@ -237,9 +235,8 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   const int64_t n_ch = fc ? a.L.n_fchunks : a.L.n_fwd_items;
   auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
     const T *rp = featl + (jj & idm) * ldf;
-    const uint64_t pol = (int)(jj >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
-    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
+    for (int v = 0; v < V; ++v) r[v] = ldg16(rp + v * G * EPV);
   };
   auto next_chunk = [&](int k) -> int64_t {
     if (a.ctr) {
@@ -539,7 +536,7 @@ __global__ void __launch_bounds__(TPB) dlt_kernel(const BwdArgs a) {
   constexpr int EPV = Tr<T>::EPV, GPW = 32 / G, FF = G * V * EPV / HT, LPH = FF / EPV;
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   for (int64_t r = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; r < a.L.rows; r += stride) {
     const T *gr = static_cast<const T *>(a.gout) + r * a.ldg + gl * EPV;
@@ -587,10 +584,10 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   __shared__ int s_i[WPB][32];        // packed destination row
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, rb = grp * G;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
+  const int rb = grp * G;
   const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
+  const uint64_t pol_cold = policy_first();
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / FF;
@@ -605,9 +602,8 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
   const int64_t stride = (int64_t)gridDim.x * WPB * GPW;
   auto row_load = [&](uint4 (&r)[V], uint32_t ii) {
     const T *rp = goutl + (ii & idm) * ldg;
-    const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
 #pragma unroll
-    for (int v = 0; v < V; ++v) r[v] = ldg16_pol(rp + v * G * EPV, pol);
+    for (int v = 0; v < V; ++v) r[v] = ldg16(rp + v * G * EPV);
   };
   for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
     const int4 item = a.L.bwd_items[it];
@@ -803,10 +799,10 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : 2)) gat_bwd_src_kernel(cons
 // lane copies and later reads back exactly its own 16-byte pieces, so the ring
 // needs no barriers, and NBF*U rows per warp are in flight without holding
 // registers (the register-batch kernel keeps 2U = 4 in 125 registers).
-template <typename T, int V, int HT, int NBF>
+template <typename T, int V, int HT, int U, int NBF>
 __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs a) {
   constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, SP = HT + 1;
-  constexpr int U = V >= 4 ? 1 : (V == 2 ? 2 : 4), RS = NBF * U;  // rows per batch, ring slots
+  constexpr int RS = NBF * U;  // ring slots (U rows per batch)
   constexpr int NB = U * V;
   constexpr bool BFLY = LPH >= 2 && LPH <= G && NB >= 2 && NB <= LPH;
   constexpr int UB = U == 1 ? 0 : (U == 2 ? 1 : (U == 4 ? 2 : 3));
@@ -817,11 +813,10 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
   __shared__ int s_i[WPB][32];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane;
   const unsigned gmask = 0xffffffffu;
-  const int H = a.H;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
   uint4 *ring = ring_all + (size_t)w * RS * V * 32;
   const uint32_t idm = a.L.id_mask, ldg = (uint32_t)a.ldg;
-  const int hot_cls = a.hot_cls;
-  const uint64_t pol_hot = row_policy_hot(a.pol_mode), pol_row = row_policy_cold(a.pol_mode), pol_cold = policy_first();
+  const uint64_t pol_cold = policy_first();
   const uint64_t pol_st = a.st_hint ? policy_first() : policy_normal();
   int hv[V];
 #pragma unroll
@@ -842,10 +837,9 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       for (int u = 0; u < U; ++u) {
         const uint32_t ii = (uint32_t)s_i[w][min(b * U + u, cnt - 1)];
         const T *rp = goutl + (ii & idm) * ldg;
-        const uint64_t pol = (int)(ii >> 26) >= hot_cls ? pol_hot : pol_row;
         uint4 *dst = ring + (((b % NBF) * U + u) * V) * 32 + lane;
 #pragma unroll
-        for (int v = 0; v < V; ++v) cp_async16(dst + v * 32, rp + v * G * EPV, pol);
+        for (int v = 0; v < V; ++v) cp_async16_plain(dst + v * 32, rp + v * G * EPV);
       }
     }
     cp_async_commit();
@@ -1082,7 +1076,8 @@ __global__ void __launch_bounds__(TPB, (V >= 4 ? 1 : (V == 2 ? 2 : 3))) gat_bwd_
   __shared__ __align__(16) float s_dz[2][WPB][32][HT];
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, gl = lane % G, grp = lane / G;
   const unsigned gmask = G == 32 ? 0xffffffffu : (((1u << G) - 1u) << (grp * G));
-  const int H = a.H, rb = grp * G;
+  constexpr int H = HT;   // heads is a power of two <= 8, dispatched as HT == heads (check_shape)
+  const int rb = grp * G;
   int hv[V];
   float dal[V][EPV], dar[V][EPV], alv[V][EPV];
 #pragma unroll
@@ -1348,31 +1343,6 @@ bool debug_sync() {
   return v == 1;
 }
 
-// L2 budget (MB) for rows pinned with evict_last; 0 disables the hints.
-double l2_hot_mb() {
-  static double v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_L2_HOT_MB");
-    v = e ? std::atof(e) : 64.0;
-  }
-  return v;
-}
-
-// Degree-class threshold: the hottest classes whose rows fit the L2 hot budget
-// (rows gathered at most once, class 0, are never hot).  64 disables the hints.
-int hot_class(const int64_t (&cls)[64], uint32_t id_mask, size_t row_bytes) {
-  const double mb = l2_hot_mb();
-  if (mb <= 0 || id_mask == 0x7fffffffu) return 64;
-  const double budget = mb * 1024.0 * 1024.0;
-  double used = 0;
-  int c = 64;
-  while (c > 1 && used + (double)cls[c - 1] * (double)row_bytes <= budget) {
-    used += (double)cls[c - 1] * (double)row_bytes;
-    --c;
-  }
-  return c;
-}
-
 int st_hint_mode() {   // MEGA_ST_HINT=0 turns the evict_first hints on streamed results off (ablation)
   static int v = -1;
   if (v < 0) {
@@ -1381,19 +1351,6 @@ int st_hint_mode() {   // MEGA_ST_HINT=0 turns the evict_first hints on streamed
   }
   return v;
 }
-// L2 policy of gathered rows (ablation knob MEGA_L2_POLICY): 0 = hot rows evict_last, the rest
-// evict_first (round 1's default); 1 = all evict_normal (default: evict_first lines get ~30 MB of
-// the L2, profiles/r02/l2/, and with the claimed schedule the pin on hot rows no longer pays);
-// 2 = hot evict_last, rest evict_normal
-int l2_policy_mode() {
-  static int v = -1;
-  if (v < 0) {
-    const char *e = std::getenv("MEGA_L2_POLICY");
-    v = e ? std::atoi(e) : 1;
-  }
-  return v;
-}
-
 mega_status check_launch(cudaStream_t s, const char *what) {
   cudaError_t e = cudaGetLastError();
   if (e != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
@@ -1581,9 +1538,11 @@ mega_status run_bwd(BwdArgs a, const Shape &s, uint32_t flags, cudaStream_t st, 
         if (a.L.n_bwd_items > 0) {
           bool ring = false;
           if constexpr (G == 32 && V <= 2) {
-            // shared-memory ring, 4 batches in flight (products 3 layers: gat_bwd 60.5 -> 52.9 ms/step)
-            constexpr int U = V == 2 ? 2 : 4, NBF = 4;
-            auto kr = gat_bwd_src_ring_kernel<T, V, HT, NBF>;
+            // shared-memory ring, NBF batches of U rows in flight: (U, NBF) = (4, 2) for 2 vectors per lane,
+            // (8, 2) for 1 (round 1: (2, 4) / (4, 4)); products per step gat_bwd_src 34.2 -> 31.4 ms, reddit
+            // 8.3 -> 7.6; (2 U, 3) and (U / 2, 6) measured slower (profiles/r02/ring/)
+            constexpr int U = V == 2 ? 4 : 8, NBF = 2;
+            auto kr = gat_bwd_src_ring_kernel<T, V, HT, U, NBF>;
             const size_t smem = (size_t)WPB * NBF * U * V * 32 * 16;
             cudaFuncSetAttribute(kr, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
             int nblk = 0;
@@ -1676,8 +1635,6 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
-  a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
   a.ctr = nullptr;
   if (sched_dynamic()) {
@@ -1737,8 +1694,6 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   // operand itself instead of fp32 grad_feat (DESIGN R-lp: 2.5 GB less written and read per products layer)
   a.lp_partial = a.lp_only && dtype == MEGA_BF16 && !(flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST)) &&
                  lp_partial_mode() ? 1 : 0;
-  a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
-  a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
   cudaStream_t st = (cudaStream_t)stream;
   a.ctr = nullptr;
@@ -1874,8 +1829,6 @@ mega_status mega_gat_fwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.ws_m = reinterpret_cast<float *>(wb + w.m);
   a.ws_l = reinterpret_cast<float *>(wb + w.l);
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
-  a.hot_cls = hot_class(P.out_cls, P.dev.id_mask, (size_t)s.D * esz);
-  a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
   // counters: 0 = the local pass, 1 = the remote pass; zeroed by the SEND phase (the RECV phase may be
   // a separate call)
@@ -1987,8 +1940,6 @@ mega_status mega_gat_bwd_dist(const mega_layout *L, int32_t part, mega_comm *com
   a.nb_dst = 0;
   a.lp_only = (flags & MEGA_BWD_LP_ONLY) && grad_feat_lp ? 1 : 0;
   a.lp_partial = 0;   // the exchange moves fp32 partials of grad_feat rows
-  a.hot_cls = hot_class(P.in_cls, P.dev.id_mask, (size_t)s.D * esz);
-  a.pol_mode = l2_policy_mode();
   a.st_hint = st_hint_mode();
   a.ctr = nullptr;
   cudaStream_t st = (cudaStream_t)stream, cs = (cudaStream_t)comm_stream;

@@ -38,10 +38,6 @@ __device__ __forceinline__ uint64_t policy_normal() {
   asm("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
   return p;
 }
-// L2 policy of gathered feature rows (MEGA_L2_POLICY): 0 = hot rows evict_last,
-// the rest evict_first; 1 = all evict_normal; 2 = hot evict_last, rest evict_normal.
-__device__ __forceinline__ uint64_t row_policy_hot(int mode) { return mode == 1 ? policy_normal() : policy_last(); }
-__device__ __forceinline__ uint64_t row_policy_cold(int mode) { return mode == 0 ? policy_first() : policy_normal(); }
 __device__ __forceinline__ uint4 ldg16(const void *p) { return __ldg(reinterpret_cast<const uint4 *>(p)); }
 __device__ __forceinline__ uint4 ldg16_pol(const void *p, uint64_t pol) {
   uint4 r;
@@ -262,6 +258,10 @@ __device__ __forceinline__ void cp_async16(void *smem, const void *gmem, uint64_
   asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "l"(pol)
                : "memory");
 }
+__device__ __forceinline__ void cp_async16_plain(void *smem, const void *gmem) {
+  const uint32_t s = (uint32_t)__cvta_generic_to_shared(smem);
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(s), "l"(gmem) : "memory");
+}
 __device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 template <int N> __device__ __forceinline__ void cp_async_wait() {
   asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory");
@@ -304,9 +304,7 @@ struct FwdArgs {
   void *out;
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
-  int hot_cls;  // source rows of degree class >= hot_cls are kept in L2 (64 = no hints)
   int st_hint;  // 1: streamed results (out rows) stored with L2 evict_first (MEGA_ST_HINT)
-  int pol_mode; // MEGA_L2_POLICY
   int *ctr;     // zeroed work-claim counter (workspace), nullptr = static striding (MEGA_SCHED_DYN=0)
 };
 
@@ -333,9 +331,7 @@ struct BwdArgs {
   int nb_dst;
   int lp_only;     // MEGA_BWD_LP_ONLY: the final rows go to gfeat_lp only
   int lp_partial;  // (bf16, lp_only) the source pass's partial rows live in gfeat_lp too (no fp32 gfeat)
-  int hot_cls;  // destination rows of degree class >= hot_cls: their g rows are kept in L2
   int st_hint;  // 1: streamed results (dWh, dz, der) and the source's own Wh row use L2 evict_first
-  int pol_mode; // MEGA_L2_POLICY
   int *ctr;     // zeroed work-claim counter of the source pass (workspace), nullptr = static striding
 };
 

@@ -45,9 +45,8 @@ struct DevPart {
   const int32_t *dorder = nullptr;   // [rows] destination-pass row order: heavy rows first (see bind)
   int32_t n_fchunks = 0, n_bchunks = 0;
   int64_t n = 0, rows = 0, row_begin = 0, edges = 0;
-  // src (CSR) and cdst (CSC) entries carry a degree class in bits [31:26] when
-  // n < 2^26: class = floor(2 log2(deg)) of the row they name (out-degree of the
-  // source in this part / in-degree of the destination); id = entry & id_mask.
+  // id = entry & id_mask (round 1 packed a degree class into the high bits for L2 hints; now
+  // plain ids, mask all ones)
   uint32_t id_mask = 0x7fffffffu;
   int32_t n_fwd_items = 0, n_fwd_splits = 0, n_fwd_slots = 0;
   int32_t n_bwd_items = 0, n_bwd_splits = 0, n_bwd_slots = 0;

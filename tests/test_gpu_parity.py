@@ -199,9 +199,8 @@ def test_lp_only_flag_matches(cuda_device):
 
 
 SCHED_VARIANTS = {
-    "round1": {"MEGA_SCHED_DYN": "0", "MEGA_SCHED_Q": "0", "MEGA_SCHED_QB": "0", "MEGA_L2_POLICY": "0",
-               "MEGA_LP_PARTIAL": "0"},
-    "static_chunks": {"MEGA_SCHED_DYN": "0", "MEGA_L2_POLICY": "2"},
+    "round1": {"MEGA_SCHED_DYN": "0", "MEGA_SCHED_Q": "0", "MEGA_SCHED_QB": "0", "MEGA_LP_PARTIAL": "0"},
+    "static_chunks": {"MEGA_SCHED_DYN": "0"},
     "claimed_items": {"MEGA_SCHED_Q": "0", "MEGA_SCHED_QB": "0"},
 }
 
