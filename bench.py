@@ -117,6 +117,12 @@ def peaks():
     return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "source": "fallback (B200_PROFILING.md)"}
 
 
+# Measured ceiling of gathering random 1 KB rows through L2 (scripts/l2probe.cu, all hits: working set
+# <= 64 MB, 16 GB requested per launch, 8 CTAs/SM): 17.4 TB/s requested (profiles/r02/l2/probe_p0.txt).
+# The gathering kernels' "gather_frac" is their requested row rate against it (E rows of D*s bytes).
+L2_GATHER_TBS = 17.4
+
+
 def floor_bytes(kernel, rows, N, E, H, D, sb, R=None):
     """SURVEY §8(d)-d3 algorithmic bytes of one launch group, with R row fetches of the
     gathered operand (R = N: the compulsory floor, every gathered row once; R = E: no
@@ -549,6 +555,12 @@ def run_mega(args):
         ent = {"call": call, "ms": calls[call], "floor_bytes": fb, "noreuse_bytes": nb, "design_bytes": db,
                "achieved_gbs": fb / t / 1e9, "frac": fb / t / 1e9 / pk["hbm_gbs"],
                "noreuse_frac": nb / t / 1e9 / pk["hbm_gbs"], "design_frac": db / t / 1e9 / pk["hbm_gbs"]}
+        if kname in ("KB2", "KB3+KB4"):   # the row-gathering kernels: requested rows vs the L2 gather ceiling
+            req = E * D * sb
+            ent["gather_requested_bytes"] = req
+            ent["gather_tbs"] = req / t / 1e12
+            ent["gather_ceiling_tbs"] = L2_GATHER_TBS
+            ent["gather_frac"] = ent["gather_tbs"] / L2_GATHER_TBS
         if ncu and kname in ncu and world == 1:
             ent["traffic"] = ncu[kname]["dram_bytes"]
             ent["traffic_gbs"] = ncu[kname]["dram_bytes"] / t / 1e9
