@@ -410,6 +410,54 @@ mega_status mega_gt_bwd(const mega_layout *layout, int32_t part, const void *q, 
  * >= 64 * SM-count entries) so the loads cannot be elided.  Time it with CUDA
  * events to get the achievable row-gather bandwidth for an index pattern.
  * Errors: INVALID_ARGUMENT, UNSUPPORTED, OUT_OF_MEMORY (sink), CUDA. */
+/* ---------------- NEXT-2: the faithful path-band representation ----------------
+ * The paper's own layout (Fig. 7): traversal F of
+ * Algorithm 1 (DESIGN.md R-band) builds a path P of node
+ * appearances with revisits that covers every edge of the symmetrised simple
+ * graph exactly once by a pair of appearances at most `window` apart (theta =
+ * 1); the directed input multiset is stored on those pairs (multiplicities,
+ * self-loops at a node's first appearance), so GAT over the band equals GAT
+ * over the input (north_star).  Node ids are the INPUT ids (no relabelling).
+ * Host build and view; the caller binds a device image like a layout. */
+typedef struct mega_band mega_band;
+typedef struct {
+  uint32_t struct_size;
+  int64_t num_nodes, num_edges, length; /* length = |P| */
+  int32_t window, cap;
+  int64_t jumps, virtual_edges, edges_u; /* tier-3 jumps, non-adjacent steps, |E_u| */
+  int64_t num_slots, num_merges;         /* partial states of nodes appearing more than once */
+  double build_seconds;
+  const int32_t *P;             /* [length] input node id of each appearance */
+  const uint64_t *own;          /* [length] bit o-1: edge {P[t], P[t-o]} covered when P[t] was appended */
+  const uint64_t *lmask, *rmask;/* [length] bit o-1: an input edge P[t-o] -> P[t] / P[t+o] -> P[t] */
+  const int32_t *cptr;          /* [length+1] offsets into cnt */
+  const uint16_t *cnt;          /* multiplicities: lmask bits ascending, rmask bits, then self-loops */
+  const int32_t *slot;          /* [length] partial slot or -1 */
+  const int32_t *merges;        /* [num_merges][3] (node, first slot, count) */
+} mega_band_view;
+/* window 0 = auto clamp(round(m/n), 1, 64) (<= 64); cap 0 = 32.
+ * Errors: INVALID_ARGUMENT, INVALID_GRAPH, UNSUPPORTED (a multiplicity > 65535), OUT_OF_MEMORY. */
+mega_status mega_band_build(const mega_csr *csr, int32_t window, int32_t cap, mega_band **out);
+void mega_band_destroy(mega_band *band);
+mega_status mega_band_view_get(const mega_band *band, mega_band_view *out);
+mega_status mega_band_device_bytes(const mega_band *band, size_t *bytes);
+mega_status mega_band_bind_device(mega_band *band, void *dev_buf, size_t bytes, mega_stream_t stream);
+/* GAT forward over the band: appearance tiles stream their window of rows
+ * feat[P[t]] (t in [t0 - window, t1 + window)) into shared memory once and
+ * aggregate each appearance's band in-edges from there (no per-edge gather);
+ * nodes appearing more than once merge their appearances' partial softmax
+ * states in fixed order.  feat / out device [num_nodes][ld] dtype (input
+ * ids), rows of 32 x 16-byte vectors x V (bf16 D = 256 / 512 / 1024, fp32 D =
+ * 128 / 256 / 512); el / er / lse: ctx planes as mega_gat_fwd (el / er
+ * computed from feat unless MEGA_FLAG_ELER_IN_CTX); ws >= ws_bytes from
+ * mega_band_gat_workspace_bytes.  Errors as mega_gat_fwd. */
+mega_status mega_band_gat_workspace_bytes(const mega_band *band, int heads, int head_dim, mega_dtype dtype,
+                                          size_t *ws_bytes);
+mega_status mega_band_gat_fwd(const mega_band *band, const void *feat, int64_t ldf, const float *attn_l,
+                              const float *attn_r, int heads, int head_dim, mega_dtype dtype, float negative_slope,
+                              uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws, size_t ws_bytes,
+                              mega_stream_t stream);
+
 mega_status mega_calib_gather(const void *table, int64_t rows, int row_bytes, const int32_t *idx, int64_t n,
                               float *sink, int64_t sink_len, mega_stream_t stream);
 

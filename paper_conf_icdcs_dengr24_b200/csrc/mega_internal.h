@@ -66,6 +66,19 @@ struct DevPart {
   int64_t n_hsend = 0, n_hrecv = 0;
 };
 
+// NEXT-2 band layout, device pointers (band.cpp / band_kernels.cu)
+struct BandDev {
+  const int32_t *P = nullptr;                  // [L] node of each appearance
+  const unsigned long long *lmask = nullptr;   // [L] bit o-1: in-edge from P[t-o]
+  const unsigned long long *rmask = nullptr;   // [L] bit o-1: in-edge from P[t+o]
+  const int32_t *cptr = nullptr;               // [L+1] offsets into cnt
+  const uint16_t *cnt = nullptr;               // multiplicities (lmask bits, rmask bits, self-loops)
+  const int32_t *slot = nullptr;               // [L] partial slot or -1
+  const int32_t *merges = nullptr;             // [n_merges][3] (node, first slot, count)
+  int64_t L = 0, n = 0;
+  int32_t omega = 0, n_merges = 0, n_slots = 0;
+};
+
 struct Part {
   int64_t row_begin = 0, row_end = 0;
   // k > 1 dist items (derived from indptr/src/bounds at bind time; host copies for the view)
@@ -109,6 +122,10 @@ void halo_plan(const mega_layout *L, int part, std::vector<int32_t> &send_idx, s
                std::vector<int32_t> &recv_idx, std::vector<int32_t> &recv_off, std::vector<int32_t> &pos);
 // comm.cpp: one exchange of (peer, pointer, bytes) messages (see mega_comm)
 struct CommMsg { int peer; int tag; const void *ptr; size_t bytes; };
+}  // namespace mega
+struct mega_band;
+namespace mega {
+const BandDev *band_dev(const mega_band *B, int &device);
 }  // namespace mega
 struct mega_comm;
 namespace mega {

@@ -121,6 +121,14 @@ def lib():
             "mega_gat_bwd_dist": (S, [P, _c.c_int32, P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32,
                                       P, I64, P, I64, P, P, I64, P, I64, P, P, P, _c.c_size_t, P, P]),
             "mega_calib_gather": (S, [P, I64, _c.c_int, P, I64, P, I64, P]),
+            "mega_band_build": (S, [P, _c.c_int32, _c.c_int32, P]),
+            "mega_band_destroy": (None, [P]),
+            "mega_band_view_get": (S, [P, P]),
+            "mega_band_device_bytes": (S, [P, P]),
+            "mega_band_bind_device": (S, [P, P, _c.c_size_t, P]),
+            "mega_band_gat_workspace_bytes": (S, [P, _c.c_int, _c.c_int, S, P]),
+            "mega_band_gat_fwd": (S, [P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64, P, P,
+                                      _c.c_size_t, P]),
             "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, _c.c_size_t, P]),
             "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, _c.c_int, S, P]),
             "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, I64, P, P, P, I64,
@@ -447,3 +455,84 @@ def mega_gt_bwd(layout: Layout, part, q, k, v, heads, head_dim, out, lse, grad_o
                              _dtype_code(q), _ptr(out), out.stride(0), _ptr(lse), _ptr(grad_out), grad_out.stride(0),
                              _ptr(grad_q), _ptr(grad_k), _ptr(grad_v), grad_k.stride(0), _ptr(ws),
                              ws.numel() * ws.element_size(), _stream(stream)))
+
+
+# ---------------- NEXT-2: the faithful path-band layout (include/mega.h) ----------------
+class mega_band_view(_c.Structure):
+    _fields_ = [("struct_size", _c.c_uint32), ("num_nodes", _c.c_int64), ("num_edges", _c.c_int64),
+                ("length", _c.c_int64), ("window", _c.c_int32), ("cap", _c.c_int32), ("jumps", _c.c_int64),
+                ("virtual_edges", _c.c_int64), ("edges_u", _c.c_int64), ("num_slots", _c.c_int64),
+                ("num_merges", _c.c_int64), ("build_seconds", _c.c_double), ("P", P), ("own", P), ("lmask", P),
+                ("rmask", P), ("cptr", P), ("cnt", P), ("slot", P), ("merges", P)]
+
+
+class Band:
+    """Owns a mega_band* and its device image."""
+
+    def __init__(self, handle):
+        self._h = _c.c_void_p(handle)
+        self._dev = None
+
+    def __del__(self):
+        if getattr(self, "_h", None) and self._h.value and _lib is not None:
+            _lib.mega_band_destroy(self._h)
+            self._h = _c.c_void_p(None)
+
+    @property
+    def handle(self):
+        return self._h
+
+    def view(self):
+        v = mega_band_view()
+        v.struct_size = _c.sizeof(mega_band_view)
+        _check(lib().mega_band_view_get(self._h, _c.byref(v)))
+        L = v.length
+        d = {k: getattr(v, k) for k, _ in mega_band_view._fields_[1:12]}
+
+        def arr(ptr, n, dt):
+            if n == 0 or not ptr:
+                return np.zeros(0, dt)
+            return np.ctypeslib.as_array(_c.cast(ptr, _c.POINTER(np.ctypeslib.as_ctypes_type(dt))), (n,)).copy()
+        d["P"] = arr(v.P, L, np.int32)
+        d["own"] = arr(v.own, L, np.uint64)
+        d["lmask"] = arr(v.lmask, L, np.uint64)
+        d["rmask"] = arr(v.rmask, L, np.uint64)
+        d["cptr"] = arr(v.cptr, L + 1, np.int32)
+        d["cnt"] = arr(v.cnt, int(d["cptr"][-1]) if L else 0, np.uint16)
+        d["slot"] = arr(v.slot, L, np.int32)
+        d["merges"] = arr(v.merges, 3 * v.num_merges, np.int32).reshape(-1, 3)
+        return d
+
+    def bind(self, stream=None):
+        import torch
+        nb = _c.c_size_t()
+        _check(lib().mega_band_device_bytes(self._h, _c.byref(nb)))
+        n = max(nb.value, 256)
+        buf = torch.empty(n + 256, dtype=torch.uint8, device="cuda")
+        off = (-buf.data_ptr()) % 256
+        _check(lib().mega_band_bind_device(self._h, _c.c_void_p(buf.data_ptr() + off), nb.value, _stream(stream)))
+        self._dev = buf
+        return buf
+
+
+def mega_band_build(indptr, indices, window=0, cap=0) -> Band:
+    indptr = np.ascontiguousarray(indptr, dtype=np.int64)
+    indices = np.ascontiguousarray(indices, dtype=np.int32)
+    csr = mega_csr(len(indptr) - 1, len(indices), indptr.ctypes.data, indices.ctypes.data)
+    h = _c.c_void_p()
+    _check(lib().mega_band_build(_c.byref(csr), window, cap, _c.byref(h)))
+    return Band(h.value)
+
+
+def mega_band_gat_workspace_bytes(band: Band, heads: int, head_dim: int, dtype: int) -> int:
+    w = _c.c_size_t()
+    _check(lib().mega_band_gat_workspace_bytes(band.handle, heads, head_dim, dtype, _c.byref(w)))
+    return w.value
+
+
+def mega_band_gat_fwd(band: Band, feat, attn_l, attn_r, heads, head_dim, out, ctx, ws, negative_slope=SLOPE,
+                      flags=0, stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_band_gat_fwd(band.handle, _ptr(feat), feat.stride(0), _ptr(attn_l), _ptr(attn_r), heads,
+                                   head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0), _ptr(ctx), _ptr(ws),
+                                   ws.numel() * ws.element_size(), _stream(stream)))
