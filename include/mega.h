@@ -458,6 +458,20 @@ mega_status mega_band_gat_fwd(const mega_band *band, const void *feat, int64_t l
                               uint32_t flags, void *out, int64_t ldo, float *ctx, void *ws, size_t ws_bytes,
                               mega_stream_t stream);
 
+/* Backward of mega_band_gat_fwd (a6-a8 on the band): Dlt per node; a source pass over
+ * appearance tiles (window rows of grad_out staged in shared memory) accumulates each
+ * appearance's share of sum alpha g_i and der_j and records c dz at each band entry; the
+ * per-appearance del sums; a node pass sums a node's appearances in order and writes
+ * grad_feat = sum alpha g + der a_r + del a_l (fp32 [num_nodes][ldgf]), the der plane
+ * of ctx and fixed-order da_l / da_r.  out / grad_out: dtype [num_nodes][ld] (input
+ * ids); ctx: as written by mega_band_gat_fwd; ws >= mega_band_gat_workspace_bytes.
+ * Errors as mega_gat_bwd. */
+mega_status mega_band_gat_bwd(const mega_band *band, const void *feat, int64_t ldf, const float *attn_l,
+                              const float *attn_r, int heads, int head_dim, mega_dtype dtype, float negative_slope,
+                              const void *out, int64_t ldo, const void *grad_out, int64_t ldg, float *ctx,
+                              float *grad_feat, int64_t ldgf, float *grad_attn_l, float *grad_attn_r, void *ws,
+                              size_t ws_bytes, mega_stream_t stream);
+
 mega_status mega_calib_gather(const void *table, int64_t rows, int row_bytes, const int32_t *idx, int64_t n,
                               float *sink, int64_t sink_len, mega_stream_t stream);
 

@@ -39,6 +39,8 @@ struct mega_band {
   std::vector<uint16_t> selfc;     // [L] self-loop count (first appearance only)
   std::vector<int32_t> slot;       // [L] partial slot or -1
   std::vector<int32_t> merges;     // [n_merge][3] (node, first slot, count)
+  std::vector<int32_t> app_ptr;    // [n+1] appearances of each node (CSR over app_idx, appearance order)
+  std::vector<int32_t> app_idx;    // [L]
   int32_t n_slots = 0;
   int64_t jumps = 0, virtual_edges = 0, edges_u = 0;
   double seconds = 0;
@@ -51,7 +53,7 @@ struct mega_band {
 namespace mega {
 namespace {
 
-constexpr int kBandArrays = 8;
+constexpr int kBandArrays = 9;
 
 struct G {
   std::vector<int64_t> beg;   // [n+1]
@@ -243,6 +245,13 @@ mega_status band_arrays(int64_t n, const int64_t *indptr, const int32_t *indices
       s += napp[v];
     }
   B.n_slots = s;
+  B.app_ptr.assign(n + 1, 0);
+  for (int64_t v = 0; v < n; ++v) B.app_ptr[v + 1] = B.app_ptr[v] + napp[v];
+  B.app_idx.assign(L, 0);
+  {
+    std::vector<int32_t> fill(B.app_ptr.begin(), B.app_ptr.end() - 1);
+    for (int64_t t = 0; t < L; ++t) B.app_idx[fill[B.P[t]]++] = (int32_t)t;
+  }
   B.slot.assign(L, -1);
   std::vector<int32_t> used(n, 0);
   for (int64_t t = 0; t < L; ++t) {
@@ -256,7 +265,8 @@ size_t align256b(size_t x) { return (x + 255) / 256 * 256; }
 
 size_t band_image(const mega_band &B, size_t offs[kBandArrays]) {
   const size_t L = B.P.size();
-  const size_t sizes[kBandArrays] = {L * 4, L * 8, L * 8, (L + 1) * 4, B.cnt.size() * 2, L * 4, B.merges.size() * 4, 0};
+  const size_t sizes[kBandArrays] = {L * 4, L * 8, L * 8, (L + 1) * 4, B.cnt.size() * 2, L * 4, B.merges.size() * 4,
+                                     B.app_ptr.size() * 4, L * 4};
   size_t off = 0;
   for (int i = 0; i < kBandArrays; ++i) {
     offs[i] = off;
@@ -356,9 +366,10 @@ mega_status mega_band_bind_device(mega_band *B, void *dev_buf, size_t bytes, meg
   if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("cudaGetDevice: ") + cudaGetErrorString(ce));
   char *base = static_cast<char *>(dev_buf);
   const void *src[kBandArrays] = {B->P.data(), B->lmask.data(), B->rmask.data(), B->cptr.data(), B->cnt.data(),
-                                  B->slot.data(), B->merges.data(), nullptr};
+                                  B->slot.data(), B->merges.data(), B->app_ptr.data(), B->app_idx.data()};
   const size_t L = B->P.size();
-  const size_t sizes[kBandArrays] = {L * 4, L * 8, L * 8, (L + 1) * 4, B->cnt.size() * 2, L * 4, B->merges.size() * 4, 0};
+  const size_t sizes[kBandArrays] = {L * 4, L * 8, L * 8, (L + 1) * 4, B->cnt.size() * 2, L * 4, B->merges.size() * 4,
+                                     B->app_ptr.size() * 4, L * 4};
   for (int i = 0; i < kBandArrays; ++i) {
     if (!sizes[i]) continue;
     ce = cudaMemcpyAsync(base + offs[i], src[i], sizes[i], cudaMemcpyHostToDevice, (cudaStream_t)stream);
@@ -374,6 +385,9 @@ mega_status mega_band_bind_device(mega_band *B, void *dev_buf, size_t bytes, meg
   D.cnt = reinterpret_cast<const uint16_t *>(base + offs[4]);
   D.slot = reinterpret_cast<const int32_t *>(base + offs[5]);
   D.merges = reinterpret_cast<const int32_t *>(base + offs[6]);
+  D.app_ptr = reinterpret_cast<const int32_t *>(base + offs[7]);
+  D.app_idx = reinterpret_cast<const int32_t *>(base + offs[8]);
+  D.n_cnt = (int64_t)B->cnt.size();
   D.L = (int64_t)L;
   D.n = B->n;
   D.omega = B->omega;

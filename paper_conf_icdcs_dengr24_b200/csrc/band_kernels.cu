@@ -41,8 +41,21 @@ struct BandArgs {
   int64_t ldo;
   float *ws_m, *ws_l, *ws_acc;
   int D, T, win_cap;
+  // backward
+  const float *al, *ar;
+  const void *gout;
+  int64_t ldg;
+  float *dlt, *der;                 // ctx planes (node ids)
+  float *accD, *derp, *delp, *dzb;  // per appearance partials / per band entry c * dz
+  float *gfeat;
+  int64_t ldgf;
+  double *pdal, *pdar;              // per-block partials of da_l / da_r
+  float *gal, *gar;
 };
 
+__device__ __forceinline__ void *a256d(void *p) {   // 8-byte alignment for the mask arrays
+  return reinterpret_cast<void *>((reinterpret_cast<uintptr_t>(p) + 7) & ~(uintptr_t)7);
+}
 // position (0-based) of the n-th set bit of a 64-bit mask
 __device__ __forceinline__ int nth_bit64(unsigned long long m, int n) {
   const unsigned lo = (unsigned)m;
@@ -228,19 +241,319 @@ __global__ void __launch_bounds__(BW * 32) band_merge_kernel(const BandArgs a) {
   }
 }
 
+// ---- backward over the band (SURVEY §8(a) a6-a8 on the band layout) ----
+// Dlt_x = g_x . out_x per node (a6)
+template <typename T, int V, int HT>
+__global__ void __launch_bounds__(BW * 32) band_dlt_kernel(const BandArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, H = HT;
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int64_t x = (int64_t)blockIdx.x * BW + w; x < a.B.n; x += (int64_t)gridDim.x * BW) {
+    const T *gr = static_cast<const T *>(a.gout) + x * a.ldg + lane * EPV;
+    const T *orr = static_cast<const T *>(a.out) + x * a.ldo + lane * EPV;
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      float xg[EPV], xo[EPV];
+      unpack(ldg16(gr + v * G * EPV), xg, T());
+      unpack(ldg16(orr + v * G * EPV), xo, T());
+      float d = 0.f;
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) d = fmaf(xg[k], xo[k], d);
+      if constexpr (LPH >= G) {
+        d = gsum<G>(d, 0xffffffffu);
+      } else {
+#pragma unroll
+        for (int o = LPH / 2; o > 0; o >>= 1) d += __shfl_xor_sync(0xffffffffu, d, o);
+      }
+      // a head may span several vectors (LPH > G): sum over v of the head in registers
+      const int h = ((v * G + lane) * EPV) / FF;
+      if constexpr (LPH > G) {
+        __shared__ float s_acc[BW][HT];
+        if (lane == 0) s_acc[w][h] = (v % (LPH / G) == 0 ? 0.f : s_acc[w][h]) + d;
+        __syncwarp();
+        if (lane == 0 && (v % (LPH / G)) == LPH / G - 1) a.dlt[x * H + h] = s_acc[w][h];
+        __syncwarp();
+      } else {
+        if ((lane % LPH) == 0) a.dlt[x * H + h] = d;
+      }
+    }
+  }
+}
+
+// Source pass (a7) over appearance tiles: appearance t is source j = P[t] of the band edges
+// t -> t + o (lmask[t+o] bit o-1), t -> t - o (rmask[t-o] bit o-1) and its own self-loops; the window
+// rows g[P[t']] and (el, lse, Dlt)[P[t']] are staged in shared memory.  Per appearance:
+// accD[t] = sum c alpha g_i, derp[t] = sum c dz; c dz is stored at the edge's band entry (dzb).
+template <typename T, int V, int HT>
+__global__ void __launch_bounds__(BW * 32, 2) band_src_kernel(const BandArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, LPH = FF / EPV, H = HT;
+  extern __shared__ __align__(16) uint4 smem[];
+  const int WC = a.win_cap;
+  uint4 *rows = smem;                                                     // [WC][V * 32] g rows
+  float *eld = reinterpret_cast<float *>(rows + (size_t)WC * V * 32);     // [WC][3][HT] el, lse, Dlt
+  int *p_w = reinterpret_cast<int *>(eld + (size_t)WC * 3 * HT);          // [WC]
+  unsigned long long *lm_w = reinterpret_cast<unsigned long long *>(a256d(p_w + WC));  // [WC]
+  unsigned long long *rm_w = lm_w + WC;                                   // [WC]
+  int *cp_w = reinterpret_cast<int *>(rm_w + WC);                         // [WC + 1]
+  __shared__ int s_wi[BW][32], s_pos[BW][32];
+  __shared__ float s_c[BW][32];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  constexpr unsigned FULL = 0xffffffffu;
+  int hv[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) hv[v] = ((v * G + lane) * EPV) / FF;
+  const T *feat = static_cast<const T *>(a.feat);
+  const T *gout = static_cast<const T *>(a.gout);
+  const int64_t L = a.B.L;
+  const int om = a.B.omega;
+  const int64_t ntiles = (L + a.T - 1) / a.T;
+  for (int64_t tile = blockIdx.x; tile < ntiles; tile += gridDim.x) {
+    const int64_t t0 = tile * a.T, t1 = min(L, t0 + a.T);
+    const int64_t wlo = max((int64_t)0, t0 - om), whi = min(L, t1 + om);
+    const int nw = (int)(whi - wlo);
+    __syncthreads();
+    for (int i = threadIdx.x; i < nw; i += blockDim.x) {
+      p_w[i] = a.B.P[wlo + i];
+      lm_w[i] = a.B.lmask[wlo + i];
+      rm_w[i] = a.B.rmask[wlo + i];
+      cp_w[i] = a.B.cptr[wlo + i];
+    }
+    if (threadIdx.x == 0) cp_w[nw] = a.B.cptr[whi];
+    __syncthreads();
+    for (int i = w; i < nw; i += BW) {
+      const T *rp = gout + (int64_t)p_w[i] * a.ldg + lane * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v) cp_async16_plain(rows + ((size_t)i * V + v) * 32 + lane, rp + v * G * EPV);
+    }
+    cp_async_commit();
+    for (int i = threadIdx.x; i < nw * 3 * H; i += blockDim.x) {
+      const int r = i / (3 * H), q = (i / H) % 3, h = i % H;
+      const float *src = q == 0 ? a.el : (q == 1 ? a.lse : a.dlt);
+      eld[i] = src[(int64_t)p_w[r] * H + h];
+    }
+    cp_async_wait<0>();
+    __syncthreads();
+    for (int64_t t = t0 + w; t < t1; t += BW) {
+      const int ti = (int)(t - wlo);
+      const int j = p_w[ti];
+      float whf[V][EPV], acc[V][EPV], erj[HT], dsum[HT];
+      {
+        const T *rp = feat + (int64_t)j * a.ldf + lane * EPV;
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          unpack(ldg16(rp + v * G * EPV), whf[v], T());
+#pragma unroll
+          for (int k = 0; k < EPV; ++k) acc[v][k] = 0.f;
+        }
+      }
+      load_h<HT>(a.er + (int64_t)j * H, H, erj);
+#pragma unroll
+      for (int h = 0; h < HT; ++h) dsum[h] = 0.f;
+      // candidate out-edges: pass 0: t -> t + o, pass 1: t -> t - o (o = lane + 1 + 32 q), pass 2: self
+      const int nself = (cp_w[ti + 1] - cp_w[ti]) - __popcll(lm_w[ti]) - __popcll(rm_w[ti]);
+      for (int pass = 0; pass < 3; ++pass) {
+        for (int q0 = 0; q0 < (pass == 2 ? 1 : (om + 31) / 32); ++q0) {
+          bool ok = false;
+          int wi = 0, pos = 0;
+          if (pass < 2) {
+            const int o = q0 * 32 + lane + 1;
+            const int64_t tp = pass == 0 ? t + o : t - o;
+            if (o <= om && tp >= wlo && tp < whi) {
+              const int di = (int)(tp - wlo);
+              const unsigned long long bit = 1ull << (o - 1);
+              if (pass == 0 && (lm_w[di] & bit)) {   // source to the left of its destination: an lmask entry
+                ok = true;
+                pos = cp_w[di] + __popcll(lm_w[di] & (bit - 1));
+              } else if (pass == 1 && (rm_w[di] & bit)) {
+                ok = true;
+                pos = cp_w[di] + __popcll(lm_w[di]) + __popcll(rm_w[di] & (bit - 1));
+              }
+              wi = di;
+            }
+          } else if (lane == 0 && nself > 0) {
+            ok = true;
+            wi = ti;
+            pos = cp_w[ti + 1] - 1;
+          }
+          const unsigned msk = __ballot_sync(FULL, ok);
+          if (ok) {
+            const int slot = __popc(msk & ((1u << lane) - 1));
+            s_wi[w][slot] = wi;
+            s_pos[w][slot] = pos;
+            s_c[w][slot] = (float)a.B.cnt[pos];
+          }
+          __syncwarp();
+          const int ne = __popc(msk);
+          for (int k = 0; k < ne; ++k) {
+            const int di = s_wi[w][k];
+            const float c = s_c[w][k];
+            const uint4 *gr = rows + (size_t)di * V * 32 + lane;
+            float p[V], xg[V][EPV];
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              unpack(gr[v * 32], xg[v], T());
+              float d = 0.f;
+#pragma unroll
+              for (int kk = 0; kk < EPV; ++kk) d = fmaf(xg[v][kk], whf[v][kk], d);
+              p[v] = d;
+            }
+            // per-head dot over the head's lanes (and vectors)
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+#pragma unroll
+              for (int o = (LPH >= G ? G : LPH) / 2; o > 0; o >>= 1) p[v] += __shfl_xor_sync(FULL, p[v], o);
+            }
+            if constexpr (LPH > G) {   // a head spans LPH / G vectors of a lane
+              constexpr int R = LPH / G;
+#pragma unroll
+              for (int v = 0; v < V; v += R) {
+                float sum = 0.f;
+#pragma unroll
+                for (int r = 0; r < R; ++r) sum += p[v + r];
+#pragma unroll
+                for (int r = 0; r < R; ++r) p[v + r] = sum;
+              }
+            }
+            const float *e3 = eld + (size_t)di * 3 * HT;
+#pragma unroll
+            for (int v = 0; v < V; ++v) {
+              const int h = hv[v];
+              const float z = e3[h] + sel<HT>(erj, h);
+              const float al = fexp(leaky(z, a.slope) - e3[HT + h]);
+              const float dz = c * al * (p[v] - e3[2 * HT + h]) * (z > 0.f ? 1.f : a.slope);
+              const float ca = c * al;
+#pragma unroll
+              for (int kk = 0; kk < EPV; kk += 2) ffma2s(acc[v][kk], acc[v][kk + 1], xg[v][kk], xg[v][kk + 1], ca);
+              // one lane per head records c dz (and sums it)
+              const bool lead = LPH >= G ? (lane == 0 && (v % (LPH >= G ? LPH / G : 1)) == 0) : ((lane % LPH) == 0);
+              if (lead) {
+                a.dzb[(int64_t)s_pos[w][k] * H + h] = dz;
+                dsum[h] += dz;
+              }
+            }
+          }
+          __syncwarp();
+        }
+      }
+      float *ap = a.accD + t * a.D + lane * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; k += 4)
+          *reinterpret_cast<float4 *>(ap + v * G * EPV + k) = make_float4(acc[v][k], acc[v][k + 1], acc[v][k + 2], acc[v][k + 3]);
+      // derp[t][h]: the per-head sums live in the head's lead lane
+#pragma unroll
+      for (int h = 0; h < HT; ++h) {
+        const int lead_lane = LPH >= G ? 0 : ((h * FF / EPV) % G);
+        const float d = __shfl_sync(FULL, dsum[h], lead_lane);
+        if (lane == 0) a.derp[t * H + h] = d;
+      }
+    }
+  }
+}
+
+// delp[t] = sum of c dz over appearance t's band entries (a8, per appearance)
+template <int HT>
+__global__ void __launch_bounds__(256) band_del_kernel(const BandArgs a) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < a.B.L * HT; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t t = i / HT;
+    const int h = (int)(i % HT);
+    float d = 0.f;
+    for (int k = a.B.cptr[t]; k < a.B.cptr[t + 1]; ++k) d += a.dzb[(int64_t)k * HT + h];
+    a.delp[i] = d;
+  }
+}
+
+// per node (a8): del, der over its appearances (appearance order), dWh = sum accD + der a_r + del a_l,
+// and the per-block partials of da_l = sum del Wh, da_r = sum der Wh (fixed order)
+template <typename T, int V, int HT>
+__global__ void __launch_bounds__(BW * 32) band_node_kernel(const BandArgs a) {
+  constexpr int G = 32, EPV = Tr<T>::EPV, FF = G * V * EPV / HT, H = HT;
+  __shared__ double s_red[1024];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  int hv[V];
+  float dal[V][EPV], dar[V][EPV], alv[V][EPV], arv[V][EPV];
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    hv[v] = ((v * G + lane) * EPV) / FF;
+#pragma unroll
+    for (int k = 0; k < EPV; ++k) {
+      dal[v][k] = dar[v][k] = 0.f;
+      alv[v][k] = a.al[(v * G + lane) * EPV + k];
+      arv[v][k] = a.ar[(v * G + lane) * EPV + k];
+    }
+  }
+  const T *feat = static_cast<const T *>(a.feat);
+  for (int64_t x = (int64_t)blockIdx.x * BW + w; x < a.B.n; x += (int64_t)gridDim.x * BW) {
+    const int a0 = a.B.app_ptr[x], a1 = a.B.app_ptr[x + 1];
+    float del[HT], der[HT], y[V][EPV];
+#pragma unroll
+    for (int h = 0; h < HT; ++h) { del[h] = 0.f; der[h] = 0.f; }
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) y[v][k] = 0.f;
+    for (int q = a0; q < a1; ++q) {
+      const int64_t t = a.B.app_idx[q];
+#pragma unroll
+      for (int h = 0; h < HT; ++h) { del[h] += a.delp[t * H + h]; der[h] += a.derp[t * H + h]; }
+      const float *ap = a.accD + t * a.D + lane * EPV;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+#pragma unroll
+        for (int k = 0; k < EPV; ++k) y[v][k] += ap[v * G * EPV + k];
+    }
+    for (int h = lane; h < H; h += G) a.der[x * H + h] = sel<HT>(der, h);
+    float *orow = a.gfeat + x * a.ldgf + lane * EPV;
+    const T *wr = feat + x * a.ldf + lane * EPV;
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      const float dl = sel<HT>(del, hv[v]), dr = sel<HT>(der, hv[v]);
+      float wh[EPV];
+      unpack(ldg16(wr + v * G * EPV), wh, T());
+#pragma unroll
+      for (int k = 0; k < EPV; ++k) {
+        orow[v * G * EPV + k] = y[v][k] + dr * arv[v][k] + dl * alv[v][k];
+        dal[v][k] = fmaf(dl, wh[k], dal[v][k]);
+        dar[v][k] = fmaf(dr, wh[k], dar[v][k]);
+      }
+    }
+  }
+  block_partial<G, V, EPV>(dal, s_red, a.pdal + (int64_t)blockIdx.x * a.D, a.D);
+  block_partial<G, V, EPV>(dar, s_red, a.pdar + (int64_t)blockIdx.x * a.D, a.D);
+}
+
+__global__ void __launch_bounds__(256) band_param_kernel(const BandArgs a, int nblocks) {
+  for (int d = blockIdx.x * blockDim.x + threadIdx.x; d < 2 * a.D; d += gridDim.x * blockDim.x) {
+    const double *pp = d < a.D ? a.pdal : a.pdar;
+    const int c = d % a.D;
+    double s = 0.0;
+    for (int b = 0; b < nblocks; ++b) s += pp[(int64_t)b * a.D + c];
+    (d < a.D ? a.gal : a.gar)[c] = (float)s;
+  }
+}
+
 }  // namespace
 }  // namespace kern
 
 namespace {
 size_t a256(size_t x) { return (x + 255) / 256 * 256; }
-struct BandWs { size_t m, l, acc, total; };
-BandWs band_ws(const BandDev &B, int H, int D) {
+constexpr int kBandMaxNodeBlocks = 1024;
+struct BandWs { size_t m, l, acc, fwd_total, accD, derp, delp, dzb, pdal, pdar, total; };
+BandWs band_ws(int64_t L, int64_t n_cnt, int32_t n_slots, int H, int D) {
   BandWs w;
-  const size_t s = (size_t)std::max(1, B.n_slots);
+  const size_t s = (size_t)std::max(1, n_slots), Lz = (size_t)std::max<int64_t>(1, L);
   w.m = 0;
   w.l = a256(s * H * 4);
   w.acc = a256(w.l + s * H * 4);
-  w.total = a256(w.acc + s * (size_t)D * 4);
+  w.fwd_total = a256(w.acc + s * (size_t)D * 4);
+  // backward (mega_band_gat_bwd): per appearance partials and per band entry c dz
+  w.accD = 0;
+  w.derp = a256(w.accD + Lz * (size_t)D * 4);
+  w.delp = a256(w.derp + Lz * H * 4);
+  w.dzb = a256(w.delp + Lz * H * 4);
+  w.pdal = a256(w.dzb + (size_t)std::max<int64_t>(1, n_cnt) * H * 4);
+  w.pdar = a256(w.pdal + (size_t)kBandMaxNodeBlocks * D * 8);
+  w.total = std::max(w.fwd_total, a256(w.pdar + (size_t)kBandMaxNodeBlocks * D * 8));
   return w;
 }
 }  // namespace
@@ -256,9 +569,7 @@ mega_status mega_band_gat_workspace_bytes(const mega_band *band, int heads, int 
   if (!band || !ws_bytes) return fail(MEGA_ERR_INVALID_ARGUMENT, "null argument");
   mega_band_view v;
   mega_band_view_get(band, &v);
-  BandDev B;
-  B.n_slots = (int32_t)v.num_slots;
-  *ws_bytes = band_ws(B, heads, heads * head_dim).total;
+  *ws_bytes = band_ws(v.length, v.cptr ? v.cptr[v.length] : 0, (int32_t)v.num_slots, heads, heads * head_dim).total;
   (void)dtype;
   return MEGA_OK;
 }
@@ -289,8 +600,8 @@ mega_status mega_band_gat_fwd(const mega_band *band, const void *feat, int64_t l
   if (lph > 32 ? (lph % 32 || V % (lph / 32)) : (32 % lph)) return fail(MEGA_ERR_UNSUPPORTED, "band kernel: head_dim");
   if (ldf < D || ldo < D || (ldf * esz) % 16 || (ldo * esz) % 16) return fail(MEGA_ERR_INVALID_ARGUMENT, "bad ld");
   const BandDev &B = *Bp;
-  const BandWs w = band_ws(B, heads, D);
-  if (ws_bytes < w.total) return fail(MEGA_ERR_OUT_OF_MEMORY, "band workspace too small");
+  const BandWs w = band_ws(B.L, B.n_cnt, B.n_slots, heads, D);
+  if (ws_bytes < w.fwd_total) return fail(MEGA_ERR_OUT_OF_MEMORY, "band workspace too small");
   const size_t row_b = (size_t)D * esz, per_row = row_b + 4 * heads + 4;
   const int win_cap = (int)(kern::BAND_SMEM / per_row);
   const int T = win_cap - 2 * B.omega;
@@ -345,6 +656,113 @@ mega_status mega_band_gat_fwd(const mega_band *band, const void *feat, int64_t l
   if (!ok) return fail(MEGA_ERR_UNSUPPORTED, "band kernel shape");
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? MEGA_OK : fail(MEGA_ERR_CUDA, std::string("band kernels: ") + cudaGetErrorString(e));
+}
+
+}  // extern "C"
+
+namespace mega {
+namespace {
+// shared shape checks of the band entry points -> V (vectors per lane) or -1
+int band_shape(int heads, int head_dim, mega_dtype dtype) {
+  if (dtype != MEGA_F32 && dtype != MEGA_BF16) return -1;
+  if (heads != 1 && heads != 2 && heads != 4 && heads != 8) return -1;
+  const int D = heads * head_dim, epv = dtype == MEGA_BF16 ? 8 : 4;
+  if (head_dim % epv || D % (32 * epv)) return -1;
+  const int V = D / (32 * epv);
+  if (V != 1 && V != 2 && V != 4) return -1;
+  const int lph = head_dim / epv;
+  if (lph > 32 ? (lph % 32 || V % (lph / 32)) : (32 % lph)) return -1;
+  return V;
+}
+}  // namespace
+}  // namespace mega
+
+extern "C" {
+
+mega_status mega_band_gat_bwd(const mega_band *band, const void *feat, int64_t ldf, const float *attn_l,
+                              const float *attn_r, int heads, int head_dim, mega_dtype dtype, float negative_slope,
+                              const void *out, int64_t ldo, const void *grad_out, int64_t ldg, float *ctx,
+                              float *grad_feat, int64_t ldgf, float *grad_attn_l, float *grad_attn_r, void *ws,
+                              size_t ws_bytes, mega_stream_t stream) {
+  clear_error();
+  NvtxRange nvtx_("mega_band_gat_bwd");
+  int bdev = -1, dev = 0;
+  if (!band) return fail(MEGA_ERR_INVALID_ARGUMENT, "null band");
+  const BandDev *Bp = band_dev(band, bdev);
+  if (!Bp) return fail(MEGA_ERR_STATE, "band not bound (mega_band_bind_device)");
+  cudaGetDevice(&dev);
+  if (bdev != dev) return fail(MEGA_ERR_STATE, "band bound to another device");
+  int major = 0;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  if (major != 10) return fail(MEGA_ERR_UNSUPPORTED, "libmega.so kernels require an sm_100 (B200) device");
+  if (!feat || !attn_l || !attn_r || !out || !grad_out || !ctx || !grad_feat || !grad_attn_l || !grad_attn_r || !ws)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "null pointer");
+  const int V = band_shape(heads, head_dim, dtype);
+  if (V < 0) return fail(MEGA_ERR_UNSUPPORTED, "band kernels: rows of 32 x 1/2/4 16-byte vectors, heads 1/2/4/8");
+  const int D = heads * head_dim, esz = dtype == MEGA_BF16 ? 2 : 4;
+  if (ldf < D || ldo < D || ldg < D || ldgf < D || (ldf * esz) % 16 || (ldo * esz) % 16 || (ldg * esz) % 16 ||
+      (ldgf * 4) % 16)
+    return fail(MEGA_ERR_INVALID_ARGUMENT, "bad leading dimension");
+  const BandDev &B = *Bp;
+  const BandWs w = band_ws(B.L, B.n_cnt, B.n_slots, heads, D);
+  if (ws_bytes < w.total) return fail(MEGA_ERR_OUT_OF_MEMORY, "band workspace too small");
+  // window: g rows + (el, lse, Dlt) + node id + masks + cptr per window entry
+  const size_t per_row = (size_t)D * esz + 12 * heads + 4 + 16 + 4;
+  const int win_cap = (int)((kern::BAND_SMEM - 64) / per_row);
+  const int T = win_cap - 1 - 2 * B.omega;
+  if (T < 8) return fail(MEGA_ERR_UNSUPPORTED, "band kernel: window + 2 omega rows do not fit in shared memory");
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t plane = B.n * heads;
+  kern::BandArgs a{};
+  a.B = B;
+  a.feat = feat; a.ldf = ldf; a.el = ctx; a.er = ctx + plane; a.lse = ctx + 2 * plane;
+  a.dlt = ctx + 3 * plane; a.der = ctx + 4 * plane;
+  a.slope = negative_slope; a.out = const_cast<void *>(out); a.ldo = ldo;
+  a.gout = grad_out; a.ldg = ldg; a.al = attn_l; a.ar = attn_r;
+  char *wb = static_cast<char *>(ws);
+  a.accD = reinterpret_cast<float *>(wb + w.accD);
+  a.derp = reinterpret_cast<float *>(wb + w.derp);
+  a.delp = reinterpret_cast<float *>(wb + w.delp);
+  a.dzb = reinterpret_cast<float *>(wb + w.dzb);
+  a.pdal = reinterpret_cast<double *>(wb + w.pdal);
+  a.pdar = reinterpret_cast<double *>(wb + w.pdar);
+  a.gfeat = grad_feat; a.ldgf = ldgf; a.gal = grad_attn_l; a.gar = grad_attn_r;
+  a.D = D; a.T = T; a.win_cap = win_cap;
+  int sms = 0;
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int64_t ntiles = (B.L + T - 1) / T;
+  const int node_blocks = (int)std::max<int64_t>(1, std::min<int64_t>((B.n + kern::BW - 1) / kern::BW,
+                                                                        std::min(2 * sms, kBandMaxNodeBlocks)));
+  bool ok = false;
+  auto go = [&](auto dk, auto sk, auto delk, auto nk) {
+    dk<<<(int)std::min<int64_t>((B.n + kern::BW - 1) / kern::BW, 8 * (int64_t)sms), kern::BW * 32, 0, st>>>(a);
+    cudaFuncSetAttribute(sk, cudaFuncAttributeMaxDynamicSharedMemorySize, kern::BAND_SMEM);
+    if (B.L > 0) sk<<<(int)std::max<int64_t>(1, std::min<int64_t>(ntiles, 2 * (int64_t)sms)), kern::BW * 32, kern::BAND_SMEM, st>>>(a);
+    delk<<<(int)std::max<int64_t>(1, std::min<int64_t>((B.L * heads + 255) / 256, 8 * (int64_t)sms)), 256, 0, st>>>(a);
+    nk<<<node_blocks, kern::BW * 32, 0, st>>>(a);
+    kern::band_param_kernel<<<(2 * D + 255) / 256, 256, 0, st>>>(a, node_blocks);
+    ok = true;
+  };
+  auto by_h = [&](auto tag_t, auto v_c) {
+    using TT = decltype(tag_t);
+    constexpr int VV = decltype(v_c)::value;
+    switch (heads) {
+      case 1: go(kern::band_dlt_kernel<TT, VV, 1>, kern::band_src_kernel<TT, VV, 1>, kern::band_del_kernel<1>, kern::band_node_kernel<TT, VV, 1>); break;
+      case 2: go(kern::band_dlt_kernel<TT, VV, 2>, kern::band_src_kernel<TT, VV, 2>, kern::band_del_kernel<2>, kern::band_node_kernel<TT, VV, 2>); break;
+      case 4: go(kern::band_dlt_kernel<TT, VV, 4>, kern::band_src_kernel<TT, VV, 4>, kern::band_del_kernel<4>, kern::band_node_kernel<TT, VV, 4>); break;
+      default: go(kern::band_dlt_kernel<TT, VV, 8>, kern::band_src_kernel<TT, VV, 8>, kern::band_del_kernel<8>, kern::band_node_kernel<TT, VV, 8>); break;
+    }
+  };
+  auto by_v = [&](auto tag_t) {
+    if (V == 1) by_h(tag_t, std::integral_constant<int, 1>());
+    else if (V == 2) by_h(tag_t, std::integral_constant<int, 2>());
+    else by_h(tag_t, std::integral_constant<int, 4>());
+  };
+  if (dtype == MEGA_BF16) by_v(__nv_bfloat16());
+  else by_v(float());
+  if (!ok) return fail(MEGA_ERR_UNSUPPORTED, "band kernel shape");
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? MEGA_OK : fail(MEGA_ERR_CUDA, std::string("band backward kernels: ") + cudaGetErrorString(e));
 }
 
 }  // extern "C"

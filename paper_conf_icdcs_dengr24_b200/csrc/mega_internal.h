@@ -75,7 +75,9 @@ struct BandDev {
   const uint16_t *cnt = nullptr;               // multiplicities (lmask bits, rmask bits, self-loops)
   const int32_t *slot = nullptr;               // [L] partial slot or -1
   const int32_t *merges = nullptr;             // [n_merges][3] (node, first slot, count)
-  int64_t L = 0, n = 0;
+  const int32_t *app_ptr = nullptr;            // [n+1] appearances of each node, in order
+  const int32_t *app_idx = nullptr;            // [L]
+  int64_t L = 0, n = 0, n_cnt = 0;
   int32_t omega = 0, n_merges = 0, n_slots = 0;
 };
 

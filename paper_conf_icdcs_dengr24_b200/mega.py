@@ -129,6 +129,8 @@ def lib():
             "mega_band_gat_workspace_bytes": (S, [P, _c.c_int, _c.c_int, S, P]),
             "mega_band_gat_fwd": (S, [P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, _c.c_uint32, P, I64, P, P,
                                       _c.c_size_t, P]),
+            "mega_band_gat_bwd": (S, [P, P, I64, P, P, _c.c_int, _c.c_int, S, _c.c_float, P, I64, P, I64, P, P, I64,
+                                      P, P, P, _c.c_size_t, P]),
             "mega_gt_fwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, _c.c_size_t, P]),
             "mega_gt_workspace_bytes": (S, [P, _c.c_int32, _c.c_int, _c.c_int, S, P]),
             "mega_gt_bwd": (S, [P, _c.c_int32, P, P, P, I64, _c.c_int, _c.c_int, S, P, I64, P, P, I64, P, P, P, I64,
@@ -536,3 +538,13 @@ def mega_band_gat_fwd(band: Band, feat, attn_l, attn_r, heads, head_dim, out, ct
     _check(lib().mega_band_gat_fwd(band.handle, _ptr(feat), feat.stride(0), _ptr(attn_l), _ptr(attn_r), heads,
                                    head_dim, dt, negative_slope, flags, _ptr(out), out.stride(0), _ptr(ctx), _ptr(ws),
                                    ws.numel() * ws.element_size(), _stream(stream)))
+
+
+def mega_band_gat_bwd(band: Band, feat, attn_l, attn_r, heads, head_dim, out, grad_out, ctx, grad_feat, grad_attn_l,
+                      grad_attn_r, ws, negative_slope=SLOPE, stream=None):
+    dt = _dtype_code(feat)
+    _check(lib().mega_band_gat_bwd(band.handle, _ptr(feat), feat.stride(0), _ptr(attn_l), _ptr(attn_r), heads,
+                                   head_dim, dt, negative_slope, _ptr(out), out.stride(0), _ptr(grad_out),
+                                   grad_out.stride(0), _ptr(ctx), _ptr(grad_feat), grad_feat.stride(0),
+                                   _ptr(grad_attn_l), _ptr(grad_attn_r), _ptr(ws), ws.numel() * ws.element_size(),
+                                   _stream(stream)))

@@ -1,4 +1,4 @@
-"""NEXT-2 measurement: GAT forward over the faithful path-band layout (mega_band_gat_fwd)
+"""NEXT-2 measurement: GAT forward and backward over the faithful path-band layout
 next to the exact-layout forward (mega_gat_fwd over mega_preprocess's layout) on the
 same graph, features and parameters; CUDA events, 10 calls after warm-up.  Prints one
 JSON line per config with |P| / n, the band's bytes, and both forward times.
@@ -66,6 +66,10 @@ def main():
         ws = torch.empty(max(M.mega_band_gat_workspace_bytes(band, H, F, M._dtype_code(Wh)), 256), dtype=torch.uint8,
                          device="cuda")
         ms_band = timed(lambda: M.mega_band_gat_fwd(band, Wh, a_l, a_r, H, F, out, ctx, ws))
+        g = torch.tensor(rng.standard_normal((n, D)).astype(np.float32), device="cuda").to(tdt)
+        gf = torch.empty(n, D, dtype=torch.float32, device="cuda")
+        gal, gar = torch.empty(D, device="cuda"), torch.empty(D, device="cuda")
+        ms_band_bwd = timed(lambda: M.mega_band_gat_bwd(band, Wh, a_l, a_r, H, F, out, g, ctx, gf, gal, gar, ws))
         # the exact layout's forward on the same graph (features permuted into its order)
         lay = M.mega_preprocess(ip, ix)
         lay.bind(0)
@@ -76,6 +80,11 @@ def main():
         fw, _ = M.mega_gat_workspace_bytes(lay, 0, H, F, M._dtype_code(Wn))
         ws2 = torch.empty(max(fw, 256), dtype=torch.uint8, device="cuda")
         ms_csr = timed(lambda: M.mega_gat_fwd(lay, 0, Wn, a_l, a_r, H, F, out2, ctx2, ws2))
+        _, bw = M.mega_gat_workspace_bytes(lay, 0, H, F, M._dtype_code(Wn))
+        wsb = torch.empty(max(bw, 256), dtype=torch.uint8, device="cuda")
+        gn = g[perm].contiguous()
+        gf2 = torch.empty(n, D, dtype=torch.float32, device="cuda")
+        ms_csr_bwd = timed(lambda: M.mega_gat_bwd(lay, 0, Wn, a_l, a_r, H, F, out2, gn, ctx2, gf2, gal, gar, wsb))
         # both compute graph attention of the same multiset: compare (band in input order)
         inv = torch.empty_like(perm)
         inv[perm] = torch.arange(n, device="cuda")
@@ -89,6 +98,7 @@ def main():
                           "multi_appearance_nodes": int(v["num_merges"]), "partial_slots": int(v["num_slots"]),
                           "band_bytes": band_bytes, "csr_index_bytes": 4 * cfg.m, "build_s": tb,
                           "band_fwd_ms": ms_band, "layout_fwd_ms": ms_csr,
+                          "band_bwd_ms": ms_band_bwd, "layout_bwd_ms": ms_csr_bwd,
                           "band_edges_per_s": cfg.m / (ms_band * 1e-3), "layout_edges_per_s": cfg.m / (ms_csr * 1e-3),
                           "max_abs_diff_band_vs_layout": diff}), flush=True)
 

@@ -17,7 +17,7 @@ from tests import gpu_harness as hz
 pytestmark = pytest.mark.gpu
 
 
-def run_band(ip, ix, Wh, a_l, a_r, dtype, window):
+def run_band(ip, ix, Wh, a_l, a_r, dtype, window, g=None):
     n, H, F = Wh.shape
     band = M.mega_band_build(ip, ix, window=window)
     band.bind()
@@ -27,10 +27,19 @@ def run_band(ip, ix, Wh, a_l, a_r, dtype, window):
     ctx = torch.zeros(M.MEGA_CTX_PLANES, n, H, dtype=torch.float32, device="cuda")
     ws = torch.empty(max(M.mega_band_gat_workspace_bytes(band, H, F, M._dtype_code(feat)), 256), dtype=torch.uint8,
                      device="cuda")
-    M.mega_band_gat_fwd(band, feat, torch.tensor(a_l, device="cuda"), torch.tensor(a_r, device="cuda"), H, F, out,
-                        ctx, ws)
+    al_t, ar_t = torch.tensor(a_l, device="cuda"), torch.tensor(a_r, device="cuda")
+    M.mega_band_gat_fwd(band, feat, al_t, ar_t, H, F, out, ctx, ws)
+    res = {"out": out.float().cpu().numpy().reshape(n, H, F), "lse": ctx[2].cpu().numpy().copy()}
+    if g is not None:
+        gt = torch.tensor(g.reshape(n, H * F), device="cuda").to(tdt).contiguous()
+        gf = torch.empty(n, H * F, dtype=torch.float32, device="cuda")
+        gal = torch.empty(H * F, dtype=torch.float32, device="cuda")
+        gar = torch.empty_like(gal)
+        M.mega_band_gat_bwd(band, feat, al_t, ar_t, H, F, out, gt, ctx, gf, gal, gar, ws)
+        res.update({"grad_feat": gf.cpu().numpy().reshape(n, H, F), "grad_attn_l": gal.cpu().numpy(),
+                    "grad_attn_r": gar.cpu().numpy()})
     torch.cuda.synchronize()
-    return {"out": out.float().cpu().numpy().reshape(n, H, F), "lse": ctx[2].cpu().numpy()}, band.view()
+    return res, band.view()
 
 
 @pytest.mark.parametrize("dtype,H,F", [("fp32", 4, 32), ("fp32", 1, 128), ("bf16", 4, 64), ("bf16", 2, 256),
@@ -54,3 +63,31 @@ def test_band_batch_workload(cuda_device, name):
     got, v = run_band(ip, ix, Wh, a_l, a_r, "fp32", 0)
     ref = coracle.gat_forward(ip, ix, Wh.astype(np.float64), a_l, a_r)
     hz.check(got, ref, "fp32", keys=("out", "lse"))
+
+
+@pytest.mark.parametrize("dtype,H,F", [("fp32", 4, 32), ("fp32", 1, 128), ("bf16", 4, 64), ("bf16", 2, 256),
+                                       ("bf16", 8, 32), ("fp32", 2, 64)])
+@pytest.mark.parametrize("window", [1, 4, 16])
+def test_band_backward_random_multigraph(cuda_device, dtype, H, F, window):
+    """mega_band_gat_bwd against the fp64 graph-attention backward (the band is exact)."""
+    ip, ix = synth.random_multigraph(23, 500, 6000, undirected=False, isolated=12)
+    n = len(ip) - 1
+    Wh, a_l, a_r, g = hz.inputs(11, n, H, F, dtype == "bf16")
+    got, v = run_band(ip, ix, Wh, a_l, a_r, dtype, window, g=g)
+    f = coracle.gat_forward(ip, ix, Wh.astype(np.float64), a_l, a_r)
+    b = coracle.gat_backward(ip, ix, Wh.astype(np.float64), a_l, a_r, g.astype(np.float64), fwd=f)
+    ref = {"out": f["out"], "lse": f["lse"], "grad_feat": b["grad_feat"], "grad_attn_l": b["grad_attn_l"].reshape(-1),
+           "grad_attn_r": b["grad_attn_r"].reshape(-1)}
+    hz.check(got, ref, dtype, graph=(ip, ix, Wh.astype(np.float64), a_l, a_r, g.astype(np.float64)))
+
+
+def test_band_backward_batch(cuda_device):
+    cfg = synth.get_config("zinc-b64")
+    ip, ix, _ = synth.make_graph(cfg)
+    Wh, a_l, a_r, g = hz.inputs(5, cfg.n, cfg.heads, cfg.head_dim, False)
+    got, _ = run_band(ip, ix, Wh, a_l, a_r, "fp32", 0, g=g)
+    f = coracle.gat_forward(ip, ix, Wh.astype(np.float64), a_l, a_r)
+    b = coracle.gat_backward(ip, ix, Wh.astype(np.float64), a_l, a_r, g.astype(np.float64), fwd=f)
+    ref = {"out": f["out"], "lse": f["lse"], "grad_feat": b["grad_feat"], "grad_attn_l": b["grad_attn_l"].reshape(-1),
+           "grad_attn_r": b["grad_attn_r"].reshape(-1)}
+    hz.check(got, ref, "fp32")
