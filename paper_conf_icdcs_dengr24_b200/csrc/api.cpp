@@ -27,6 +27,7 @@ static size_t align_up(size_t x) { return (x + kAlign - 1) / kAlign * kAlign; }
 std::vector<int32_t> make_chunks(const std::vector<int32_t> &items, int q, int cap) {
   std::vector<int32_t> c;
   const int64_t n = (int64_t)items.size() / 4;
+  if (n < kChunkMinItems) q = 0;   // small graphs: every item its own chunk (parallelism over latency)
   c.reserve(n / 4 + 2);
   c.push_back(0);
   int64_t cost = 0, cnt = 0;

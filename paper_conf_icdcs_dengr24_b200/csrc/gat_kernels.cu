@@ -1425,6 +1425,11 @@ bool lp_partial_mode() {
   }
   return v != 0;
 }
+// Claiming pays once a launch has many rounds of chunks to hand out: with few (the paper's small
+// batches, ~50 chunks) every group takes at most a chunk or two, the warps cannot drift apart, and the
+// counter reset plus the claim -> bounds -> descriptor chain only add latency to a launch-bound step
+// (zinc-b64: 0.17 -> 0.27 ms/step with claiming everywhere).
+bool claim_pays(int64_t n_chunks, int dev) { return n_chunks >= 16 * 16 * (int64_t)dev_info(dev).sms; }
 // MEGA_SCHED_DYN=0: static striding over the chunks instead of claiming them (ablation)
 bool sched_dynamic() {
   static int v = -1;
@@ -1637,7 +1642,7 @@ mega_status mega_gat_fwd(const mega_layout *L, int32_t part, const void *feat, i
   a.ws_acc = reinterpret_cast<float *>(wb + w.acc);
   a.st_hint = st_hint_mode();
   a.ctr = nullptr;
-  if (sched_dynamic()) {
+  if (sched_dynamic() && claim_pays(P.dev.fchunk ? P.dev.n_fchunks : P.dev.n_fwd_items, dev)) {
     a.ctr = reinterpret_cast<int *>(wb + w.ctr);
     cudaError_t ce = cudaMemsetAsync(a.ctr, 0, kCtrs * 4, st);
     if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));
@@ -1698,7 +1703,8 @@ mega_status mega_gat_bwd(const mega_layout *L, int32_t part, const void *feat, i
   cudaStream_t st = (cudaStream_t)stream;
   a.ctr = nullptr;
   const uint32_t ph = flags & (MEGA_BWD_PHASE_SRC | MEGA_BWD_PHASE_DST);
-  if (sched_dynamic() && (ph == 0 || (ph & MEGA_BWD_PHASE_SRC))) {
+  if (sched_dynamic() && (ph == 0 || (ph & MEGA_BWD_PHASE_SRC)) &&
+      claim_pays(P.dev.bchunk ? P.dev.n_bchunks : P.dev.n_bwd_items, dev)) {
     a.ctr = reinterpret_cast<int *>(wb + w.ctr);
     cudaError_t ce = cudaMemsetAsync(a.ctr, 0, kCtrs * 4, st);
     if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("counter reset: ") + cudaGetErrorString(ce));

@@ -145,7 +145,10 @@ cudaEvent_t comm_done_event(mega_comm *c);
 // stay within a few rounds of each other and the rows gathered concurrently stay in a narrow
 // window of the order (L2 reuse).  q = 0: one item per chunk (plain item striding).
 // MEGA_SCHED_Q / MEGA_SCHED_QB override q for the forward / source pass at bind time.
+// Parts with fewer than kChunkMinItems work items keep one item per chunk: grouping a small graph's
+// items would leave most of the grid idle (the paper's batches have ~1-5K items).
 constexpr int kChunkItemCost = 2, kChunkEdgesFwd = 256, kChunkEdgesBwd = 256, kChunkCapFwd = 8, kChunkCapBwd = 1 << 30;
+constexpr int64_t kChunkMinItems = 1 << 18;
 std::vector<int32_t> make_chunks(const std::vector<int32_t> &items, int q, int cap);
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]);
 // degree class: floor(2 log2 d) for d >= 1, clamped to 63; 0 for d = 0
