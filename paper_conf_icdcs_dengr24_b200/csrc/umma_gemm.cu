@@ -31,6 +31,7 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 
@@ -751,8 +752,20 @@ mega_status umma_project_dx(const void *gf, int64_t ldgf, int64_t rows, int in_d
   return launch_persistent<DX, 64, 32>(ta, tb, to, g, st);
 }
 
+// dW reductions of at most kUnsplitKb 64-row K blocks run in one CTA per output tile, writing grad_w
+// directly (no partials, no reduction launch).  MEGA_DW_UNSPLIT_KB: 8 (default) / 32 / 128 measured
+// 0.160 / 0.167 / 0.167 ms per zinc-b64 step and 0.206 / 0.210 / 0.289 for zinc-b256 (profiles/r02/dw_split/)
+int unsplit_kb() {
+  static int v = -1;
+  if (v < 0) {
+    const char *e = std::getenv("MEGA_DW_UNSPLIT_KB");
+    v = e ? std::atoi(e) : 8;
+  }
+  return v;
+}
 // workspace of umma_project_dw: split partials
 void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, size_t &bytes) {
+  const int kUnsplitKb = unsplit_kb();
   const int BN = std::min(D, 256);
   const int64_t mt = (in_dim + BM - 1) / BM, nt = (D + BN - 1) / BN;
   const int64_t kbt = (rows + BK - 1) / BK;
@@ -761,8 +774,8 @@ void umma_dw_plan(int64_t rows, int in_dim, int D, int &splits, int64_t &mpad, s
   // very short reductions (<= 512 rows) run unsplit, writing grad_w directly (one launch); longer
   // ones split: one CTA walking ~100 K blocks was measured slower (zinc-b256 step 0.26 -> 0.31 ms)
   // than a split GEMM plus its reduction
-  if (kbt <= 8) s = 1;
-  const int64_t per = std::max<int64_t>(kbt <= 8 ? kbt : 4, (kbt + s - 1) / s);   // >= 4 K blocks per split
+  if (kbt <= kUnsplitKb) s = 1;
+  const int64_t per = std::max<int64_t>(kbt <= kUnsplitKb ? kbt : 4, (kbt + s - 1) / s);   // >= 4 K blocks per split
   splits = (int)((kbt + per - 1) / per);   // every split non-empty
   mpad = mt * BM;
   bytes = splits == 1 ? 256 : (size_t)splits * (size_t)mpad * (size_t)D * 4;
