@@ -233,8 +233,9 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   const int64_t W = (int64_t)gridDim.x * WPB * GPW, gid = ((int64_t)blockIdx.x * WPB + w) * GPW + grp;
   const int32_t *fc = a.L.fchunk;
   const int64_t n_ch = fc ? a.L.n_fchunks : a.L.n_fwd_items;
-  auto row_load = [&](uint4 (&r)[V], uint32_t jj) {
-    const T *rp = featl + (jj & idm) * ldf;
+  // rows by element offset: stage_er replaces each staged source id by (id * ldf) once per edge
+  auto row_load = [&](uint4 (&r)[V], uint32_t off) {
+    const T *rp = featl + off;
 #pragma unroll
     for (int v = 0; v < V; ++v) r[v] = ldg16(rp + v * G * EPV);
   };
@@ -267,9 +268,10 @@ __global__ void __launch_bounds__(TPB, FwdCfg<V, 0>::MINB) gat_fwd_pipe_kernel(c
   };
   // er of the staged chunk's sources
   auto stage_er = [&](int b, int4 itm, int bse) {
-    const uint32_t jj = (uint32_t)s_src[b][w][rb + gl];
-    cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)(jj & idm) * H);
+    const uint32_t jj = (uint32_t)s_src[b][w][rb + gl] & idm;
+    cp_async_h<HT>(&s_er[b][w][rb + gl][0], a.er + (int64_t)jj * H);
     cp_async_commit();
+    s_src[b][w][rb + gl] = (int)(jj * ldf);   // element offset of the row (n * ldf < 2^32, checked on the host)
   };
   // prologue: descriptor batches 0 and 1 staged, batch 2's bounds in registers, batch 3's chunk claimed
   int kb = 0, cnt_cur, cnt_nxt, b2, n2;
@@ -835,8 +837,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
     if (b * U < cnt) {
 #pragma unroll
       for (int u = 0; u < U; ++u) {
-        const uint32_t ii = (uint32_t)s_i[w][min(b * U + u, cnt - 1)];
-        const T *rp = goutl + (ii & idm) * ldg;
+        const T *rp = goutl + (uint32_t)s_i[w][min(b * U + u, cnt - 1)];   // element offset (see below)
         uint4 *dst = ring + (((b % NBF) * U + u) * V) * 32 + lane;
 #pragma unroll
         for (int v = 0; v < V; ++v) cp_async16_plain(dst + v * 32, rp + v * G * EPV);
@@ -896,7 +897,7 @@ __global__ void __launch_bounds__(TPB, 2) gat_bwd_src_ring_kernel(const BwdArgs 
       load_h<HT>(a.el + gi * H, H, eli);
       load_h<HT>(a.lse + gi * H, H, lsei);
       load_h<HT>(a.dlt + gi * H, H, dli);
-      s_i[w][lane] = ir;
+      s_i[w][lane] = (int)(((uint32_t)ir & idm) * ldg);   // the g row's element offset (n * ldg < 2^32)
       __syncwarp();
 #pragma unroll
       for (int b = 0; b < NBF; ++b) issue(b, cnt);
