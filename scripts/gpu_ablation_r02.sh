@@ -1,6 +1,6 @@
 #!/bin/bash
 # Order ablation at HEAD: same kernels, different node orders.
-O=gpurun_out/r02/ablation
+O=${OUT:-gpurun_out/r02/ablation}
 mkdir -p $O
 export PYTHONPATH=$PWD
 for CFG in ${CFGS:-products reddit}; do
