@@ -10,15 +10,15 @@
 //     softmax state with shuffles; the first U source rows of the chunk are
 //     requested before the scores are evaluated (their addresses only need
 //     the source ids), later batches follow from shared memory;
-//   * L2 residency: rows of high-degree nodes ("hot": gathered often) are
-//     loaded with an L2 evict_last policy, the rest with evict_first, so the
-//     126 MB L2 keeps the rows that the power-law degree distribution makes
-//     most reused; the threshold comes from the layout's degree histogram;
+//   * L2 residency comes from the schedule, not from cache hints: work items
+//     are grouped into balanced chunks that the groups claim in layout order
+//     (DevPart::fchunk / bchunk, a workspace counter), so the rows gathered
+//     concurrently stay within about one round of chunks of the MEGA order
+//      and its L2 blocks; gathered rows use plain loads;
 //   * rows/sources longer than S edges were split by mega_preprocess into
 //     segments whose partial softmax states are merged in fixed order
-//     (no atomics anywhere on the value path);
-//   * items are taken grid-stride in path order, so co-resident groups work
-//     on neighbouring rows of the MEGA order.
+//     (no atomics anywhere on the value path; the claim counter only hands
+//     out work).
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
