@@ -44,6 +44,48 @@ struct Args {
   float *ws_m, *ws_l, *ws_acc;        // fwd slots (fwd_items)
   float *ws_dq;                       // dst-pass slots [fwd slots][D]
   float *ws_dk, *ws_dv;               // src-pass slots [bwd slots][D]
+  int *ctr;                           // claim counters (fwd, bwd dst, bwd src) or nullptr: static striding
+};
+
+// The GAT kernels' schedule: work items in balanced chunks (DevPart::fchunk / bchunk)
+// claimed in layout order from a counter, one chunk ahead; without a counter, chunks gid, gid + W, ...
+template <int G> struct ChunkSeq {
+  const int32_t *bc;
+  int64_t n_ch, ch, ch_next, it_end, stride;
+  int *ctr;
+  unsigned gmask;
+  int gl, rb;
+  __device__ int64_t claim(int64_t stat) {
+    if (!ctr) return stat;
+    int c = 0;
+    if (gl == 0) c = atomicAdd(ctr, 1);
+    return __shfl_sync(gmask, c, rb);
+  }
+  __device__ int64_t begin() {
+    if (ch >= n_ch) return -1;
+    it_end = bc ? __ldg(bc + ch + 1) : ch + 1;
+    return bc ? __ldg(bc + ch) : ch;
+  }
+  __device__ int64_t next(int64_t it) {
+    if (++it < it_end) return it;
+    ch = ch_next;
+    ch_next = claim(ch + stride);
+    return begin();
+  }
+  __device__ int64_t first(const int32_t *chunks, int64_t nchunks, int64_t nitems, int *c, int64_t gid, int64_t W,
+                           unsigned m, int l, int r) {
+    bc = chunks;
+    n_ch = chunks ? nchunks : nitems;
+    ctr = c;
+    gmask = m;
+    gl = l;
+    rb = r;
+    stride = W;
+    ch = claim(gid);
+    ch_next = claim(ch + stride);
+    it_end = 0;
+    return begin();
+  }
 };
 
 template <int G> __device__ __forceinline__ unsigned group_mask(int grp) {
@@ -62,7 +104,10 @@ __global__ void __launch_bounds__(TPB) gtb_fwd_kernel(const Args a) {
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / F;
-  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
+  ChunkSeq<G> seq;
+  for (int64_t it = seq.first(a.L.fchunk, a.L.n_fchunks, a.L.n_fwd_items, a.ctr ? a.ctr + 0 : nullptr,
+                              ((int64_t)blockIdx.x * WPB + w) * GPW + grp, stride, gmask, gl, grp * G);
+       it >= 0; it = seq.next(it)) {
     const int4 item = a.L.fwd_items[it];
     const int64_t row = a.L.row_begin + item.x;
     float q[V][EPV], acc[V][EPV], m[V], S[V];
@@ -182,7 +227,10 @@ __global__ void __launch_bounds__(TPB) gtb_bwd_dst_kernel(const Args a) {
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / F;
-  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_fwd_items; it += stride) {
+  ChunkSeq<G> seq;
+  for (int64_t it = seq.first(a.L.fchunk, a.L.n_fchunks, a.L.n_fwd_items, a.ctr ? a.ctr + 1 : nullptr,
+                              ((int64_t)blockIdx.x * WPB + w) * GPW + grp, stride, gmask, gl, grp * G);
+       it >= 0; it = seq.next(it)) {
     const int4 item = a.L.fwd_items[it];
     const int64_t lrow = item.x, row = a.L.row_begin + lrow;
     float q[V][EPV], g[V][EPV], dq[V][EPV], dl[1][V], lse[V];
@@ -270,7 +318,10 @@ __global__ void __launch_bounds__(TPB) gtb_bwd_src_kernel(const Args a) {
   int hv[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) hv[v] = ((v * G + gl) * EPV) / F;
-  for (int64_t it = ((int64_t)blockIdx.x * WPB + w) * GPW + grp; it < a.L.n_bwd_items; it += stride) {
+  ChunkSeq<G> seq;
+  for (int64_t it = seq.first(a.L.bchunk, a.L.n_bchunks, a.L.n_bwd_items, a.ctr ? a.ctr + 2 : nullptr,
+                              ((int64_t)blockIdx.x * WPB + w) * GPW + grp, stride, group_mask<G>(grp), gl, grp * G);
+       it >= 0; it = seq.next(it)) {
     const int4 item = a.L.bwd_items[it];
     const int64_t j = item.x;
     float dk[V][EPV], dv[V][EPV];
@@ -387,7 +438,7 @@ size_t gtb_workspace_bytes(const Part &P, int H, int D) {
   auto al = [](size_t x) { return (x + 255) / 256 * 256; };
   const size_t e = std::max<size_t>(1, P.src.size());
   const size_t fs = (size_t)std::max(1, P.n_fwd_slots), bs = (size_t)std::max(1, P.n_bwd_slots);
-  return 2 * al(e * H * 4) + al(fs * H * 4) * 2 + al(fs * D * 4) * 2 + al(bs * D * 4) * 2;
+  return 2 * al(e * H * 4) + al(fs * H * 4) * 2 + al(fs * D * 4) * 2 + al(bs * D * 4) * 2 + 256;   // + claim counters
 }
 
 mega_status gtb_run(const mega_layout *L, int32_t part, bool bwd, const void *q, const void *k, const void *v,
@@ -418,7 +469,15 @@ mega_status gtb_run(const mega_layout *L, int32_t part, bool bwd, const void *q,
   a.ws_acc = reinterpret_cast<float *>(w + off); off += al(fs * D * 4);
   a.ws_dq = reinterpret_cast<float *>(w + off); off += al(fs * D * 4);
   a.ws_dk = reinterpret_cast<float *>(w + off); off += al(bs * D * 4);
-  a.ws_dv = reinterpret_cast<float *>(w + off);
+  a.ws_dv = reinterpret_cast<float *>(w + off); off += al(bs * D * 4);
+  a.ctr = nullptr;
+  const int64_t nch = std::max<int64_t>(a.L.fchunk ? a.L.n_fchunks : a.L.n_fwd_items,
+                                        a.L.bchunk ? a.L.n_bchunks : a.L.n_bwd_items);
+  if (nch >= 16 * 16 * (int64_t)sms) {   // claiming pays with many rounds of chunks (as the GAT kernels)
+    a.ctr = reinterpret_cast<int *>(w + off);
+    cudaError_t ce = cudaMemsetAsync(a.ctr, 0, 3 * sizeof(int), st);
+    if (ce != cudaSuccess) return fail(MEGA_ERR_CUDA, std::string("GT counter reset: ") + cudaGetErrorString(ce));
+  }
   mega_status rc = MEGA_OK;
   const bool ok = gtb_dispatch(nv, [&](auto gg, auto vv) {
     constexpr int G = decltype(gg)::value, V = decltype(vv)::value;
