@@ -81,7 +81,11 @@ class ClockSampler:
             self.t.start()
         except OSError:
             self.proc = None
-        time.sleep(0.25)
+        t0 = time.time()   # the sampler must be live before the timed region starts
+        while self.proc is not None and not self.rows and time.time() - t0 < 3.0:
+            time.sleep(0.02)
+        self.skip = len(self.rows)   # samples taken before the timed region are not counted
+        self.after = False
         return self
 
     def _read(self):
@@ -89,6 +93,14 @@ class ClockSampler:
             self.rows.append([x.strip() for x in line.split(",")])
 
     def __exit__(self, *exc):
+        if self.proc and len(self.rows) <= self.skip:   # a region shorter than the 100 ms sampling period
+            try:
+                out = subprocess.run(["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits", "-i",
+                                      str(self.index)], capture_output=True, text=True, timeout=10).stdout
+                self.rows += [[x.strip() for x in ln.split(",")] for ln in out.splitlines() if ln.strip()]
+                self.after = True
+            except (OSError, subprocess.TimeoutExpired):
+                pass
         if self.proc:
             self.proc.terminate()
             try:
@@ -97,15 +109,20 @@ class ClockSampler:
                 self.proc.kill()
 
     def summary(self):
-        if not self.rows:
+        rows = self.rows[getattr(self, "skip", 0):]
+        if not rows:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.rows = rows
         sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
         mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
         names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
         reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 4 + i and "Active" in r[4 + i]
                           and "Not" not in r[4 + i]})
-        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": reasons, "samples": len(self.rows)}
+        out = {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+               "reasons": reasons, "samples": len(self.rows)}
+        if getattr(self, "after", False):
+            out["sampled"] = "right after the timed region (shorter than the 100 ms sampling period)"
+        return out
 
 
 def peaks():
