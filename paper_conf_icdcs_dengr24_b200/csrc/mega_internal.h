@@ -147,7 +147,7 @@ cudaEvent_t comm_done_event(mega_comm *c);
 // MEGA_SCHED_Q / MEGA_SCHED_QB override q for the forward / source pass at bind time.
 // Parts with fewer than kChunkMinItems work items keep one item per chunk: grouping a small graph's
 // items would leave most of the grid idle (the paper's batches have ~1-5K items).
-constexpr int kChunkItemCost = 2, kChunkEdgesFwd = 256, kChunkEdgesBwd = 256, kChunkCapFwd = 8, kChunkCapBwd = 1 << 30;
+constexpr int kChunkItemCost = 2, kChunkEdgesFwd = 128, kChunkEdgesBwd = 128, kChunkCapFwd = 8, kChunkCapBwd = 1 << 30;
 constexpr int64_t kChunkMinItems = 1 << 18;
 std::vector<int32_t> make_chunks(const std::vector<int32_t> &items, int q, int cap);
 size_t part_image_bytes(const mega_layout *L, int part, size_t offs[kImageArrays]);
